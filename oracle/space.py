@@ -1,0 +1,266 @@
+"""oracle.space — brute-force enumeration of the csTuner parameter space.
+
+TEST INFRASTRUCTURE ONLY (see oracle/__init__.py).  Plain nested loops in canonical field
+order (Table I row order; values ascending), every rule checked as soon as the
+fields it reads are fixed.  The C++ enumerator in libcst (csrc/space) must reproduce the
+count, the ordered tuple stream (FNV-1a-64) and rank/unrank bit-exactly.
+
+Space (readings Q14/Q15 of SURVEY.md §8(c)):
+
+  #   field          range                          note
+  1-3 TB_x,TB_y,TB_z p2[1,1024], p2[1,1024], p2[1,64] Table I
+  4   staging        {1 none, 2 smem ld/st, 3 TMA}  useShared {1,2} + B200 TMA
+  5   use_constant   {1,2}
+  6   use_streaming  {1,2}
+  7   SD             {1 x, 2 y, 3 z}                P:141; canonical 1 if streaming off
+  8   SB             p2[1, M_SD]                    P:142; canonical 1 if streaming off
+  9-11 UF_x,y,z      p2[1, M_d]
+  12-14 CM_x,y,z     p2[1, M_d]
+  15-17 BM_x,y,z     p2[1, M_d]
+  18  use_retiming   {1,2}
+  19  prefetch       {1 off, 2, 3, 4 stages}        usePrefetching {1,2} + depth
+
+Rules: paper R1 prod TB <= 1024; R2 SD=SB=1 when streaming off; R3 UF_SD <= SB when
+streaming on.  Ours (Q15): R4 prod TB >= 32; R5 T_d = TB_d*BM_d*CM_d <= E_d (E_d = M_d,
+E_SD = SB when streaming); R6 UF_d <= trip_d (trip_d = BM_d*CM_d; trip_SD = SB / T_SD when
+streaming); R7 prod(BM*CM) <= 16; R8 streaming => SD != 1; R9 prefetch > 1 => streaming;
+R10 modelled smem <= SMEM_LIMIT; R11 modelled registers <= 255; R12 TMA box: T_x even and
+every box extent <= 256.
+"""
+from __future__ import annotations
+
+import math
+
+FIELDS = ("tb_x", "tb_y", "tb_z", "staging", "use_constant", "use_streaming", "sd", "sb",
+          "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z", "bm_x", "bm_y", "bm_z",
+          "use_retiming", "prefetch")
+
+STAR, BOX, HYPTERM = 1, 2, 3
+SMEM_LIMIT = 227 * 1024 - 1024      # data bytes; 1 KiB kept for mbarriers / alignment
+REG_LIMIT = 255
+
+
+def p2(lo: int, hi: int):
+    v, out = 1, []
+    while v <= hi:
+        if v >= lo:
+            out.append(v)
+        v *= 2
+    return out
+
+
+def n_arrays(kind: int) -> int:
+    return 8 if kind == HYPTERM else 1
+
+
+def live_doubles_per_point(kind: int, r: int) -> int:
+    return {STAR: 2 * r + 2, BOX: 12, HYPTERM: 50}[kind]
+
+
+def retention(kind: int, r: int) -> int:
+    """Planes the gather (non-retimed) streaming path must keep after loading (T_SD == 1)."""
+    return 2 * r if kind == BOX else r
+
+
+def tiles(s: dict):
+    return [s["tb_x"] * s["bm_x"] * s["cm_x"], s["tb_y"] * s["bm_y"] * s["cm_y"],
+            s["tb_z"] * s["bm_z"] * s["cm_z"]]
+
+
+def plane_geometry(kind: int, r: int, s: dict):
+    """(in-plane elements P, ring planes NP) of the smem staging for a streaming setting;
+    (box elements, 1) for a non-streaming one."""
+    T = tiles(s)
+    if s["use_streaming"] == 1:
+        return (T[0] + 2 * r) * (T[1] + 2 * r) * (T[2] + 2 * r), 1
+    sd = s["sd"] - 1
+    a, b = [d for d in range(3) if d != sd]
+    P = (T[a] + 2 * r) * (T[b] + 2 * r)
+    D = s["prefetch"]
+    if T[sd] == 1:
+        NP = D + (0 if s["use_retiming"] == 2 else retention(kind, r))
+    else:
+        NP = D * T[sd] + 2 * r
+    return P, NP
+
+
+def smem_bytes(kind: int, r: int, s: dict) -> int:
+    if s["staging"] == 1:
+        return 0
+    P, NP = plane_geometry(kind, r, s)
+    plane = -(-(P * 8) // 128) * 128
+    return n_arrays(kind) * NP * plane
+
+
+def est_regs(kind: int, r: int, s: dict) -> int:
+    ppt = 1
+    for d in "xyz":
+        ppt *= s["bm_" + d] * s["cm_" + d]
+    nthr = s["tb_x"] * s["tb_y"] * s["tb_z"]
+    pf = 0
+    if s["staging"] == 2 and s["prefetch"] > 1:
+        P, _ = plane_geometry(kind, r, s)
+        T = tiles(s)
+        per_step = T[s["sd"] - 1] if s["use_streaming"] == 2 else 1
+        pf = (s["prefetch"] - 1) * -(-(n_arrays(kind) * P * per_step) // nthr)
+    return 32 + 2 * ppt * live_doubles_per_point(kind, r) + 2 * pf
+
+
+def tma_ok(r: int, s: dict) -> bool:
+    T = tiles(s)
+    if T[0] % 2:
+        return False
+    if s["use_streaming"] == 1:
+        ext = [t + 2 * r for t in T]
+    else:
+        sd = s["sd"] - 1
+        ext = [T[d] + 2 * r if d != sd else T[d] for d in range(3)]
+    return all(e <= 256 for e in ext)
+
+
+def check(kind: int, r: int, M, s: dict):
+    """Return None if valid else the name of the first failing rule (R1..R12)."""
+    tb = s["tb_x"] * s["tb_y"] * s["tb_z"]
+    if tb > 1024:
+        return "R1"
+    stream = s["use_streaming"] == 2
+    if not stream and (s["sd"] != 1 or s["sb"] != 1):
+        return "R2"
+    if stream and s["sd"] == 1:
+        return "R8"
+    if tb < 32:
+        return "R4"
+    T = tiles(s)
+    sd = s["sd"] - 1
+    for d in range(3):
+        E = s["sb"] if (stream and d == sd) else M[d]
+        if T[d] > E:
+            return "R5"
+    if stream and s["uf_" + "xyz"[sd]] > s["sb"]:
+        return "R3"
+    for d in range(3):
+        trip = s["sb"] // T[d] if (stream and d == sd) else s["bm_" + "xyz"[d]] * s["cm_" + "xyz"[d]]
+        if s["uf_" + "xyz"[d]] > trip:
+            return "R6"
+    ppt = 1
+    for d in "xyz":
+        ppt *= s["bm_" + d] * s["cm_" + d]
+    if ppt > 16:
+        return "R7"
+    if s["prefetch"] > 1 and not stream:
+        return "R9"
+    if smem_bytes(kind, r, s) > SMEM_LIMIT:
+        return "R10"
+    if est_regs(kind, r, s) > REG_LIMIT:
+        return "R11"
+    if s["staging"] == 3 and not tma_ok(r, s):
+        return "R12"
+    return None
+
+
+def enumerate_space(kind: int, r: int, M):
+    """Yield every valid setting (dict) in canonical order, by nested loops.  Rules that
+    only read already-fixed fields are checked early purely to prune; the final `check`
+    call decides validity."""
+    Mx, My, Mz = M
+    for tbx in p2(1, 1024):
+        if tbx > Mx:
+            continue
+        for tby in p2(1, 1024):
+            if tby > My or tbx * tby > 1024:
+                continue
+            for tbz in p2(1, 64):
+                if tbz > Mz or tbx * tby * tbz > 1024 or tbx * tby * tbz < 32:
+                    continue
+                for stg in (1, 2, 3):
+                    for uc in (1, 2):
+                        for st in (1, 2):
+                            for sd in (1, 2, 3):
+                                if st == 1 and sd != 1:
+                                    continue
+                                if st == 2 and sd == 1:
+                                    continue
+                                sbs = p2(1, M[sd - 1]) if st == 2 else [1]
+                                for sb in sbs:
+                                    yield from _inner(kind, r, M, dict(
+                                        tb_x=tbx, tb_y=tby, tb_z=tbz, staging=stg,
+                                        use_constant=uc, use_streaming=st, sd=sd, sb=sb))
+
+
+def _inner(kind, r, M, s):
+    """Valid completions of the outer prefix `s`.  The loops run CM/BM before UF so that
+    R7 can prune; the completions are then sorted into canonical (UF, CM, BM, ...) order.
+    The outer prefix fields precede every inner field, so this yields the global order."""
+    found = []
+    for cmx in p2(1, M[0]):
+        for cmy in p2(1, M[1]):
+            for cmz in p2(1, M[2]):
+                if cmx * cmy * cmz > 16:
+                    continue
+                for bmx in p2(1, M[0]):
+                    for bmy in p2(1, M[1]):
+                        for bmz in p2(1, M[2]):
+                            if cmx * cmy * cmz * bmx * bmy * bmz > 16:
+                                continue
+                            T = tiles(dict(s, bm_x=bmx, bm_y=bmy, bm_z=bmz, cm_x=cmx,
+                                           cm_y=cmy, cm_z=cmz))
+                            if any(T[d] > M[d] for d in range(3)):
+                                continue      # implied by R5 (SB <= M_SD)
+                            # UF_d <= max(BM_d*CM_d, SB) is implied by R3/R6 (prune only)
+                            bnd = [bmx * cmx, bmy * cmy, bmz * cmz]
+                            if s["use_streaming"] == 2:
+                                bnd[s["sd"] - 1] = s["sb"]
+                            for ufx in p2(1, bnd[0]):
+                                for ufy in p2(1, bnd[1]):
+                                    for ufz in p2(1, bnd[2]):
+                                        for ret in (1, 2):
+                                            for pf in (1, 2, 3, 4):
+                                                t = dict(s, uf_x=ufx, uf_y=ufy, uf_z=ufz,
+                                                         cm_x=cmx, cm_y=cmy, cm_z=cmz,
+                                                         bm_x=bmx, bm_y=bmy, bm_z=bmz,
+                                                         use_retiming=ret, prefetch=pf)
+                                                if check(kind, r, M, t) is None:
+                                                    found.append(t)
+    found.sort(key=as_tuple)
+    yield from found
+
+
+def as_tuple(s: dict):
+    return tuple(s[f] for f in FIELDS)
+
+
+FNV_OFFSET = 0xCBF29CE484222325
+FNV_PRIME = 0x100000001B3
+
+
+def fnv1a64_stream(settings) -> tuple[int, int]:
+    """(count, FNV-1a-64 over the little-endian int32 encoding of every tuple in order)."""
+    h, n = FNV_OFFSET, 0
+    for s in settings:
+        for v in as_tuple(s):
+            for byte in int(v).to_bytes(4, "little", signed=True):
+                h ^= byte
+                h = (h * FNV_PRIME) & 0xFFFFFFFFFFFFFFFF
+        n += 1
+    return n, h
+
+
+def literal_table1_count(M) -> int:
+    """Size of the literal Table I space (useShared, usePrefetching in {1,2}) under the
+    paper's explicit rules only (R1, R2, R3), by closed-form product counting."""
+    Mx, My, Mz = M
+    nlog = lambda m: int(math.floor(math.log2(m))) + 1
+    ntb = sum(1 for a in p2(1, 1024) for b in p2(1, 1024) for c in p2(1, 64) if a * b * c <= 1024)
+    per_dim = [nlog(m) for m in M]
+    uf_cm_bm_all = 1
+    for n in per_dim:
+        uf_cm_bm_all *= n ** 3
+    base = ntb * 2 * 2 * 2 * 2          # TB, useShared, useConstant, useRetiming, usePrefetching
+    off = uf_cm_bm_all                  # streaming off: SD = SB = 1 canonical
+    on = 0
+    for sd in range(3):
+        for sb in p2(1, M[sd]):
+            nuf_sd = sum(1 for u in p2(1, M[sd]) if u <= sb)
+            rest = uf_cm_bm_all // per_dim[sd] * nuf_sd
+            on += rest
+    return base * (off + on)
