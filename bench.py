@@ -1,0 +1,318 @@
+"""bench.py — GStencil/s of the complex-stencil sweep on B200 (BASELINE.json configs[1]).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl cst|reference]
+
+N=1 workload: order-4 25-point star (FD Laplacian, weights /5040), 512^3 FP64 interior,
+halo 4, the tuned setting from tuned/star25_512.json (cst_tune output; the default setting
+if absent).  A step = one sweep (one kernel launch) over inputs resident in HBM; the two
+1.18 GB arrays exceed the 126 MB L2, so no flush is needed between steps.
+N>1 (torchrun, one rank per GPU): weak scaling of the z-slab decomposition — every rank owns
+a 512^3 slab of a (512*N) x 512 x 512 grid and exchanges 4-plane halos with its neighbours
+(cst_dist_sweep, NCCL) every step.  value = all ranks' points / max-over-ranks time.
+
+Extra keys: roofline (dominant kernel = the sweep), cpu_baseline (the oracle on a bounded
+sample, rank 0 at N=1), e2e (cst_sweep_host: H2D + sweep + D2H through the C ABI), clocks
+(nvidia-smi during the timed region), gpu_launches.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+BASE = json.load(open(os.path.join(ROOT, "BASELINE.json")))
+METRIC = BASE["metric"]
+UNIT = "GStencil/s"
+N = 512
+R = 4
+SEED = 2
+D2_R4 = [-9, 128, -1008, 8064, -14350, 8064, -1008, 128, -9]
+
+
+def star_coeffs():
+    w = [v / 5040.0 for v in D2_R4]
+    side = w[:R] + w[R + 1:]
+    return [3 * w[R]] + side * 3
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+def load_setting(C, h):
+    p = os.path.join(ROOT, "tuned", "star25_512.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        s = C.cst_setting.from_dict(d["setting"])
+        C.cst_setting_check(h, s)
+        return s, "tuned/star25_512.json"
+    return C.cst_setting_default(h), "cst_setting_default"
+
+
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.FIELDS,
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        sm = [float(r[0]) for r in self.rows if len(r) >= 7 and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) >= 7 and r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            if len(r) < 7:
+                continue
+            for n, v in zip(names, r[3:7]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def ncu_traffic():
+    p = os.path.join(ROOT, "profiles", "ncu_star25_512.json")
+    if os.path.exists(p):
+        try:
+            d = json.load(open(p))
+            return d.get("dram_bytes_per_launch")
+        except Exception:
+            return None
+    return None
+
+
+def cpu_baseline(target_s: float = 10.0):
+    """The oracle, as it stands, on a bounded sample of the same workload: a 512 x 512 x 16
+    slab of the 512^3 star25 grid swept repeatedly until >= target_s seconds."""
+    import numpy as np
+
+    import cstgen
+    from oracle import stencil as ost
+    nz_s = 16
+    L = cstgen.make_layout(N, N, nz_s, R)
+    u = cstgen.fill(L, SEED, 0)
+    v = np.full(L.numel, np.nan)
+    c = ost.star_laplacian_coeffs(R)
+    cores = os.cpu_count() or 1
+    pts, t0 = 0, time.perf_counter()
+    while True:
+        ost.sweep(1, R, c, L, [u], [v], nthreads=cores)
+        pts += N * N * nz_s
+        el = time.perf_counter() - t0
+        if el >= target_s:
+            break
+    return {"value": pts / el / 1e9, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{N}x{N}x{nz_s} slab of the 512^3 star25 workload, swept "
+                      f"{pts // (N * N * nz_s)} times ({el:.1f} s, {cores} OpenMP threads)"}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the oracle (CPU) timed on the box's host cores, rank 0 only."""
+    if rank != 0:
+        return
+    import numpy as np
+
+    import cstgen
+    from oracle import stencil as ost
+    nz_s = 8
+    L = cstgen.make_layout(N, N, nz_s, R)
+    u = cstgen.fill(L, SEED, 0)
+    v = np.full(L.numel, np.nan)
+    c = ost.star_laplacian_coeffs(R)
+    cores = os.cpu_count() or 1
+    for _ in range(args.warmup):
+        ost.sweep(1, R, c, L, [u], [v], nthreads=cores)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        ost.sweep(1, R, c, L, [u], [v], nthreads=cores)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    pts = N * N * nz_s * args.steps
+    val = pts / tot / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (cstgen splitmix64 U[-1,1), seed 2)",
+            "config": {"workload": "star25 (order-4 25-point star FD Laplacian) 512^3 FP64 "
+                                   "(BASELINE configs[1]); each step a bounded 512x512x8 slab"},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": f"{N}x{N}x{nz_s} slab per step"},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="cst", choices=["cst", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    args = ap.parse_args()
+    assert args.warmup >= 3 or args.impl == "reference" or True
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_cluster_sunlyjldlq21_b200 import cst as C
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    grid = C.make_grid(N, N, N, R)
+    h = C.cst_stencil_create(C.CST_STAR, R, star_coeffs(), grid, local)
+    s, s_src = load_setting(C, h)
+    u = torch.empty(grid.numel, dtype=torch.float64, device="cuda")
+    v = torch.empty(grid.numel, dtype=torch.float64, device="cuda")
+    stream = torch.cuda.current_stream()
+    z0 = rank * N
+    C.cst_fill_uniform(grid, u.data_ptr(), SEED, 0, N, N, z0, float("nan"), stream.cuda_stream)
+    C.cst_fill_uniform(grid, v.data_ptr(), SEED, 0, N, N, z0, float("nan"), stream.cuda_stream)
+    dist_h = None
+    if world > 1:
+        uid = C.cst_dist_nccl_unique_id() if rank == 0 else None
+        obj = [uid]
+        dist.broadcast_object_list(obj, src=0)
+        dist_h = C.cst_dist_create(h, world, rank, obj[0])
+
+    def step():
+        if dist_h is not None:
+            C.cst_dist_sweep(dist_h, s, [u.data_ptr()], [v.data_ptr()], 1, stream.cuda_stream)
+        else:
+            C.cst_sweep(h, s, [u.data_ptr()], [v.data_ptr()], 1, stream.cuda_stream)
+
+    for _ in range(max(args.warmup, 3)):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches = 0
+    evs[0].record(stream)
+    for i in range(args.steps):
+        step()
+        launches += C.cst_last_launch_count(h) if dist_h is None else 0
+        evs[i + 1].record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    per = [evs[i].elapsed_time(evs[i + 1]) for i in range(args.steps)]
+    total_ms = evs[0].elapsed_time(evs[-1])
+    if world > 1:
+        t = torch.tensor([total_ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    ms_step = total_ms / args.steps
+    pts = N * N * N
+    value = pts * world / (ms_step * 1e-3) / 1e9
+
+    peak, peak_src = measured_peaks()
+    avg_launch_ms = statistics.mean(per)
+    alg_bytes = 16 * pts                           # read u once + write out once (FP64)
+    achieved = alg_bytes / (avg_launch_ms * 1e-3) / 1e9
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+            "frac": achieved / peak, "traffic": ncu_traffic(), "peak_source": peak_src,
+            "alg_bytes_per_launch": alg_bytes, "kernel": "cst_kernel (star25 sweep)",
+            "avg_launch_ms": avg_launch_ms, "frac_of_nominal_8TBs": achieved / 8000.0}
+
+    # ---- e2e: the same metric through cst_sweep_host (pinned host buffers, H2D + D2H)
+    e2e = None
+    if rank == 0 and world == 1 and args.e2e_steps > 0:
+        hu = torch.empty(grid.numel, dtype=torch.float64).pin_memory()
+        hv = torch.empty(grid.numel, dtype=torch.float64).pin_memory()
+        hu.copy_(u.cpu())
+        C.cst_sweep_host(h, s, [hu.data_ptr()], [hv.data_ptr()], 1)     # warm-up / alloc
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            C.cst_sweep_host(h, s, [hu.data_ptr()], [hv.data_ptr()], 1)
+        el = (time.perf_counter() - t0) / args.e2e_steps
+        e2e = {"value": pts / el / 1e9, "unit": UNIT, "h2d_bytes_per_step": grid.numel * 8,
+               "d2h_bytes_per_step": pts * 8, "ms_per_step": el * 1e3,
+               "steps": args.e2e_steps, "api": "cst_sweep_host"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline()
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+                "steps": args.steps, "warmup": max(args.warmup, 3), "ms_per_step": ms_step,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic (cstgen splitmix64 U[-1,1), seed 2, device generator)",
+                "config": {"workload": "star25: order-4 25-point star (FD Laplacian /5040), "
+                                       "512^3 FP64 interior per GPU (BASELINE configs[1])"
+                                       + ("; z-slab weak scaling, NCCL halo exchange" if world > 1 else ""),
+                           "grid": [N, N, N * world], "halo": R,
+                           "setting": s.as_dict(), "setting_source": s_src,
+                           "l2": "inputs larger than L2 (2 x %.2f GB per GPU), no flush"
+                                 % (grid.numel * 8 / 1e9),
+                           "parallelism": f"z-slab x{world}" if world > 1 else "single GPU"},
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
+                "gpu_launches": launches if dist_h is None else None,
+                "per_step_ms": {"min": min(per), "median": statistics.median(per), "max": max(per)}}
+        print(json.dumps(line), flush=True)
+    if dist_h is not None:
+        C.cst_dist_destroy(dist_h)
+    C.cst_stencil_destroy(h)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

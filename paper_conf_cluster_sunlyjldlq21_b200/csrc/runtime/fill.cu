@@ -1,0 +1,46 @@
+// fill.cu — device twin of the cstgen input generator (cstgen/cst_gen.h).
+// Fills the logical padded region of a grid with U[-1,1) values keyed by the GLOBAL padded
+// index, so any rank can generate its own slab (and its halo) without the global array.
+#include "../../../cstgen/cst_gen.h"
+#include "internal.h"
+
+namespace {
+
+__global__ void fill_kernel(double* __restrict__ dst, int64_t nx, int64_t ny, int64_t nz,
+                            int64_t halo, int64_t lead_x, int64_t pitch_x, int64_t pitch_y,
+                            uint64_t key, int64_t nxg, int64_t nyg, int64_t z0, double pad) {
+  const int64_t row = blockIdx.x;  // (z, y) row of the allocation
+  const int64_t planes = nz + 2 * halo;
+  const int64_t zz = row / pitch_y, yy = row % pitch_y;
+  if (zz >= planes) return;
+  const int64_t y = yy - halo, z = zz - halo;
+  double* r = dst + row * pitch_x;
+  const bool row_in = y < ny + halo;
+  for (int64_t xx = threadIdx.x; xx < pitch_x; xx += blockDim.x) {
+    const int64_t x = xx - lead_x;
+    double v = pad;
+    if (row_in && x >= -halo && x < nx + halo)
+      v = cstgen_value(key, cstgen_index(nxg, nyg, halo, x, y, z + z0));
+    r[xx] = v;
+  }
+}
+
+}  // namespace
+
+extern "C" cst_status cst_fill_uniform(const cst_grid* g, double* dev, uint64_t seed,
+                                       uint64_t array_id, int64_t nx_global, int64_t ny_global,
+                                       int64_t z0, double pad_value, void* stream) {
+  if (!g || !dev) return cst::fail(CST_E_INVALID, "null argument");
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) {
+    cudaGetLastError();
+    return cst::fail(CST_E_CUDA, "no CUDA device available (libcst has no CPU fallback)");
+  }
+  const int64_t rows = (g->nz + 2 * (int64_t)g->halo) * g->pitch_y;
+  if (rows > 0x7fffffffLL) return cst::fail(CST_E_UNSUPPORTED, "grid too large for fill");
+  fill_kernel<<<(unsigned)rows, 256, 0, (cudaStream_t)stream>>>(
+      dev, g->nx, g->ny, g->nz, g->halo, g->lead_x, g->pitch_x, g->pitch_y,
+      cstgen_key(seed, array_id), nx_global, ny_global, z0, pad_value);
+  CST_CUDA(cudaGetLastError());
+  return CST_OK;
+}

@@ -1,0 +1,138 @@
+// internal.h — host-side internals of libcst (not part of the C ABI).
+#pragma once
+
+#include <cuda.h>
+#include <cudaTypedefs.h>
+#include <cuda_runtime.h>
+
+#include <array>
+#include <cstdint>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../../include/cst.h"
+#include "../kernels/cst_params.h"
+
+namespace cst {
+
+// ------------------------------------------------------------------ error handling
+void set_error(const std::string& msg);
+cst_status fail(cst_status s, const std::string& msg);
+#define CST_CUDA(call)                                                              \
+  do {                                                                              \
+    cudaError_t e_ = (call);                                                        \
+    if (e_ != cudaSuccess)                                                          \
+      return ::cst::fail(CST_E_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+
+// ------------------------------------------------------------------ settings
+// The 19 fields in canonical order (Table I row order).
+enum Field {
+  F_TBX, F_TBY, F_TBZ, F_STAGING, F_CONST, F_STREAM, F_SD, F_SB, F_UFX, F_UFY, F_UFZ,
+  F_CMX, F_CMY, F_CMZ, F_BMX, F_BMY, F_BMZ, F_RET, F_PF, F_COUNT
+};
+using Tuple = std::array<int32_t, F_COUNT>;
+Tuple to_tuple(const cst_setting& s);
+cst_setting from_tuple(const Tuple& t);
+std::string setting_key(const cst_setting& s);
+extern const char* const kFieldNames[F_COUNT];
+
+struct StencilInfo {
+  int kind, r;
+  int64_t M[3];  // nx, ny, nz
+};
+
+// Rule check (R1..R12).  Returns nullptr if valid else the rule id.
+const char* check_rules(const StencilInfo& st, const Tuple& t);
+int64_t model_smem_bytes(int kind, int r, const Tuple& t);
+int64_t model_regs(int kind, int r, const Tuple& t);
+// Dynamic shared memory the kernel variant actually uses (<= model for fast paths).
+int64_t kernel_smem_bytes(int kind, int r, const Tuple& t);
+
+// ------------------------------------------------------------------ space
+class Space {
+ public:
+  explicit Space(const StencilInfo& st);
+  uint64_t count() const { return total_; }
+  bool at(uint64_t rank, Tuple* out) const;
+  bool rank(const Tuple& t, uint64_t* out) const;
+
+ private:
+  struct Core {  // (CM x3, BM x3, ret, pf) and its per-dim UF bounds (counts)
+    int32_t cm[3], bm[3], ret, pf;
+    int32_t nuf[3];
+  };
+  struct Prefix {
+    int32_t v[8];       // TBx TBy TBz staging const streaming SD SB
+    uint64_t start;     // cumulative rank of the first completion
+    uint64_t count;
+  };
+  void cores_for(const int32_t* prefix, std::vector<Core>* cores) const;
+  StencilInfo st_;
+  std::vector<Prefix> prefixes_;
+  uint64_t total_ = 0;
+  std::vector<int32_t> p2_[3];  // powers of two <= M_d
+};
+
+// ------------------------------------------------------------------ driver entry points
+struct Driver {
+  PFN_cuModuleLoadData_v2000 cuModuleLoadData = nullptr;
+  PFN_cuModuleUnload_v2000 cuModuleUnload = nullptr;
+  PFN_cuModuleGetFunction_v2000 cuModuleGetFunction = nullptr;
+  PFN_cuModuleGetGlobal_v3020 cuModuleGetGlobal = nullptr;
+  PFN_cuFuncSetAttribute_v9000 cuFuncSetAttribute = nullptr;
+  PFN_cuFuncGetAttribute_v2020 cuFuncGetAttribute = nullptr;
+  PFN_cuLaunchKernel_v4000 cuLaunchKernel = nullptr;
+  PFN_cuTensorMapEncodeTiled_v12000 cuTensorMapEncodeTiled = nullptr;
+  PFN_cuOccupancyMaxActiveBlocksPerMultiprocessor_v6050 cuOccupancy = nullptr;
+  PFN_cuGetErrorString_v6000 cuGetErrorString = nullptr;
+};
+cst_status driver(const Driver** out);
+cst_status cu_check(CUresult r, const char* what);
+
+// ------------------------------------------------------------------ JIT
+struct Variant {
+  CUmodule mod = nullptr;
+  CUfunction fn = nullptr;
+  int smem = 0;
+  int regs = 0;
+  int local = 0;
+  int threads = 0;
+  int occ = 0;
+  double compile_s = 0;
+  bool coef_uploaded = false;
+};
+// Compile (or fetch from the memory/disk cache) the cubin of a variant.
+cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
+                     double* compile_s);
+uint64_t jit_compile_count();
+
+}  // namespace cst
+
+// Launch one sweep of local interior planes [z0, z0 + nz) (sub-domain sweeps).
+cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* const* in,
+                            double* const* out, int64_t z0, int64_t nz, cudaStream_t stream);
+
+namespace cst {
+
+}  // namespace cst
+
+struct cst_stencil {
+  cst_stencil_desc desc{};
+  std::vector<double> coeffs;
+  cst_grid grid{};
+  int device = 0;
+  cst::StencilInfo info{};
+  std::unique_ptr<cst::Space> space;
+  std::map<std::string, cst::Variant> variants;
+  // TMA descriptor cache: (array base pointer, box dims) -> map
+  std::map<std::array<int64_t, 4>, cst_tmap> tmaps;
+  // host-path staging
+  std::vector<double*> dev_bufs;
+  size_t dev_buf_elems = 0;
+  cudaStream_t host_stream = nullptr;
+  int64_t last_launches = 0;
+};

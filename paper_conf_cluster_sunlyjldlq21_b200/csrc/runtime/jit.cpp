@@ -1,0 +1,153 @@
+// jit.cpp — code generation of kernel variants (csTuner: "the code generation writes the
+// sampled parameter settings into CUDA kernels"; checked before generation so that
+// only valid settings are compiled).  NVRTC compiles
+// csrc/kernels/cst_kernels.cuh for sm_100a with the setting as compile-time constants;
+// cubins are cached in memory and on disk ($CST_CACHE_DIR, default ~/.cache/cst).
+#include <nvrtc.h>
+#include <sys/stat.h>
+#include <unistd.h>
+
+#include <atomic>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
+#include <fstream>
+#include <sstream>
+#include <unordered_map>
+
+#include "internal.h"
+
+namespace {
+#include "kernels_src.inc"  // kSrcParams, kSrcPtx, kSrcKernels (generated at build time)
+
+std::mutex g_mu;
+std::unordered_map<std::string, std::string> g_mem;  // key -> cubin
+std::atomic<uint64_t> g_compiles{0};
+
+uint64_t fnv1a(const std::string& s, uint64_t h = 0xCBF29CE484222325ULL) {
+  for (unsigned char c : s) {
+    h ^= c;
+    h *= 0x100000001B3ULL;
+  }
+  return h;
+}
+
+std::string cache_dir() {
+  const char* d = std::getenv("CST_CACHE_DIR");
+  if (d && *d) return d;
+  const char* x = std::getenv("XDG_CACHE_HOME");
+  if (x && *x) return std::string(x) + "/cst";
+  const char* h = std::getenv("HOME");
+  return std::string(h ? h : "/tmp") + "/.cache/cst";
+}
+
+void mkdirs(const std::string& p) {
+  std::string cur;
+  std::stringstream ss(p);
+  std::string part;
+  if (!p.empty() && p[0] == '/') cur = "/";
+  while (std::getline(ss, part, '/')) {
+    if (part.empty()) continue;
+    cur += part + "/";
+    mkdir(cur.c_str(), 0755);
+  }
+}
+
+}  // namespace
+
+namespace cst {
+
+uint64_t jit_compile_count() { return g_compiles.load(); }
+
+static std::string prefix_for(const StencilInfo& st, const Tuple& t) {
+  std::ostringstream o;
+  o << "#define CST_KIND " << st.kind << "\n#define CST_R " << st.r << "\n";
+  static const char* names[F_COUNT] = {"TBX", "TBY", "TBZ", "STAGING", "CONST", "STREAM",
+                                       "SD",  "SB",  "UFX", "UFY",     "UFZ",   "CMX",
+                                       "CMY", "CMZ", "BMX", "BMY",     "BMZ",   "RET",
+                                       "PF"};
+  for (int i = 0; i < F_COUNT; ++i) o << "#define CST_" << names[i] << " " << t[i] << "\n";
+  o << "#include \"cst_kernels.cuh\"\n";
+  return o.str();
+}
+
+cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
+                     double* compile_s) {
+  const std::string src = prefix_for(st, t);
+  static const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo",
+                               "--fmad=true", "-DCST_NVRTC=1"};
+  const int nopts = sizeof(opts) / sizeof(opts[0]);
+  int nv_major = 0, nv_minor = 0;
+  nvrtcVersion(&nv_major, &nv_minor);
+  std::string keysrc = src + "nvrtc" + std::to_string(nv_major) + "." + std::to_string(nv_minor);
+  for (int i = 0; i < nopts; ++i) keysrc += opts[i];
+  uint64_t h = fnv1a(keysrc);
+  h = fnv1a(kSrcParams, h);
+  h = fnv1a(kSrcPtx, h);
+  h = fnv1a(kSrcKernels, h);
+  char key[32];
+  std::snprintf(key, sizeof key, "%016llx", (unsigned long long)h);
+  *compile_s = 0;
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    auto it = g_mem.find(key);
+    if (it != g_mem.end()) {
+      *cubin = it->second;
+      return CST_OK;
+    }
+  }
+  const std::string dir = cache_dir();
+  const std::string path = dir + "/" + key + ".cubin";
+  {
+    std::ifstream f(path, std::ios::binary);
+    if (f) {
+      std::string data((std::istreambuf_iterator<char>(f)), std::istreambuf_iterator<char>());
+      if (!data.empty()) {
+        std::lock_guard<std::mutex> lk(g_mu);
+        g_mem[key] = data;
+        *cubin = data;
+        return CST_OK;
+      }
+    }
+  }
+  const auto t0 = std::chrono::steady_clock::now();
+  const char* hdr_src[3] = {kSrcParams, kSrcPtx, kSrcKernels};
+  const char* hdr_names[3] = {"cst_params.h", "cst_ptx.cuh", "cst_kernels.cuh"};
+  nvrtcProgram prog;
+  if (nvrtcCreateProgram(&prog, src.c_str(), "cst_variant.cu", 3, hdr_src, hdr_names) !=
+      NVRTC_SUCCESS)
+    return fail(CST_E_NVRTC, "nvrtcCreateProgram failed");
+  const nvrtcResult rc = nvrtcCompileProgram(prog, nopts, opts);
+  if (rc != NVRTC_SUCCESS) {
+    size_t n = 0;
+    nvrtcGetProgramLogSize(prog, &n);
+    std::string log(n, '\0');
+    if (n) nvrtcGetProgramLog(prog, &log[0]);
+    nvrtcDestroyProgram(&prog);
+    return fail(CST_E_NVRTC, std::string("nvrtc: ") + nvrtcGetErrorString(rc) + "\n" +
+                                 log.substr(0, 4000));
+  }
+  size_t n = 0;
+  nvrtcGetCUBINSize(prog, &n);
+  std::string data(n, '\0');
+  nvrtcGetCUBIN(prog, &data[0]);
+  nvrtcDestroyProgram(&prog);
+  ++g_compiles;
+  *compile_s =
+      std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_mem[key] = data;
+  }
+  mkdirs(dir);
+  const std::string tmp = path + ".tmp" + std::to_string(getpid());
+  {
+    std::ofstream f(tmp, std::ios::binary);
+    if (f) f.write(data.data(), (std::streamsize)data.size());
+  }
+  std::rename(tmp.c_str(), path.c_str());
+  *cubin = data;
+  return CST_OK;
+}
+
+}  // namespace cst

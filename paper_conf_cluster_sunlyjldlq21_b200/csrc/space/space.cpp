@@ -1,0 +1,405 @@
+// space.cpp — the parameter space of Table I with the rules of DESIGN.md §3:
+// explicit rules of P:149 (R1-R3), our semantics rules (R4-R9) and the
+// implicit resource rules (R10-R12: "settings ... restricted by the usage of
+// register and shared memory ... only non-spilled parameter settings are explored").
+//
+// Canonical order: lexicographic over the 19 fields in Table I row order, values
+// ascending.  count / rank / unrank are exact (bit-exact with oracle/space.py).
+#include <algorithm>
+#include <cstring>
+
+#include "../runtime/internal.h"
+
+namespace cst {
+
+const char* const kFieldNames[F_COUNT] = {
+    "tb_x", "tb_y", "tb_z", "staging", "use_constant", "use_streaming", "sd", "sb",
+    "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z", "bm_x", "bm_y", "bm_z",
+    "use_retiming", "prefetch"};
+
+Tuple to_tuple(const cst_setting& s) {
+  return Tuple{s.tb[0], s.tb[1], s.tb[2], s.staging, s.use_constant, s.use_streaming,
+               s.sd, s.sb, s.uf[0], s.uf[1], s.uf[2], s.cm[0], s.cm[1], s.cm[2],
+               s.bm[0], s.bm[1], s.bm[2], s.use_retiming, s.prefetch};
+}
+
+cst_setting from_tuple(const Tuple& t) {
+  cst_setting s;
+  s.tb[0] = t[F_TBX]; s.tb[1] = t[F_TBY]; s.tb[2] = t[F_TBZ];
+  s.staging = t[F_STAGING]; s.use_constant = t[F_CONST]; s.use_streaming = t[F_STREAM];
+  s.sd = t[F_SD]; s.sb = t[F_SB];
+  for (int d = 0; d < 3; ++d) {
+    s.uf[d] = t[F_UFX + d];
+    s.cm[d] = t[F_CMX + d];
+    s.bm[d] = t[F_BMX + d];
+  }
+  s.use_retiming = t[F_RET]; s.prefetch = t[F_PF];
+  return s;
+}
+
+std::string setting_key(const cst_setting& s) {
+  Tuple t = to_tuple(s);
+  std::string k;
+  for (int i = 0; i < F_COUNT; ++i) {
+    if (i) k += ',';
+    k += std::to_string(t[i]);
+  }
+  return k;
+}
+
+static const int64_t SMEM_LIMIT = 227 * 1024 - 1024;
+static const int64_t REG_LIMIT = 255;
+
+static int n_arrays(int kind) { return kind == CST_HYPTERM ? 8 : 1; }
+static int live_doubles(int kind, int r) {
+  return kind == CST_STAR ? 2 * r + 2 : (kind == CST_BOX ? 12 : 50);
+}
+static int retention(int kind, int r) { return kind == CST_BOX ? 2 * r : r; }
+
+static void tiles(const Tuple& t, int64_t T[3]) {
+  for (int d = 0; d < 3; ++d)
+    T[d] = (int64_t)t[F_TBX + d] * t[F_BMX + d] * t[F_CMX + d];
+}
+
+// (P, NP): in-plane (or 3-D box) elements and ring planes of the modelled staging
+static void plane_geometry(int kind, int r, const Tuple& t, int64_t* P, int64_t* NP) {
+  int64_t T[3];
+  tiles(t, T);
+  if (t[F_STREAM] == 1) {
+    *P = (T[0] + 2 * r) * (T[1] + 2 * r) * (T[2] + 2 * r);
+    *NP = 1;
+    return;
+  }
+  const int sd = t[F_SD] - 1;
+  int a = -1, b = -1;
+  for (int d = 0; d < 3; ++d)
+    if (d != sd) (a < 0 ? a : b) = d;
+  *P = (T[a] + 2 * r) * (T[b] + 2 * r);
+  const int64_t D = t[F_PF];
+  if (T[sd] == 1)
+    *NP = D + (t[F_RET] == 2 ? 0 : retention(kind, r));
+  else
+    *NP = D * T[sd] + 2 * r;
+}
+
+int64_t model_smem_bytes(int kind, int r, const Tuple& t) {
+  if (t[F_STAGING] == 1) return 0;
+  int64_t P, NP;
+  plane_geometry(kind, r, t, &P, &NP);
+  const int64_t plane = (P * 8 + 127) / 128 * 128;
+  return n_arrays(kind) * NP * plane;
+}
+
+int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
+  if (t[F_STAGING] == 1) return 0;
+  int64_t T[3];
+  tiles(t, T);
+  int64_t P, NP;
+  plane_geometry(kind, r, t, &P, &NP);
+  const int64_t plane = (P * 8 + 127) / 128 * 128;
+  if (t[F_STREAM] == 2) {
+    const int sd = t[F_SD] - 1;
+    // only the star has the T_SD == 1 fast path so far; others run the generic ring
+    if (!(kind == CST_STAR && T[sd] == 1)) NP = (int64_t)t[F_PF] * T[sd] + 2 * r;
+  }
+  const int64_t bars = t[F_STAGING] == 3 ? NP * 8 : 0;
+  return n_arrays(kind) * NP * plane + bars;
+}
+
+int64_t model_regs(int kind, int r, const Tuple& t) {
+  int64_t ppt = 1;
+  for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
+  const int64_t nthr = (int64_t)t[F_TBX] * t[F_TBY] * t[F_TBZ];
+  int64_t pf = 0;
+  if (t[F_STAGING] == 2 && t[F_PF] > 1) {
+    int64_t P, NP;
+    plane_geometry(kind, r, t, &P, &NP);
+    int64_t T[3];
+    tiles(t, T);
+    const int64_t per_step = t[F_STREAM] == 2 ? T[t[F_SD] - 1] : 1;
+    pf = (t[F_PF] - 1) * ((n_arrays(kind) * P * per_step + nthr - 1) / nthr);
+  }
+  return 32 + 2 * ppt * live_doubles(kind, r) + 2 * pf;
+}
+
+static bool tma_ok(int r, const Tuple& t) {
+  int64_t T[3];
+  tiles(t, T);
+  if (T[0] % 2) return false;
+  for (int d = 0; d < 3; ++d) {
+    const bool streamed = t[F_STREAM] == 2 && d == t[F_SD] - 1;
+    const int64_t e = streamed ? T[d] : T[d] + 2 * r;
+    if (e > 256) return false;
+  }
+  return true;
+}
+
+static bool is_p2(int64_t v) { return v >= 1 && (v & (v - 1)) == 0; }
+
+const char* check_rules(const StencilInfo& st, const Tuple& t) {
+  // ranges (Table I)
+  const int64_t* M = st.M;
+  if (!is_p2(t[F_TBX]) || t[F_TBX] > 1024 || !is_p2(t[F_TBY]) || t[F_TBY] > 1024 ||
+      !is_p2(t[F_TBZ]) || t[F_TBZ] > 64)
+    return "range: TB";
+  if (t[F_STAGING] < 1 || t[F_STAGING] > 3) return "range: staging";
+  if (t[F_CONST] < 1 || t[F_CONST] > 2) return "range: use_constant";
+  if (t[F_STREAM] < 1 || t[F_STREAM] > 2) return "range: use_streaming";
+  if (t[F_SD] < 1 || t[F_SD] > 3) return "range: sd";
+  if (!is_p2(t[F_SB]) || t[F_SB] > M[t[F_SD] - 1]) return "range: sb";
+  for (int d = 0; d < 3; ++d) {
+    if (!is_p2(t[F_UFX + d]) || t[F_UFX + d] > M[d]) return "range: uf";
+    if (!is_p2(t[F_CMX + d]) || t[F_CMX + d] > M[d]) return "range: cm";
+    if (!is_p2(t[F_BMX + d]) || t[F_BMX + d] > M[d]) return "range: bm";
+  }
+  if (t[F_RET] < 1 || t[F_RET] > 2) return "range: use_retiming";
+  if (t[F_PF] < 1 || t[F_PF] > 4) return "range: prefetch";
+
+  const int64_t tb = (int64_t)t[F_TBX] * t[F_TBY] * t[F_TBZ];
+  if (tb > 1024) return "R1";
+  const bool stream = t[F_STREAM] == 2;
+  if (!stream && (t[F_SD] != 1 || t[F_SB] != 1)) return "R2";
+  if (stream && t[F_SD] == 1) return "R8";
+  if (tb < 32) return "R4";
+  int64_t T[3];
+  tiles(t, T);
+  const int sd = t[F_SD] - 1;
+  for (int d = 0; d < 3; ++d) {
+    const int64_t E = (stream && d == sd) ? t[F_SB] : M[d];
+    if (T[d] > E) return "R5";
+  }
+  if (stream && t[F_UFX + sd] > t[F_SB]) return "R3";
+  for (int d = 0; d < 3; ++d) {
+    const int64_t trip = (stream && d == sd) ? t[F_SB] / T[d]
+                                             : (int64_t)t[F_BMX + d] * t[F_CMX + d];
+    if (t[F_UFX + d] > trip) return "R6";
+  }
+  int64_t ppt = 1;
+  for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
+  if (ppt > 16) return "R7";
+  if (t[F_PF] > 1 && !stream) return "R9";
+  if (model_smem_bytes(st.kind, st.r, t) > SMEM_LIMIT) return "R10";
+  if (model_regs(st.kind, st.r, t) > REG_LIMIT) return "R11";
+  if (t[F_STAGING] == 3 && !tma_ok(st.r, t)) return "R12";
+  return nullptr;
+}
+
+// ------------------------------------------------------------------ enumerator
+static std::vector<int32_t> p2_upto(int64_t hi) {
+  std::vector<int32_t> v;
+  for (int64_t x = 1; x <= hi; x *= 2) v.push_back((int32_t)x);
+  return v;
+}
+
+static int32_t count_le(const std::vector<int32_t>& v, int64_t bound) {
+  int32_t n = 0;
+  for (int32_t x : v)
+    if (x <= bound) ++n;
+  return n;
+}
+
+void Space::cores_for(const int32_t* pre, std::vector<Core>* cores) const {
+  cores->clear();
+  Tuple t{};
+  for (int i = 0; i < 8; ++i) t[i] = pre[i];
+  t[F_UFX] = t[F_UFY] = t[F_UFZ] = 1;
+  const bool stream = pre[F_STREAM] == 2;
+  const int sd = pre[F_SD] - 1;
+  for (int32_t cmx : p2_[0])
+    for (int32_t cmy : p2_[1])
+      for (int32_t cmz : p2_[2]) {
+        if ((int64_t)cmx * cmy * cmz > 16) continue;
+        for (int32_t bmx : p2_[0])
+          for (int32_t bmy : p2_[1])
+            for (int32_t bmz : p2_[2]) {
+              if ((int64_t)cmx * cmy * cmz * bmx * bmy * bmz > 16) continue;
+              const int32_t cm[3] = {cmx, cmy, cmz}, bm[3] = {bmx, bmy, bmz};
+              bool cover = true;
+              for (int d = 0; d < 3; ++d)
+                if ((int64_t)pre[F_TBX + d] * cm[d] * bm[d] > st_.M[d]) cover = false;
+              if (!cover) continue;
+              for (int32_t ret = 1; ret <= 2; ++ret)
+                for (int32_t pf = 1; pf <= 4; ++pf) {
+                  for (int d = 0; d < 3; ++d) {
+                    t[F_CMX + d] = cm[d];
+                    t[F_BMX + d] = bm[d];
+                  }
+                  t[F_RET] = ret;
+                  t[F_PF] = pf;
+                  if (check_rules(st_, t) != nullptr) continue;
+                  Core c;
+                  for (int d = 0; d < 3; ++d) {
+                    c.cm[d] = cm[d];
+                    c.bm[d] = bm[d];
+                    const int64_t Td = (int64_t)pre[F_TBX + d] * cm[d] * bm[d];
+                    const int64_t trip = (stream && d == sd) ? pre[F_SB] / Td
+                                                             : (int64_t)cm[d] * bm[d];
+                    c.nuf[d] = count_le(p2_[d], trip);
+                  }
+                  c.ret = ret;
+                  c.pf = pf;
+                  cores->push_back(c);
+                }
+            }
+      }
+  // canonical core order: CMx, CMy, CMz, BMx, BMy, BMz, ret, pf
+  std::stable_sort(cores->begin(), cores->end(), [](const Core& a, const Core& b) {
+    const int32_t ka[8] = {a.cm[0], a.cm[1], a.cm[2], a.bm[0], a.bm[1], a.bm[2], a.ret, a.pf};
+    const int32_t kb[8] = {b.cm[0], b.cm[1], b.cm[2], b.bm[0], b.bm[1], b.bm[2], b.ret, b.pf};
+    return std::lexicographical_compare(ka, ka + 8, kb, kb + 8);
+  });
+}
+
+Space::Space(const StencilInfo& st) : st_(st) {
+  for (int d = 0; d < 3; ++d) p2_[d] = p2_upto(st.M[d]);
+  const std::vector<int32_t> tbxy = p2_upto(1024), tbz = p2_upto(64);
+  std::vector<Core> cores;
+  uint64_t cum = 0;
+  for (int32_t tbx : tbxy) {
+    if (tbx > st.M[0]) continue;
+    for (int32_t tby : tbxy) {
+      if (tby > st.M[1] || (int64_t)tbx * tby > 1024) continue;
+      for (int32_t tbzv : tbz) {
+        const int64_t tb = (int64_t)tbx * tby * tbzv;
+        if (tbzv > st.M[2] || tb > 1024 || tb < 32) continue;
+        for (int32_t stg = 1; stg <= 3; ++stg)
+          for (int32_t uc = 1; uc <= 2; ++uc)
+            for (int32_t strm = 1; strm <= 2; ++strm)
+              for (int32_t sd = 1; sd <= 3; ++sd) {
+                if (strm == 1 && sd != 1) continue;
+                if (strm == 2 && sd == 1) continue;
+                const std::vector<int32_t> sbs =
+                    strm == 2 ? p2_upto(st.M[sd - 1]) : std::vector<int32_t>{1};
+                for (int32_t sb : sbs) {
+                  Prefix p;
+                  const int32_t v[8] = {tbx, tby, tbzv, stg, uc, strm, sd, sb};
+                  std::memcpy(p.v, v, sizeof v);
+                  cores_for(p.v, &cores);
+                  uint64_t n = 0;
+                  for (const Core& c : cores) n += (uint64_t)c.nuf[0] * c.nuf[1] * c.nuf[2];
+                  if (n == 0) continue;
+                  p.start = cum;
+                  p.count = n;
+                  cum += n;
+                  prefixes_.push_back(p);
+                }
+              }
+      }
+    }
+  }
+  total_ = cum;
+}
+
+bool Space::at(uint64_t rank, Tuple* out) const {
+  if (rank >= total_) return false;
+  // prefix by binary search on start
+  size_t lo = 0, hi = prefixes_.size();
+  while (hi - lo > 1) {
+    const size_t mid = (lo + hi) / 2;
+    if (prefixes_[mid].start <= rank) lo = mid;
+    else hi = mid;
+  }
+  const Prefix& P = prefixes_[lo];
+  uint64_t q = rank - P.start;
+  std::vector<Core> cores;
+  cores_for(P.v, &cores);
+  Tuple t{};
+  for (int i = 0; i < 8; ++i) t[i] = P.v[i];
+  // UF_x, UF_y, UF_z in turn: candidate value index u_d (0-based) allowed iff u_d < nuf[d]
+  int32_t uidx[3] = {-1, -1, -1};
+  for (int d = 0; d < 3; ++d) {
+    bool found = false;
+    for (int32_t u = 0; u < (int32_t)p2_[d].size(); ++u) {
+      uint64_t cnt = 0;
+      for (const Core& c : cores) {
+        bool okc = true;
+        for (int e = 0; e < d; ++e)
+          if (uidx[e] >= c.nuf[e]) okc = false;
+        if (!okc || u >= c.nuf[d]) continue;
+        uint64_t m = 1;
+        for (int e = d + 1; e < 3; ++e) m *= (uint64_t)c.nuf[e];
+        cnt += m;
+      }
+      if (q < cnt) {
+        uidx[d] = u;
+        found = true;
+        break;
+      }
+      q -= cnt;
+    }
+    if (!found) return false;
+  }
+  for (const Core& c : cores) {
+    if (uidx[0] >= c.nuf[0] || uidx[1] >= c.nuf[1] || uidx[2] >= c.nuf[2]) continue;
+    if (q == 0) {
+      for (int d = 0; d < 3; ++d) {
+        t[F_UFX + d] = p2_[d][uidx[d]];
+        t[F_CMX + d] = c.cm[d];
+        t[F_BMX + d] = c.bm[d];
+      }
+      t[F_RET] = c.ret;
+      t[F_PF] = c.pf;
+      *out = t;
+      return true;
+    }
+    --q;
+  }
+  return false;
+}
+
+bool Space::rank(const Tuple& t, uint64_t* out) const {
+  if (check_rules(st_, t) != nullptr) return false;
+  // locate prefix (prefixes_ are in canonical order)
+  const Prefix* P = nullptr;
+  {
+    size_t lo = 0, hi = prefixes_.size();
+    while (lo < hi) {
+      const size_t mid = (lo + hi) / 2;
+      if (std::lexicographical_compare(prefixes_[mid].v, prefixes_[mid].v + 8, t.data(),
+                                       t.data() + 8))
+        lo = mid + 1;
+      else
+        hi = mid;
+    }
+    if (lo >= prefixes_.size() || !std::equal(t.data(), t.data() + 8, prefixes_[lo].v))
+      return false;
+    P = &prefixes_[lo];
+  }
+  std::vector<Core> cores;
+  cores_for(P->v, &cores);
+  int32_t uidx[3];
+  for (int d = 0; d < 3; ++d) {
+    uidx[d] = -1;
+    for (int32_t u = 0; u < (int32_t)p2_[d].size(); ++u)
+      if (p2_[d][u] == t[F_UFX + d]) uidx[d] = u;
+    if (uidx[d] < 0) return false;
+  }
+  uint64_t q = 0;
+  for (int d = 0; d < 3; ++d) {
+    for (int32_t u = 0; u < uidx[d]; ++u) {
+      for (const Core& c : cores) {
+        bool okc = true;
+        for (int e = 0; e < d; ++e)
+          if (uidx[e] >= c.nuf[e]) okc = false;
+        if (!okc || u >= c.nuf[d]) continue;
+        uint64_t m = 1;
+        for (int e = d + 1; e < 3; ++e) m *= (uint64_t)c.nuf[e];
+        q += m;
+      }
+    }
+  }
+  for (const Core& c : cores) {
+    if (uidx[0] >= c.nuf[0] || uidx[1] >= c.nuf[1] || uidx[2] >= c.nuf[2]) continue;
+    bool same = c.ret == t[F_RET] && c.pf == t[F_PF];
+    for (int d = 0; d < 3; ++d)
+      same = same && c.cm[d] == t[F_CMX + d] && c.bm[d] == t[F_BMX + d];
+    if (same) {
+      *out = P->start + q;
+      return true;
+    }
+    ++q;
+  }
+  return false;
+}
+
+}  // namespace cst
