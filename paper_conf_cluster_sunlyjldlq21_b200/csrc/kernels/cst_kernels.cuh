@@ -190,12 +190,37 @@ __device__ __forceinline__ int thread_z() { return (int)(threadIdx.x / (TBX * TB
 
 __host__ __device__ constexpr int round_slot(int elems) { return ((elems * 8 + 127) / 128) * 128 / 8; }
 
+// x-halo kept in shared memory / TMA boxes: R rounded up to even, so every box row starts
+// 16-B aligned in global memory (TMA requirement) and double2 loads stay aligned.
+constexpr int XR = R + (R & 1);
+
+template <bool B, class T, class F>
+struct Cond {
+  using type = T;
+};
+template <class T, class F>
+struct Cond<false, T, F> {
+  using type = F;
+};
+
+template <int V>
+struct IC {
+  static constexpr int value = V;
+};
+template <int I, int N, class F>
+__device__ __forceinline__ void static_for(F&& f) {
+  if constexpr (I < N) {
+    f(IC<I>{});
+    static_for<I + 1, N>(f);
+  }
+}
+
 // =============================================================================
 // 3-D tile path (use_streaming = 1)
 // =============================================================================
 __device__ __forceinline__ void kernel_tile3d(const cst_kparams& P, double* smem) {
   Ctx C{P};
-  constexpr int BX = TX + 2 * R, BY = TY + 2 * R, BZ = TZ + 2 * R;
+  constexpr int BX = TX + 2 * XR, BY = TY + 2 * R, BZ = TZ + 2 * R;
   constexpr int BOX = BX * BY * BZ;
   constexpr int BOXS = round_slot(BOX);
   const int tile_xy = blockIdx.x;
@@ -216,7 +241,7 @@ __device__ __forceinline__ void kernel_tile3d(const cst_kparams& P, double* smem
       mbar_arrive_expect_tx(bar, NIN * BOX * 8);
 #pragma unroll
       for (int a = 0; a < NIN; ++a)
-        tma_load_3d(smem + a * BOXS, &P.tma[a], bar, P.tox + x0 - R, P.toy + y0 - R,
+        tma_load_3d(smem + a * BOXS, &P.tma[a], bar, P.tox + x0 - XR, P.toy + y0 - R,
                     P.toz + z0 - R);
     }
     mbar_wait(bar, 0);
@@ -224,9 +249,9 @@ __device__ __forceinline__ void kernel_tile3d(const cst_kparams& P, double* smem
     for (int e = tid; e < NIN * BOX; e += NTHR) {
       const int a = e / BOX, r = e % BOX;
       const int ex = r % BX, ey = (r / BX) % BY, ez = r / (BX * BY);
-      const int gx = x0 - R + ex, gy = y0 - R + ey, gz = z0 - R + ez;
+      const int gx = x0 - XR + ex, gy = y0 - R + ey, gz = z0 - R + ez;
       double v = 0.0;
-      if (gx < P.nx + R && gy < P.ny + R && gz < P.nz + R)
+      if (gx >= -R && gx < P.nx + R && gy < P.ny + R && gz < P.nz + R)
         v = P.in[a][gx + gy * P.py + gz * P.pz];
       smem[a * BOXS + r] = v;
     }
@@ -253,7 +278,7 @@ __device__ __forceinline__ void kernel_tile3d(const cst_kparams& P, double* smem
           point(C, U, o);
         } else {
           auto U = [&](int a, int dx, int dy, int dz) {
-            return smem[a * BOXS + ((lz + R + dz) * BY + (ly + R + dy)) * BX + lx + R + dx];
+            return smem[a * BOXS + ((lz + R + dz) * BY + (ly + R + dy)) * BX + lx + XR + dx];
           };
           point(C, U, o);
         }
@@ -266,8 +291,12 @@ __device__ __forceinline__ void kernel_tile3d(const cst_kparams& P, double* smem
 }
 
 // =============================================================================
-// streaming geometry shared by both streaming paths
+// streaming geometry, plane staging (ring of plane slots; slot = NIN arrays)
 // =============================================================================
+constexpr int PA = TA + 2 * XR, PB = TB + 2 * R;
+constexpr int PL = PA * PB;
+constexpr int SLOT = round_slot(PL);
+
 struct SGeo {
   int n_a, n_b, n_s;
   long long st_b, st_s;  // element strides of b and s
@@ -289,51 +318,211 @@ __device__ __forceinline__ SGeo stream_geo(const cst_kparams& P) {
   return g;
 }
 
-// TMA coordinates of in-plane box origin (a0-R, b0-R) at stream plane p
+// TMA: in-plane box origin (a0 - XR, b0 - R) at stream plane p, all arrays
 __device__ __forceinline__ void tma_plane(const cst_kparams& P, const SGeo& g, double* dst,
                                           u64* bar, int p) {
 #pragma unroll
   for (int a = 0; a < NIN; ++a) {
-    constexpr int PA = TA + 2 * R, PB = TB + 2 * R;
-    constexpr int SLOT = round_slot(PA * PB);
     if constexpr (SZ)
-      tma_load_3d(dst + a * SLOT, &P.tma[a], bar, P.tox + g.a0 - R, P.toy + g.b0 - R,
+      tma_load_3d(dst + a * SLOT, &P.tma[a], bar, P.tox + g.a0 - XR, P.toy + g.b0 - R,
                   P.toz + p);
     else
-      tma_load_3d(dst + a * SLOT, &P.tma[a], bar, P.tox + g.a0 - R, P.toy + p,
+      tma_load_3d(dst + a * SLOT, &P.tma[a], bar, P.tox + g.a0 - XR, P.toy + p,
                   P.toz + g.b0 - R);
   }
 }
 
-// cooperative ld/st copy of one plane (all arrays) into a ring slot
-template <int PA, int PB, int SLOT>
+// global value of element r (0 <= r < NIN*PL) of plane p, 0 outside the padded region
+__device__ __forceinline__ double plane_elem(const cst_kparams& P, const SGeo& g, int e, int p) {
+  const int a = e / PL, r = e % PL;
+  const int ga = g.a0 - XR + r % PA, gb = g.b0 - R + r / PA;
+  if (ga >= -R && ga < g.n_a + R && gb < g.n_b + R)
+    return P.in[a][ga + gb * g.st_b + (long long)p * g.st_s];
+  return 0.0;
+}
+
 __device__ __forceinline__ void ldst_plane(const cst_kparams& P, const SGeo& g, double* dst,
                                            int p) {
-  constexpr int PL = PA * PB;
-  for (int e = threadIdx.x; e < NIN * PL; e += NTHR) {
-    const int a = e / PL, r = e % PL;
-    const int ea = r % PA, eb = r / PA;
-    const int ga = g.a0 - R + ea, gb = g.b0 - R + eb;
-    double v = 0.0;
-    if (ga < g.n_a + R && gb < g.n_b + R) v = P.in[a][ga + gb * g.st_b + p * g.st_s];
-    dst[a * SLOT + r] = v;
+  for (int e = threadIdx.x; e < NIN * PL; e += NTHR) dst[(e / PL) * SLOT + e % PL] = plane_elem(P, g, e, p);
+}
+
+// plane accessors: element (la, lb) of the tile-local in-plane coordinates
+struct SmemPlane {
+  static constexpr bool VEC = true;
+  const double* base;  // slot base of one array
+  __device__ __forceinline__ double at(int la, int lb) const { return base[(lb + R) * PA + la + XR]; }
+  __device__ __forceinline__ double2 at2(int la, int lb) const {
+    return *reinterpret_cast<const double2*>(base + (lb + R) * PA + la + XR);
+  }
+};
+struct GlobPlane {
+  static constexpr bool VEC = false;
+  const double* base;  // &u(a0, b0, p)
+  long long stb;
+  __device__ __forceinline__ double at(int la, int lb) const { return ldg_nc(base + la + lb * stb); }
+  __device__ __forceinline__ double2 at2(int la, int lb) const {
+    return make_double2(at(la, lb), at(la + 1, lb));
+  }
+};
+
+constexpr int NCA = BMA * CMA, NCB = BMB * CMB;
+constexpr int W = 2 * R + 1;
+
+// load the x-window [la0 - XR, la0 + BMA + XR) of row lb (only [la0-R, la0+BMA+R) used)
+template <class LD>
+__device__ __forceinline__ void load_xwin(const LD& ld, int la0, int lb, double* w) {
+  constexpr int WX = BMA + 2 * XR;
+  if constexpr (LD::VEC && (BMA % 2 == 0)) {
+#pragma unroll
+    for (int q = 0; q < WX / 2; ++q) {
+      const double2 v = ld.at2(la0 - XR + 2 * q, lb);
+      w[2 * q] = v.x;
+      w[2 * q + 1] = v.y;
+    }
+  } else {
+#pragma unroll
+    for (int q = XR - R; q < WX - (XR - R); ++q) w[q] = ld.at(la0 - XR + q, lb);
   }
 }
 
 // =============================================================================
-// fast streaming path, T_SD == 1: star
+// star: in-plane part  ip = c0*u + sum_k wa[k] u(a+k) + sum_k wb[k] u(b+k)  (oracle order)
+// register-blocked over the thread's BM_a x BM_b points (merging reuse)
 // =============================================================================
-__device__ __forceinline__ void kernel_star_stream1(const cst_kparams& P, double* smem) {
-  Ctx C{P};
-  constexpr int PA = TA + 2 * R, PB = TB + 2 * R;
-  constexpr int PL = PA * PB;
-  constexpr int SLOT = round_slot(PL);
-  constexpr int D = PF;
-  constexpr int NP = STAGING == 1 ? 1 : D + (RETIME ? 0 : R);
-  constexpr int NCA = BMA * CMA, NCB = BMB * CMB, NC = NCA * NCB;
-  constexpr int W = 2 * R + 1;
-  constexpr int FR = (NIN * PL + NTHR - 1) / NTHR;  // ld/st prefetch fragment per thread
+template <class LD>
+__device__ __forceinline__ void star_inplane(const Ctx& C, const LD& ld, const int* la,
+                                             const int* lb, double (&ip)[NCB][NCA],
+                                             double (&cen)[NCB][NCA]) {
+#pragma unroll
+  for (int ib = 0; ib < NCB; ++ib) {
+#pragma unroll
+    for (int ca = 0; ca < CMA; ++ca) {
+      double w[BMA + 2 * XR];
+      load_xwin(ld, la[ca * BMA], lb[ib], w);
+#pragma unroll
+      for (int b = 0; b < BMA; ++b) {
+        const double c = w[XR + b];
+        double s = C.coef(0) * c;
+#pragma unroll
+        for (int k = -R; k <= R; ++k)
+          if (k != 0) s = fma(C.coef(star_ci(AX_A, k)), w[XR + b + k], s);
+        ip[ib][ca * BMA + b] = s;
+        cen[ib][ca * BMA + b] = c;
+      }
+    }
+  }
+#pragma unroll
+  for (int cb = 0; cb < CMB; ++cb) {
+    const int lb0 = lb[cb * BMB];
+#pragma unroll
+    for (int ia = 0; ia < NCA; ++ia) {
+      constexpr bool PAIR = LD::VEC && (BMA % 2 == 0);
+      if (PAIR && (ia % 2)) continue;
+      double top[PAIR ? 2 : 1][R], bot[PAIR ? 2 : 1][R];
+#pragma unroll
+      for (int t = 0; t < R; ++t) {
+        if constexpr (PAIR) {
+          const double2 a = ld.at2(la[ia], lb0 - 1 - t);
+          const double2 b = ld.at2(la[ia], lb0 + BMB + t);
+          top[0][t] = a.x; top[1][t] = a.y;
+          bot[0][t] = b.x; bot[1][t] = b.y;
+        } else {
+          top[0][t] = ld.at(la[ia], lb0 - 1 - t);
+          bot[0][t] = ld.at(la[ia], lb0 + BMB + t);
+        }
+      }
+#pragma unroll
+      for (int pc = 0; pc < (PAIR ? 2 : 1); ++pc) {
+        const int iac = ia + pc;
+#pragma unroll
+        for (int rb = 0; rb < BMB; ++rb) {
+          double s = ip[cb * BMB + rb][iac];
+#pragma unroll
+          for (int k = -R; k <= R; ++k) {
+            if (k == 0) continue;
+            const int rr = rb + k;
+            const double v = rr < 0 ? top[pc][-rr - 1]
+                                    : (rr >= BMB ? bot[pc][rr - BMB] : cen[cb * BMB + rr][iac]);
+            s = fma(C.coef(star_ci(AX_B, k)), v, s);
+          }
+          ip[cb * BMB + rb][iac] = s;
+        }
+      }
+    }
+  }
+}
 
+template <class LD>
+__device__ __forceinline__ void load_centres(const LD& ld, const int* la, const int* lb,
+                                             double (&cen)[NCB][NCA]) {
+#pragma unroll
+  for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+    for (int ia = 0; ia < NCA; ++ia) {
+      if constexpr (LD::VEC && (BMA % 2 == 0)) {
+        if (ia % 2) continue;
+        const double2 v = ld.at2(la[ia], lb[ib]);
+        cen[ib][ia] = v.x;
+        cen[ib][ia + 1] = v.y;
+      } else {
+        cen[ib][ia] = ld.at(la[ia], lb[ib]);
+      }
+    }
+}
+
+// =============================================================================
+// box (r = 1): slice sums  S_ds(p) = sum_{db,da} c(ds, db, da) u(a+da, b+db, p)
+// =============================================================================
+__host__ __device__ constexpr int box_ci(int ds, int db, int da) {
+  // coefficient c[dz][dy][dx] (z-major); s = z (SD = 3) or y (SD = 2)
+  return SZ ? ((ds + R) * W + (db + R)) * W + (da + R) : ((db + R) * W + (ds + R)) * W + (da + R);
+}
+
+// accumulate slices ds = DS0 + q*DSTEP (q < NS) of plane `ld` into chains S[q][ib][ia]
+// (db, da ascending within each chain)
+template <int NS, int DS0, int DSTEP, class LD>
+__device__ __forceinline__ void box_slices(const Ctx& C, const LD& ld, const int* la, const int* lb,
+                                           double (&S)[NS][NCB][NCA]) {
+#pragma unroll
+  for (int cb = 0; cb < CMB; ++cb) {
+    const int lb0 = lb[cb * BMB];
+#pragma unroll
+    for (int ca = 0; ca < CMA; ++ca) {
+      const int la0 = la[ca * BMA];
+#pragma unroll
+      for (int wr = -R; wr < BMB + R; ++wr) {  // window rows
+        double w[BMA + 2 * XR];
+        load_xwin(ld, la0, lb0 + wr, w);
+#pragma unroll
+        for (int rb = 0; rb < BMB; ++rb) {
+          const int db = wr - rb;
+          if (db < -R || db > R) continue;
+#pragma unroll
+          for (int b = 0; b < BMA; ++b)
+#pragma unroll
+            for (int da = -R; da <= R; ++da)
+#pragma unroll
+              for (int q = 0; q < NS; ++q) {
+                double& acc = S[q][cb * BMB + rb][ca * BMA + b];
+                acc = fma(C.coef(box_ci(DS0 + q * DSTEP, db, da)), w[XR + b + da], acc);
+              }
+        }
+      }
+    }
+  }
+}
+
+// =============================================================================
+// fast streaming path, T_SD == 1 (star / box): one plane per step, rotation-unrolled
+// =============================================================================
+constexpr int RETAIN = RETIME ? 0 : (KIND == 2 ? 2 * R : R);
+constexpr int NP1 = PF + RETAIN;                          // ring slots
+constexpr int FR = (NIN * PL + NTHR - 1) / NTHR;          // ld/st prefetch fragment
+
+__device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* smem) {
+  Ctx C{P};
+  constexpr int D = PF;
+  constexpr int NP = STAGING == 1 ? 1 : NP1;
   const SGeo g = stream_geo(P);
   const int ta = thread_x();
   const int tb = SZ ? thread_y() : thread_z();
@@ -341,23 +530,23 @@ __device__ __forceinline__ void kernel_star_stream1(const cst_kparams& P, double
   const int n_planes = (g.s_end - g.s_start) + 2 * R;
   const double* __restrict__ in = P.in[0];
   double* __restrict__ out = P.out[0];
-  u64* bars = (u64*)(smem + NP * SLOT);
+  u64* bars = (u64*)(smem + NP * NIN * SLOT);
 
-  int la[NC], lb[NC];
-  bool ok[NC];
+  int la[NCA], lb[NCB];
 #pragma unroll
-  for (int i = 0; i < NC; ++i) {
-    la[i] = merged_pos(i % NCA, ta, TBA, BMA);
-    lb[i] = merged_pos(i / NCA, tb, TBB, BMB);
-    ok[i] = (g.a0 + la[i] < g.n_a) && (g.b0 + lb[i] < g.n_b);
-  }
+  for (int i = 0; i < NCA; ++i) la[i] = merged_pos(i, ta, TBA, BMA);
+#pragma unroll
+  for (int i = 0; i < NCB; ++i) lb[i] = merged_pos(i, tb, TBB, BMB);
   const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
 
-  double acc[NC][W];  // retimed: acc[i][m] = output plane p-R+m ; gather: queue of centres
+  // retimed: acc = pending outputs (2R+1 per point); gather: queue of centre values
+  double acc[NCB][NCA][W];
 #pragma unroll
-  for (int i = 0; i < NC; ++i)
+  for (int ib = 0; ib < NCB; ++ib)
 #pragma unroll
-    for (int m = 0; m < W; ++m) acc[i][m] = 0.0;
+    for (int ia = 0; ia < NCA; ++ia)
+#pragma unroll
+      for (int m = 0; m < W; ++m) acc[ib][ia][m] = 0.0;
 
   double frag[D > 1 && STAGING == 2 ? (D - 1) * FR : 1];
 
@@ -375,155 +564,476 @@ __device__ __forceinline__ void kernel_star_stream1(const cst_kparams& P, double
       }
     }
   } else if constexpr (STAGING == 2) {
-    ldst_plane<PA, PB, SLOT>(P, g, smem, g.s_start - R);
+    ldst_plane(P, g, smem, g.s_start - R);
     if constexpr (D > 1) {
 #pragma unroll
-      for (int f = 0; f < D - 1; ++f) {
-        const int p = g.s_start - R + 1 + f;
+      for (int f = 0; f < D - 1; ++f)
 #pragma unroll
         for (int q = 0; q < FR; ++q) {
           const int e = tid + q * NTHR;
-          double v = 0.0;
-          if (e < NIN * PL && 1 + f < n_planes) {
-            const int r = e % PL;
-            const int ga = g.a0 - R + r % PA, gb = g.b0 - R + r / PA;
-            if (ga < g.n_a + R && gb < g.n_b + R) v = in[ga + gb * g.st_b + (long long)p * g.st_s];
-          }
-          frag[f * FR + q] = v;
+          frag[f * FR + q] =
+              (e < NIN * PL && 1 + f < n_planes) ? plane_elem(P, g, e, g.s_start - R + 1 + f) : 0.0;
         }
-      }
     }
     __syncthreads();
   }
 
-  // in-plane accessor of plane held in ring slot `slot` (or global plane p)
-  auto inplane = [&](int i, int slot, int p) -> double {
-    // c0*u + sum_a + sum_b ; summation order c0, a(=x), b
-    if constexpr (STAGING == 1) {
-      const double* c = in + col0 + la[i] + (long long)lb[i] * g.st_b + (long long)p * g.st_s;
-      double s = C.coef(0) * ldg_nc(c);
-#pragma unroll
-      for (int k = -R; k <= R; ++k)
-        if (k != 0) s = fma(C.coef(star_ci(AX_A, k)), ldg_nc(c + k), s);
-#pragma unroll
-      for (int k = -R; k <= R; ++k)
-        if (k != 0) s = fma(C.coef(star_ci(AX_B, k)), ldg_nc(c + k * g.st_b), s);
-      return s;
-    } else {
-      const double* c = smem + slot * NIN * SLOT + (lb[i] + R) * PA + la[i] + R;
-      double s = C.coef(0) * c[0];
-#pragma unroll
-      for (int k = -R; k <= R; ++k)
-        if (k != 0) s = fma(C.coef(star_ci(AX_A, k)), c[k], s);
-#pragma unroll
-      for (int k = -R; k <= R; ++k)
-        if (k != 0) s = fma(C.coef(star_ci(AX_B, k)), c[k * PA], s);
-      return s;
-    }
-  };
-  auto centre = [&](int i, int slot, int p) -> double {
+  auto plane_ld = [&](int slot, int p) {
     if constexpr (STAGING == 1)
-      return ldg_nc(in + col0 + la[i] + (long long)lb[i] * g.st_b + (long long)p * g.st_s);
+      return GlobPlane{in + col0 + (long long)p * g.st_s, g.st_b};
     else
-      return smem[slot * NIN * SLOT + (lb[i] + R) * PA + la[i] + R];
+      return SmemPlane{smem + slot * NIN * SLOT};
+  };
+  auto store = [&](int ib, int ia, int po, double v) {
+    if (g.a0 + la[ia] < g.n_a && g.b0 + lb[ib] < g.n_b)
+      out[col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)po * g.st_s] = v;
   };
 
 #pragma unroll(UFS)
-  for (int j = 0; j < n_planes; ++j) {
-    const int p = g.s_start - R + j;
-    const int slot = j % NP;
-    if constexpr (STAGING == 3) mbar_wait(&bars[slot], (u32)((j / NP) & 1));
+  for (int j0 = 0; j0 < n_planes; j0 += W) {
+    static_for<0, W>([&](auto UU) {
+      constexpr int u = decltype(UU)::value;
+      const int j = j0 + u;
+      if (j >= n_planes) return;  // CTA-uniform
+      const int p = g.s_start - R + j;
+      const int slot = j % NP;
+      if constexpr (STAGING == 3) mbar_wait(&bars[slot], (u32)((j / NP) & 1));
 
-    if constexpr (RETIME) {
-      // retiming: plane p contributes ws[p-o]*u to outputs o = p-R..p+R and its
-      // in-plane partial sum to output p; output p-R is complete afterwards.
+      if constexpr (KIND == 1 && RETIME) {
+        // retiming: plane p adds ws[p-o]*u to outputs o = p-R..p+R, its in-plane
+        // part to output p; output p-R is then complete.   logical m -> phys (m+u)%W
+        double ip[NCB][NCA], cen[NCB][NCA];
+        star_inplane(C, plane_ld(slot, p), la, lb, ip, cen);
 #pragma unroll
-      for (int i = 0; i < NC; ++i) {
-        const double v = centre(i, slot, p);
+        for (int ib = 0; ib < NCB; ++ib)
 #pragma unroll
-        for (int m = 0; m < W; ++m) {
-          if (m == R) continue;
-          acc[i][m] = fma(C.coef(star_ci(AX_S, R - m)), v, acc[i][m]);
-        }
-        acc[i][R] += inplane(i, slot, p);
-      }
-      if (j >= 2 * R) {
-        const long long so = (long long)(p - R) * g.st_s;
+          for (int ia = 0; ia < NCA; ++ia) {
 #pragma unroll
-        for (int i = 0; i < NC; ++i)
-          if (ok[i]) out[col0 + la[i] + (long long)lb[i] * g.st_b + so] = acc[i][0];
-      }
-#pragma unroll
-      for (int i = 0; i < NC; ++i) {
-#pragma unroll
-        for (int m = 0; m < W - 1; ++m) acc[i][m] = acc[i][m + 1];
-        acc[i][W - 1] = 0.0;
-      }
-    } else {
-      // gather: register queue of the 2R+1 centre values along s (2.5-D blocking)
-#pragma unroll
-      for (int i = 0; i < NC; ++i) {
-#pragma unroll
-        for (int m = 0; m < W - 1; ++m) acc[i][m] = acc[i][m + 1];
-        acc[i][W - 1] = centre(i, slot, p);
-      }
-      if (j >= 2 * R) {
-        const int po = p - R;
-        const int slot_o = (j - R) % NP;
-        const long long so = (long long)po * g.st_s;
-#pragma unroll
-        for (int i = 0; i < NC; ++i) {
-          double s = inplane(i, slot_o, po);
-#pragma unroll
-          for (int k = -R; k <= R; ++k)
-            if (k != 0) s = fma(C.coef(star_ci(AX_S, k)), acc[i][R + k], s);
-          if (ok[i]) out[col0 + la[i] + (long long)lb[i] * g.st_b + so] = s;
-        }
-      }
-    }
-
-    // ---- release the oldest live slot and refill it with plane j + D
-    if constexpr (STAGING == 3) {
-      __syncthreads();
-      if (tid == 0 && j + D < n_planes) {
-        const int sl = (j + D) % NP;
-        fence_proxy_async();
-        mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
-        tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);
-      }
-    } else if constexpr (STAGING == 2) {
-      __syncthreads();
-      if (j + 1 < n_planes) {
-        double* dst = smem + ((j + 1) % NP) * NIN * SLOT;
-        if constexpr (D == 1) {
-          ldst_plane<PA, PB, SLOT>(P, g, dst, p + 1);
-        } else {
-#pragma unroll
-          for (int q = 0; q < FR; ++q) {
-            const int e = tid + q * NTHR;
-            if (e < NIN * PL) dst[e] = frag[q];
-          }
-#pragma unroll
-          for (int f = 0; f < D - 2; ++f)
-#pragma unroll
-            for (int q = 0; q < FR; ++q) frag[f * FR + q] = frag[(f + 1) * FR + q];
-          const int pn = p + D;
-#pragma unroll
-          for (int q = 0; q < FR; ++q) {
-            const int e = tid + q * NTHR;
-            double v = 0.0;
-            if (e < NIN * PL && j + D < n_planes) {
-              const int r = e % PL;
-              const int ga = g.a0 - R + r % PA, gb = g.b0 - R + r / PA;
-              if (ga < g.n_a + R && gb < g.n_b + R)
-                v = in[ga + gb * g.st_b + (long long)pn * g.st_s];
+            for (int m = 0; m < W; ++m) {
+              if (m == R) continue;
+              double& a = acc[ib][ia][(m + u) % W];
+              a = fma(C.coef(star_ci(AX_S, R - m)), cen[ib][ia], a);
             }
-            frag[(D - 2) * FR + q] = v;
+            acc[ib][ia][(R + u) % W] += ip[ib][ia];
           }
+        if (j >= 2 * R) {
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) store(ib, ia, p - R, acc[ib][ia][u % W]);
+        }
+#pragma unroll
+        for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+          for (int ia = 0; ia < NCA; ++ia) acc[ib][ia][u % W] = 0.0;
+      } else if constexpr (KIND == 1) {
+        // gather: register queue of the 2R+1 centre values (2.5-D blocking)
+        // logical q[m] (plane p-2R+m) -> phys (m+u+1)%W ; newest (m = 2R) -> phys u
+        {
+          double cen[NCB][NCA];
+          load_centres(plane_ld(slot, p), la, lb, cen);
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) acc[ib][ia][u % W] = cen[ib][ia];
+        }
+        if (j >= 2 * R) {
+          const int po = p - R;
+          double ip[NCB][NCA], cen[NCB][NCA];
+          star_inplane(C, plane_ld((j - R) % NP, po), la, lb, ip, cen);
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) {
+              double s = ip[ib][ia];
+#pragma unroll
+              for (int k = -R; k <= R; ++k)
+                if (k != 0) s = fma(C.coef(star_ci(AX_S, k)), acc[ib][ia][(R + k + u + 1) % W], s);
+              store(ib, ia, po, s);
+            }
+        }
+      } else if constexpr (KIND == 2 && RETIME) {
+        // box retimed: slices ds = +1, 0, -1 of plane p go to outputs p-1, p, p+1
+        double S[3][NCB][NCA];
+#pragma unroll
+        for (int q = 0; q < 3; ++q)
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) S[q][ib][ia] = 0.0;
+        box_slices<3, R, -1>(C, plane_ld(slot, p), la, lb, S);
+#pragma unroll
+        for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+          for (int ia = 0; ia < NCA; ++ia)
+#pragma unroll
+            for (int m = 0; m < W; ++m) acc[ib][ia][(m + u) % W] += S[m][ib][ia];
+        if (j >= 2 * R) {
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) store(ib, ia, p - R, acc[ib][ia][u % W]);
+        }
+#pragma unroll
+        for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+          for (int ia = 0; ia < NCA; ++ia) acc[ib][ia][u % W] = 0.0;
+      } else if constexpr (KIND == 2) {
+        // box gather: one chain over planes o-1, o, o+1 (oracle order dz, dy, dx)
+        if (j >= 2 * R) {
+          const int po = p - R;
+          double S[1][NCB][NCA];
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) S[0][ib][ia] = 0.0;
+          static_for<0, W>([&](auto QQ) {
+            constexpr int ds = decltype(QQ)::value - R;
+            box_slices<1, ds, 0>(C, plane_ld((j - R + ds) % NP, po + ds), la, lb, S);
+          });
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) store(ib, ia, po, S[0][ib][ia]);
         }
       }
-      __syncthreads();
+
+      // ---- release the oldest live slot and refill it with plane j + D
+      if constexpr (STAGING == 3) {
+        __syncthreads();
+        if (tid == 0 && j + D < n_planes) {
+          const int sl = (j + D) % NP;
+          fence_proxy_async();
+          mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
+          tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);
+        }
+      } else if constexpr (STAGING == 2) {
+        __syncthreads();
+        if (j + 1 < n_planes) {
+          double* dst = smem + ((j + 1) % NP) * NIN * SLOT;
+          if constexpr (D == 1) {
+            ldst_plane(P, g, dst, p + 1);
+          } else {
+#pragma unroll
+            for (int q = 0; q < FR; ++q) {
+              const int e = tid + q * NTHR;
+              if (e < NIN * PL) dst[(e / PL) * SLOT + e % PL] = frag[q];
+            }
+#pragma unroll
+            for (int f = 0; f < D - 2; ++f)
+#pragma unroll
+              for (int q = 0; q < FR; ++q) frag[f * FR + q] = frag[(f + 1) * FR + q];
+#pragma unroll
+            for (int q = 0; q < FR; ++q) {
+              const int e = tid + q * NTHR;
+              frag[(D - 2) * FR + q] =
+                  (e < NIN * PL && j + D < n_planes) ? plane_elem(P, g, e, p + D) : 0.0;
+            }
+          }
+        }
+        __syncthreads();
+      }
+    });
+  }
+}
+
+
+// =============================================================================
+// hypterm-like fast streaming path, T_SD == 1 (Table III "hypterm")
+//   directions: a = x, b = other in-plane dim, s = streamed dim
+//   in-plane terms T_a, T_b from register-blocked windows of the staged plane;
+//   streamed-direction terms from per-plane products E_f scattered into 2R+1 pending
+//   outputs (retiming) or gathered from a 2R+1 register queue.
+// =============================================================================
+constexpr int DA = 0, DB = SZ ? 1 : 2, DS = SZ ? 2 : 1;  // direction (0 x, 1 y, 2 z)
+
+// load a line of values through the point block: along a (x-window of row lb, starting
+// la - XR, length BMA + 2XR) or along b (column la, rows lb - R .., length BMB + 2R)
+template <int AXIS, class LD>
+__device__ __forceinline__ void load_line(const LD& ld, int la, int lb, double* w) {
+  if constexpr (AXIS == 0) {
+    load_xwin(ld, la, lb, w);
+  } else {
+#pragma unroll
+    for (int q = 0; q < BMB + 2 * R; ++q) w[q] = ld.at(la, lb - R + q);
+  }
+}
+
+// T_d[f] (d = DIR, f = 0..4) for the thread's points, d in {a, b}:
+//   T_d[f] = dxinv_d * sum_k a_k e_k[f]   (k = 1..4 ascending, oracle term order)
+template <int AXIS, class LD>
+__device__ __forceinline__ void hyp_inplane(const Ctx& C, const LD* ld, const int* la,
+                                            const int* lb, double (&t)[5][NCB][NCA]) {
+  constexpr int DIR = AXIS == 0 ? DA : DB;
+  constexpr int QD = 4 + DIR;
+  constexpr int LEN = AXIS == 0 ? BMA + 2 * XR : BMB + 2 * R;
+  constexpr int OFF = AXIS == 0 ? XR : R;          // window index of the run's first point
+  constexpr int NL = AXIS == 0 ? NCB * CMA : NCA * CMB;  // lines
+  constexpr int NPL = AXIS == 0 ? BMA : BMB;             // points per line
+  const double dxi = C.coef(4 + DIR);
+#pragma unroll
+  for (int line = 0; line < NL; ++line) {
+    // line -> (run start la0, lb0) and point (ib, ia) of its t-th point
+    const int ib0 = AXIS == 0 ? line / CMA : (line % CMB) * BMB;
+    const int ia0 = AXIS == 0 ? (line % CMA) * BMA : line / CMB;
+    const int la0 = la[ia0], lb0 = lb[ib0];
+    double wq[LEN], w4[LEN], wc[LEN];
+    load_line<AXIS>(ld[QD], la0, lb0, wq);
+    load_line<AXIS>(ld[7], la0, lb0, w4);
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      load_line<AXIS>(ld[m], la0, lb0, wc);
+#pragma unroll
+      for (int pt = 0; pt < NPL; ++pt) {
+        const int ib = AXIS == 0 ? ib0 : ib0 + pt;
+        const int ia = AXIS == 0 ? ia0 + pt : ia0;
+        const int c = OFF + pt;
+        if (m == DIR) {  // mass flux: cons_d(+k) - cons_d(-k)
+          double sum = 0.0;
+#pragma unroll
+          for (int k = 1; k <= 4; ++k) {
+            const double e = wc[c + k] - wc[c - k];
+            sum = (k == 1) ? C.coef(0) * e : fma(C.coef(k - 1), e, sum);
+          }
+          t[0][ib][ia] = dxi * sum;
+        }
+        double sum = 0.0;
+#pragma unroll
+        for (int k = 1; k <= 4; ++k) {
+          double e = fma(wc[c + k], wq[c + k], -(wc[c - k] * wq[c - k]));
+          if (m == 3)
+            e = e + fma(w4[c + k], wq[c + k], -(w4[c - k] * wq[c - k]));
+          else if (m == DIR)
+            e = e + (w4[c + k] - w4[c - k]);
+          sum = (k == 1) ? C.coef(0) * e : fma(C.coef(k - 1), e, sum);
+        }
+        t[m + 1][ib][ia] = dxi * sum;
+      }
     }
+  }
+}
+
+// per-plane streamed-direction products E_f at the thread's points
+template <class LD>
+__device__ __forceinline__ void hyp_products(const LD* ld, const int* la, const int* lb,
+                                             double (&E)[5][NCB][NCA]) {
+  constexpr int QS = 4 + DS;
+#pragma unroll
+  for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+    for (int ia = 0; ia < NCA; ++ia) {
+      const double qs = ld[QS].at(la[ia], lb[ib]);
+      const double q4 = ld[7].at(la[ia], lb[ib]);
+      double cm[4];
+#pragma unroll
+      for (int m = 0; m < 4; ++m) cm[m] = ld[m].at(la[ia], lb[ib]);
+      E[0][ib][ia] = cm[DS];
+#pragma unroll
+      for (int m = 0; m < 3; ++m) E[m + 1][ib][ia] = m == DS ? fma(cm[m], qs, q4) : cm[m] * qs;
+      E[4][ib][ia] = fma(cm[3], qs, q4 * qs);
+    }
+}
+
+__device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double* smem) {
+  Ctx C{P};
+  constexpr int D = PF;
+  constexpr int NP = STAGING == 1 ? 1 : NP1;
+  const SGeo g = stream_geo(P);
+  const int ta = thread_x();
+  const int tb = SZ ? thread_y() : thread_z();
+  const int tid = threadIdx.x;
+  const int n_planes = (g.s_end - g.s_start) + 2 * R;
+  u64* bars = (u64*)(smem + NP * NIN * SLOT);
+
+  int la[NCA], lb[NCB];
+#pragma unroll
+  for (int i = 0; i < NCA; ++i) la[i] = merged_pos(i, ta, TBA, BMA);
+#pragma unroll
+  for (int i = 0; i < NCB; ++i) lb[i] = merged_pos(i, tb, TBB, BMB);
+  const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
+
+  // streamed-direction weights: plane p contributes ws[p-o] * E_f(p) to flux_f(o)
+  double ws[W];
+#pragma unroll
+  for (int k = -R; k <= R; ++k)
+    ws[k + R] = k == 0 ? 0.0 : (k > 0 ? -1.0 : 1.0) * C.coef(4 + DS) * C.coef((k > 0 ? k : -k) - 1);
+
+  double acc[5][NCB][NCA][W];  // retimed: pending fluxes ; gather: queue of E_f
+#pragma unroll
+  for (int f = 0; f < 5; ++f)
+#pragma unroll
+    for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+      for (int ia = 0; ia < NCA; ++ia)
+#pragma unroll
+        for (int m = 0; m < W; ++m) acc[f][ib][ia][m] = 0.0;
+
+  double frag[D > 1 && STAGING == 2 ? (D - 1) * FR : 1];
+  if constexpr (STAGING == 3) {
+    if (tid == 0) {
+      for (int s = 0; s < NP; ++s) mbar_init(&bars[s], 1);
+      fence_mbar_init();
+    }
+    __syncthreads();
+    if (tid == 0) {
+      for (int j = 0; j < D && j < n_planes; ++j) {
+        mbar_arrive_expect_tx(&bars[j % NP], NIN * PL * 8);
+        tma_plane(P, g, smem + (j % NP) * NIN * SLOT, &bars[j % NP], g.s_start - R + j);
+      }
+    }
+  } else if constexpr (STAGING == 2) {
+    ldst_plane(P, g, smem, g.s_start - R);
+    if constexpr (D > 1) {
+#pragma unroll
+      for (int f = 0; f < D - 1; ++f)
+#pragma unroll
+        for (int q = 0; q < FR; ++q) {
+          const int e = tid + q * NTHR;
+          frag[f * FR + q] =
+              (e < NIN * PL && 1 + f < n_planes) ? plane_elem(P, g, e, g.s_start - R + 1 + f) : 0.0;
+        }
+    }
+    __syncthreads();
+  }
+
+  auto loaders = [&](int slot, int p, auto* out8) {
+#pragma unroll
+    for (int a = 0; a < NIN; ++a) {
+      if constexpr (STAGING == 1)
+        out8[a] = GlobPlane{P.in[a] + col0 + (long long)p * g.st_s, g.st_b};
+      else
+        out8[a] = SmemPlane{smem + (slot * NIN + a) * SLOT};
+    }
+  };
+  using LDT = typename Cond<STAGING == 1, GlobPlane, SmemPlane>::type;
+  auto store5 = [&](int ib, int ia, int po, double (&v)[5]) {
+    if (g.a0 + la[ia] < g.n_a && g.b0 + lb[ib] < g.n_b) {
+      const long long off = col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)po * g.st_s;
+#pragma unroll
+      for (int f = 0; f < 5; ++f) P.out[f][off] = v[f];
+    }
+  };
+
+#pragma unroll(UFS)
+  for (int j0 = 0; j0 < n_planes; j0 += W) {
+    static_for<0, W>([&](auto UU) {
+      constexpr int u = decltype(UU)::value;
+      const int j = j0 + u;
+      if (j >= n_planes) return;
+      const int p = g.s_start - R + j;
+      const int slot = j % NP;
+      if constexpr (STAGING == 3) mbar_wait(&bars[slot], (u32)((j / NP) & 1));
+      LDT ld[NIN];
+      loaders(slot, p, ld);
+      double E[5][NCB][NCA];
+      hyp_products(ld, la, lb, E);
+      if constexpr (RETIME) {
+        double ta_[5][NCB][NCA], tb_[5][NCB][NCA];
+        hyp_inplane<0>(C, ld, la, lb, ta_);
+        hyp_inplane<1>(C, ld, la, lb, tb_);
+#pragma unroll
+        for (int f = 0; f < 5; ++f)
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) {
+#pragma unroll
+              for (int m = 0; m < W; ++m) {
+                if (m == R) continue;
+                double& a = acc[f][ib][ia][(m + u) % W];
+                a = fma(ws[2 * R - m], E[f][ib][ia], a);  // k = p - o = R - m
+              }
+              acc[f][ib][ia][(R + u) % W] += -ta_[f][ib][ia] - tb_[f][ib][ia];
+            }
+        if (j >= 2 * R) {
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) {
+              double v[5];
+#pragma unroll
+              for (int f = 0; f < 5; ++f) v[f] = acc[f][ib][ia][u % W];
+              store5(ib, ia, p - R, v);
+            }
+        }
+#pragma unroll
+        for (int f = 0; f < 5; ++f)
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) acc[f][ib][ia][u % W] = 0.0;
+      } else {
+        // gather: queue of E_f, newest at phys u
+#pragma unroll
+        for (int f = 0; f < 5; ++f)
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) acc[f][ib][ia][u % W] = E[f][ib][ia];
+        if (j >= 2 * R) {
+          const int po = p - R;
+          LDT ldo[NIN];
+          loaders((j - R) % NP, po, ldo);
+          double ta_[5][NCB][NCA], tb_[5][NCB][NCA];
+          hyp_inplane<0>(C, ldo, la, lb, ta_);
+          hyp_inplane<1>(C, ldo, la, lb, tb_);
+          const double dxs = C.coef(4 + DS);
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int ia = 0; ia < NCA; ++ia) {
+              double v[5];
+#pragma unroll
+              for (int f = 0; f < 5; ++f) {
+                double sum = 0.0;
+#pragma unroll
+                for (int k = 1; k <= R; ++k) {
+                  const double e = acc[f][ib][ia][(R + k + u + 1) % W] -
+                                   acc[f][ib][ia][(R - k + u + 1) % W];
+                  sum = (k == 1) ? C.coef(0) * e : fma(C.coef(k - 1), e, sum);
+                }
+                v[f] = -ta_[f][ib][ia] - tb_[f][ib][ia] - dxs * sum;
+              }
+              store5(ib, ia, po, v);
+            }
+        }
+      }
+
+      if constexpr (STAGING == 3) {
+        __syncthreads();
+        if (tid == 0 && j + D < n_planes) {
+          const int sl = (j + D) % NP;
+          fence_proxy_async();
+          mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
+          tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);
+        }
+      } else if constexpr (STAGING == 2) {
+        __syncthreads();
+        if (j + 1 < n_planes) {
+          double* dst = smem + ((j + 1) % NP) * NIN * SLOT;
+          if constexpr (D == 1) {
+            ldst_plane(P, g, dst, p + 1);
+          } else {
+#pragma unroll
+            for (int q = 0; q < FR; ++q) {
+              const int e = tid + q * NTHR;
+              if (e < NIN * PL) dst[(e / PL) * SLOT + e % PL] = frag[q];
+            }
+#pragma unroll
+            for (int f = 0; f < D - 2; ++f)
+#pragma unroll
+              for (int q = 0; q < FR; ++q) frag[f * FR + q] = frag[(f + 1) * FR + q];
+#pragma unroll
+            for (int q = 0; q < FR; ++q) {
+              const int e = tid + q * NTHR;
+              frag[(D - 2) * FR + q] =
+                  (e < NIN * PL && j + D < n_planes) ? plane_elem(P, g, e, p + D) : 0.0;
+            }
+          }
+        }
+        __syncthreads();
+      }
+    });
   }
 }
 
@@ -532,9 +1042,6 @@ __device__ __forceinline__ void kernel_star_stream1(const cst_kparams& P, double
 // =============================================================================
 __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, double* smem) {
   Ctx C{P};
-  constexpr int PA = TA + 2 * R, PB = TB + 2 * R;
-  constexpr int PL = PA * PB;
-  constexpr int SLOT = round_slot(PL);
   constexpr int D = PF;
   constexpr int NP = D * TS + 2 * R;
   const SGeo g = stream_geo(P);
@@ -557,7 +1064,7 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
         tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], g.s_start - R + j);
       }
     } else if constexpr (STAGING == 2) {
-      ldst_plane<PA, PB, SLOT>(P, g, smem + sl * NIN * SLOT, g.s_start - R + j);
+      ldst_plane(P, g, smem + sl * NIN * SLOT, g.s_start - R + j);
     }
   };
 
@@ -584,11 +1091,11 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
       const int s = g.s_start + k * TS + ls;
 #pragma unroll(UFB)
       for (int ib = 0; ib < BMB * CMB; ++ib) {
-        const int lb = merged_pos(ib, tb, TBB, BMB);
+        const int lbp = merged_pos(ib, tb, TBB, BMB);
 #pragma unroll(UFA)
         for (int ia = 0; ia < BMA * CMA; ++ia) {
-          const int la = merged_pos(ia, ta, TBA, BMA);
-          const int a = g.a0 + la, b = g.b0 + lb;
+          const int lap = merged_pos(ia, ta, TBA, BMA);
+          const int a = g.a0 + lap, b = g.b0 + lbp;
           if (a >= g.n_a || b >= g.n_b || s >= g.s_end) continue;
           const long long off = a + b * g.st_b + (long long)s * g.st_s;
           double o[NOUT];
@@ -601,8 +1108,8 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
             const int jp = s - g.s_start + R;  // sequence index of the point's plane
             auto U = [&](int arr, int dx, int dy, int dz) {
               const int da = dx, db = SZ ? dy : dz, ds = SZ ? dz : dy;
-              return smem[((jp + ds) % NP) * NIN * SLOT + arr * SLOT + (lb + R + db) * PA +
-                          la + R + da];
+              return smem[((jp + ds) % NP) * NIN * SLOT + arr * SLOT + (lbp + R + db) * PA +
+                          lap + XR + da];
             };
             point(C, U, o);
           }
@@ -626,8 +1133,10 @@ extern "C" __global__ void __launch_bounds__(NTHR) cst_kernel(const __grid_const
   extern __shared__ __align__(128) double cst_smem[];
   if constexpr (!STREAM) {
     kernel_tile3d(P, cst_smem);
-  } else if constexpr (KIND == 1 && TS == 1) {
-    kernel_star_stream1(P, cst_smem);
+  } else if constexpr (KIND != 3 && TS == 1) {
+    kernel_stream1(P, cst_smem);
+  } else if constexpr (KIND == 3 && TS == 1) {
+    kernel_hyp_stream1(P, cst_smem);
   } else {
     kernel_stream_generic(P, cst_smem);
   }

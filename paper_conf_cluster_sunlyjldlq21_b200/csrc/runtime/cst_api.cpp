@@ -81,6 +81,7 @@ static Geometry geometry(const StencilInfo& st, const Tuple& t, int64_t nx, int6
                          int64_t nz) {
   Geometry g{};
   const int r = st.r;
+  const int xr = r + (r & 1);  // even x halo of the smem/TMA boxes (kernels' XR)
   int64_t T[3];
   for (int d = 0; d < 3; ++d) T[d] = (int64_t)t[F_TBX + d] * t[F_BMX + d] * t[F_CMX + d];
   g.threads = (unsigned)(t[F_TBX] * t[F_TBY] * t[F_TBZ]);
@@ -92,7 +93,7 @@ static Geometry geometry(const StencilInfo& st, const Tuple& t, int64_t nx, int6
     g.tiles_c = 1;
     g.grid_x = (unsigned)(g.tiles_a * (int64_t)g.tiles_b);
     g.grid_y = (unsigned)g.chunks;
-    g.box[0] = (int)T[0] + 2 * r;
+    g.box[0] = (int)T[0] + 2 * xr;
     if (sz) {
       g.box[1] = (int)T[1] + 2 * r;
       g.box[2] = 1;
@@ -107,7 +108,7 @@ static Geometry geometry(const StencilInfo& st, const Tuple& t, int64_t nx, int6
     g.chunks = 1;
     g.grid_x = (unsigned)(g.tiles_a * (int64_t)g.tiles_b);
     g.grid_y = (unsigned)g.tiles_c;
-    for (int d = 0; d < 3; ++d) g.box[d] = (int)T[d] + 2 * r;
+    for (int d = 0; d < 3; ++d) g.box[d] = (int)T[d] + 2 * (d == 0 ? xr : r);
   }
   return g;
 }

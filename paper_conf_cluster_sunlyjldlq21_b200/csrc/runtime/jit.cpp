@@ -75,7 +75,7 @@ cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
                      double* compile_s) {
   const std::string src = prefix_for(st, t);
   static const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo",
-                               "--fmad=true", "-DCST_NVRTC=1"};
+                               "--fmad=true", "-default-device", "-DCST_NVRTC=1"};
   const int nopts = sizeof(opts) / sizeof(opts[0]);
   int nv_major = 0, nv_minor = 0;
   nvrtcVersion(&nv_major, &nv_minor);

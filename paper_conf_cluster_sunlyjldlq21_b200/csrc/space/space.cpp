@@ -91,17 +91,26 @@ int64_t model_smem_bytes(int kind, int r, const Tuple& t) {
 }
 
 int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
+  // mirrors csrc/kernels/cst_kernels.cuh: x halo XR = r rounded up to even
   if (t[F_STAGING] == 1) return 0;
+  const int64_t XR = r + (r & 1);
   int64_t T[3];
   tiles(t, T);
-  int64_t P, NP;
-  plane_geometry(kind, r, t, &P, &NP);
-  const int64_t plane = (P * 8 + 127) / 128 * 128;
-  if (t[F_STREAM] == 2) {
+  int64_t plane_elems, NP;
+  if (t[F_STREAM] == 1) {
+    plane_elems = (T[0] + 2 * XR) * (T[1] + 2 * r) * (T[2] + 2 * r);
+    NP = 1;
+  } else {
     const int sd = t[F_SD] - 1;
-    // only the star has the T_SD == 1 fast path so far; others run the generic ring
-    if (!(kind == CST_STAR && T[sd] == 1)) NP = (int64_t)t[F_PF] * T[sd] + 2 * r;
+    const int b = sd == 2 ? 1 : 2;
+    plane_elems = (T[0] + 2 * XR) * (T[b] + 2 * r);
+    const int64_t D = t[F_PF];
+    if (kind != CST_HYPTERM && T[sd] == 1)
+      NP = D + (t[F_RET] == 2 ? 0 : retention(kind, r));
+    else
+      NP = D * T[sd] + 2 * r;
   }
+  const int64_t plane = (plane_elems * 8 + 127) / 128 * 128;
   const int64_t bars = t[F_STAGING] == 3 ? NP * 8 : 0;
   return n_arrays(kind) * NP * plane + bars;
 }
