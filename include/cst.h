@@ -183,7 +183,9 @@ typedef struct {
   double time_budget_s;      /* 100; <= 0 = unlimited                   */
   int32_t reps;              /* timed reps per evaluation (median)              */
   int32_t warmup;            /* untimed sweeps per evaluation                   */
-  const char* log_path;      /* JSONL log, or NULL                              */
+  const char* log_path;      /* JSON report of every stage, or NULL              */
+  int32_t n_user_metrics;    /* metrics supplied by the eval callback (0 = model) */
+  int32_t quantile_sample;   /* settings sampled to set thresholds / gene tables  */
 } cst_tune_opts;
 
 typedef struct {
@@ -202,12 +204,13 @@ void cst_tune_opts_default(cst_tune_opts* o);
 
 /* Evaluation callback: fitness of `n` candidate settings (e.g. spread over GPUs by the
  * caller — population-parallel evaluation).  Must write ms[i] (> 0, or
- * <= 0 / inf for an invalid or failed candidate).  Returns 0 on success. */
-typedef int (*cst_eval_fn)(void* user, const cst_setting* settings, int32_t n, double* ms);
+ * <= 0 / inf for an invalid or failed candidate).  If opts->n_user_metrics > 0 it must
+ * also write metrics[i * n_user_metrics + k] (the dataset's "GPU metrics");
+ * otherwise metrics is NULL and the tuner uses its modelled features.
+ * Returns 0 on success. */
+typedef int (*cst_eval_fn)(void* user, const cst_setting* settings, int32_t n, double* ms,
+                           double* metrics);
 
-/* Synchronous.  Evaluates candidates on the handle's device using `in`/`scratch_out`
- * (device buffers as for cst_sweep) unless `eval` is non-NULL, in which case every
- * batch of candidates is handed to it.  Writes the best setting and a report. */
 cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const double* const* in,
                     double* const* scratch_out, cst_eval_fn eval, void* eval_user,
                     cst_setting* best, cst_tune_report* rep);

@@ -66,10 +66,18 @@ def encode(field: str, v: int) -> float:
 
 
 def cv(values) -> float:
-    """Eq. 1: population standard deviation over mean; 0 when sigma == 0."""
-    x = np.asarray(values, dtype=np.float64)
-    mu = x.mean()
-    sigma = math.sqrt(float(np.mean((x - mu) ** 2)))
+    """Eq. 1: population standard deviation over mean; 0 when sigma == 0.
+    Plain sequential sums (the C++ tuner sums in the same order)."""
+    x = [float(v) for v in values]
+    n = float(len(x))
+    s = 0.0
+    for v in x:
+        s += v
+    mu = s / n
+    q = 0.0
+    for v in x:
+        q += (v - mu) * (v - mu)
+    sigma = math.sqrt(q / n)
     if sigma == 0.0:
         return 0.0
     return sigma / mu
@@ -142,14 +150,26 @@ def group_parameters(dq: deque) -> list[list[int]]:
 
 
 def pcc(x, y) -> float:
-    """Eq. 2 (garbled; Q10): the standard Pearson correlation coefficient."""
-    x = np.asarray(x, dtype=np.float64)
-    y = np.asarray(y, dtype=np.float64)
-    dx, dy = x - x.mean(), y - y.mean()
-    sx, sy = math.sqrt(float(np.sum(dx * dx))), math.sqrt(float(np.sum(dy * dy)))
-    if sx == 0.0 or sy == 0.0:
+    """Eq. 2 (garbled; Q10): the standard Pearson correlation coefficient
+    (sequential sums)."""
+    x = [float(v) for v in x]
+    y = [float(v) for v in y]
+    n = float(len(x))
+    sx = sy = 0.0
+    for a, b in zip(x, y):
+        sx += a
+        sy += b
+    mx, my = sx / n, sy / n
+    sxy = sxx = syy = 0.0
+    for a, b in zip(x, y):
+        dx, dy = a - mx, b - my
+        sxy += dx * dy
+        sxx += dx * dx
+        syy += dy * dy
+    ax, ay = math.sqrt(sxx), math.sqrt(syy)
+    if ax == 0.0 or ay == 0.0:
         return 0.0
-    return float(np.sum(dx * dy)) / (sx * sy)
+    return sxy / (ax * ay)
 
 
 def metric_pairs(metrics: np.ndarray):
@@ -230,7 +250,9 @@ def pmnf_fit(groups, X: np.ndarray, y: np.ndarray):
         A = pmnf_features(groups, X, i, j)
         coef, rank = lstsq_rank(A, y)
         resid = y - A @ coef
-        ssr = float(np.sum(resid * resid))
+        ssr = 0.0
+        for e in resid:
+            ssr += float(e) * float(e)
         dof = m - rank
         rse = math.sqrt(ssr / dof) if dof > 0 else float("inf")
         fits.append((i, j, coef, rse))

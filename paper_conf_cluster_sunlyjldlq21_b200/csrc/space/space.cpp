@@ -105,7 +105,7 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
     const int b = sd == 2 ? 1 : 2;
     plane_elems = (T[0] + 2 * XR) * (T[b] + 2 * r);
     const int64_t D = t[F_PF];
-    if (kind != CST_HYPTERM && T[sd] == 1)
+    if (T[sd] == 1)
       NP = D + (t[F_RET] == 2 ? 0 : retention(kind, r));
     else
       NP = D * T[sd] + 2 * r;

@@ -1,0 +1,900 @@
+// tuner.cpp — csTuner (Sun et al., CLUSTER'21) as host C++: P:n = PAPER.md line n.
+//
+//   1. dataset: 128 seeded random settings, evaluated with metrics
+//   2. pair CVs (Eq. 1) from the dataset + Algorithm 1 grouping
+//   3. metric PCCs (Eq. 2) + Algorithm 2 combination + selection
+//   4. PMNF surrogate per selected metric (Eq. 3), min-RSE hypothesis
+//   5. threshold filter -> sampled space (10 %)
+//   6. re-indexing of each group's valid value tuples
+//   7. grouped multi-population GA with CV_top-n approximation stop
+// Readings of the garbled / silent parts: DESIGN.md §5.  Steps 1-6
+// are bit-exact with oracle/tuner.py (plain sequential sums; built -ffp-contract=off);
+// the GA is pinned by properties (exhaustive fallback, synthetic optimum, determinism).
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <deque>
+#include <fstream>
+#include <map>
+#include <set>
+#include <sstream>
+#include <thread>
+
+#include "../runtime/internal.h"
+
+namespace cst {
+namespace tune {
+
+static const uint64_t GOLDEN = 0x9E3779B97F4A7C15ULL;
+
+static uint64_t sm64(uint64_t x) {
+  uint64_t z = x + GOLDEN;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+  return z ^ (z >> 31);
+}
+
+// Counter-based RNG (splitmix64 stream) for the GA.
+struct Rng {
+  uint64_t key, ctr = 0;
+  explicit Rng(uint64_t seed) : key(sm64(seed ^ 0xC0FFEE1234567ULL)) {}
+  uint64_t next() { return sm64(key + (ctr++)); }
+  double uniform() { return (double)(next() >> 11) * 0x1.0p-53; }
+};
+
+// Dataset sampler (oracle.tuner.sample_ranks): distinct idx = (u * count) >> 64.
+std::vector<uint64_t> sample_ranks(uint64_t seed, uint64_t count, uint64_t n) {
+  std::vector<uint64_t> out;
+  if (count <= n) {
+    for (uint64_t i = 0; i < count; ++i) out.push_back(i);
+    return out;
+  }
+  const uint64_t base = sm64(seed);
+  std::set<uint64_t> seen;
+  for (uint64_t i = 0; out.size() < n; ++i) {
+    const uint64_t u = sm64(base + i);
+    const uint64_t idx = (uint64_t)(((unsigned __int128)u * count) >> 64);
+    if (seen.insert(idx).second) out.push_back(idx);
+  }
+  return out;
+}
+
+static bool pow2_field(int f) {
+  return f == F_TBX || f == F_TBY || f == F_TBZ || f == F_SB || (f >= F_UFX && f <= F_BMZ);
+}
+static double encode(int f, int32_t v) { return pow2_field(f) ? std::log2((double)v) : (double)v; }
+
+// Eq. 1: population sigma / mean; 0 when sigma == 0 (sequential sums).
+double cv(const std::vector<double>& x) {
+  const double n = (double)x.size();
+  double s = 0;
+  for (double v : x) s += v;
+  const double mu = s / n;
+  double q = 0;
+  for (double v : x) q += (v - mu) * (v - mu);
+  const double sigma = std::sqrt(q / n);
+  if (sigma == 0.0) return 0.0;
+  return sigma / mu;
+}
+
+// Eq. 2 (Q10): Pearson r; 0 if either series is constant.
+double pcc(const std::vector<double>& x, const std::vector<double>& y) {
+  const double n = (double)x.size();
+  double sx = 0, sy = 0;
+  for (size_t i = 0; i < x.size(); ++i) {
+    sx += x[i];
+    sy += y[i];
+  }
+  const double mx = sx / n, my = sy / n;
+  double sxy = 0, sxx = 0, syy = 0;
+  for (size_t i = 0; i < x.size(); ++i) {
+    const double dx = x[i] - mx, dy = y[i] - my;
+    sxy += dx * dy;
+    sxx += dx * dx;
+    syy += dy * dy;
+  }
+  const double a = std::sqrt(sxx), b = std::sqrt(syy);
+  if (a == 0.0 || b == 0.0) return 0.0;
+  return sxy / (a * b);
+}
+
+using Pair = std::pair<int, int>;
+
+// Deque ordered by ascending score, ties in input order.
+std::deque<Pair> ascending(const std::vector<std::pair<Pair, double>>& v, bool absval) {
+  std::vector<size_t> idx(v.size());
+  for (size_t i = 0; i < v.size(); ++i) idx[i] = i;
+  std::stable_sort(idx.begin(), idx.end(), [&](size_t a, size_t b) {
+    const double sa = absval ? std::fabs(v[a].second) : v[a].second;
+    const double sb = absval ? std::fabs(v[b].second) : v[b].second;
+    return sa < sb;
+  });
+  std::deque<Pair> d;
+  for (size_t i : idx) d.push_back(v[i].first);
+  return d;
+}
+
+static int where(const std::vector<std::vector<int>>& g, int p) {
+  for (size_t i = 0; i < g.size(); ++i)
+    for (int q : g[i])
+      if (q == p) return (int)i;
+  return -1;
+}
+
+// Algorithm 1, text reading (Q6).
+std::vector<std::vector<int>> group_parameters(std::deque<Pair> dq) {
+  std::vector<std::vector<int>> groups;
+  const size_t n = dq.size();
+  for (size_t i = 0; i < n; ++i) {
+    if (i % 2 == 0) {
+      const Pair p = dq.front();
+      dq.pop_front();
+      const int ga = where(groups, p.first), gb = where(groups, p.second);
+      if (ga < 0 && gb < 0) groups.push_back({p.first, p.second});
+      else if (ga >= 0 && gb >= 0) continue;
+      else if (ga >= 0) groups[ga].push_back(p.second);
+      else groups[gb].push_back(p.first);
+    } else {
+      const Pair p = dq.back();
+      dq.pop_back();
+      if (where(groups, p.first) >= 0 && where(groups, p.second) >= 0) continue;
+      if (where(groups, p.first) < 0) groups.push_back({p.first});
+      if (where(groups, p.second) < 0) groups.push_back({p.second});
+    }
+  }
+  return groups;
+}
+
+// Algorithm 2 (Q11).
+std::vector<std::vector<int>> combine_metrics(std::deque<Pair> dq, int num_collections) {
+  std::vector<std::vector<int>> cols;
+  while (!dq.empty()) {
+    const Pair p = dq.back();
+    dq.pop_back();
+    const int ca = where(cols, p.first), cb = where(cols, p.second);
+    if (ca < 0 && cb < 0) {
+      if ((int)cols.size() < num_collections) cols.push_back({p.first, p.second});
+      continue;
+    }
+    if (ca >= 0 && cb >= 0) continue;
+    if (ca >= 0) cols[ca].push_back(p.second);
+    else cols[cb].push_back(p.first);
+  }
+  return cols;
+}
+
+// ------------------------------------------------------------------ PMNF (Eq. 3)
+struct Fit {
+  int i = 0, j = 0;
+  std::vector<double> coef;
+  double rse = 0;
+  int rank = 0;
+};
+
+static double feature(const std::vector<int>& g, const Tuple& t, int i, int j) {
+  double col = 1.0;
+  for (int l : g) {
+    const double p = (double)t[l];
+    col = col * std::pow(p, i) * std::pow(std::log2(p), j);
+  }
+  return col;
+}
+
+// Least squares by Householder QR with column pivoting; numerical rank with
+// tol = max(m, n) * eps * |R00| (LAPACK-lstsq-like); dropped columns get coefficient 0.
+static void lstsq(std::vector<std::vector<double>> A, std::vector<double> y, int m, int n,
+                  std::vector<double>* coef, int* rank) {
+  std::vector<int> perm(n);
+  for (int c = 0; c < n; ++c) perm[c] = c;
+  std::vector<double> norms(n);
+  auto colnorm = [&](int c, int k) {
+    double s = 0;
+    for (int r = k; r < m; ++r) s += A[r][c] * A[r][c];
+    return s;
+  };
+  int kmax = std::min(m, n);
+  double r00 = 0;
+  int rk = 0;
+  for (int k = 0; k < kmax; ++k) {
+    int best = k;
+    double bn = -1;
+    for (int c = k; c < n; ++c) {
+      const double s = colnorm(c, k);
+      if (s > bn) {
+        bn = s;
+        best = c;
+      }
+    }
+    if (best != k) {
+      for (int r = 0; r < m; ++r) std::swap(A[r][k], A[r][best]);
+      std::swap(perm[k], perm[best]);
+    }
+    const double nrm = std::sqrt(bn);
+    if (k == 0) r00 = nrm;
+    const double tol = (double)std::max(m, n) * 2.220446049250313e-16 * r00;
+    if (nrm <= tol || nrm == 0.0) break;
+    const double alpha = A[k][k] > 0 ? -nrm : nrm;
+    std::vector<double> v(m, 0.0);
+    for (int r = k; r < m; ++r) v[r] = A[r][k];
+    v[k] -= alpha;
+    double vn = 0;
+    for (int r = k; r < m; ++r) vn += v[r] * v[r];
+    if (vn > 0) {
+      for (int c = k; c < n; ++c) {
+        double d = 0;
+        for (int r = k; r < m; ++r) d += v[r] * A[r][c];
+        const double f = 2 * d / vn;
+        for (int r = k; r < m; ++r) A[r][c] -= f * v[r];
+      }
+      double d = 0;
+      for (int r = k; r < m; ++r) d += v[r] * y[r];
+      const double f = 2 * d / vn;
+      for (int r = k; r < m; ++r) y[r] -= f * v[r];
+    }
+    ++rk;
+  }
+  std::vector<double> x(n, 0.0);
+  for (int k = rk - 1; k >= 0; --k) {
+    double s = y[k];
+    for (int c = k + 1; c < rk; ++c) s -= A[k][c] * x[c];
+    x[k] = s / A[k][k];
+  }
+  coef->assign(n, 0.0);
+  for (int k = 0; k < rk; ++k) (*coef)[perm[k]] = x[k];
+  *rank = rk;
+}
+
+std::vector<Fit> pmnf_fit(const std::vector<std::vector<int>>& groups,
+                          const std::vector<Tuple>& X, const std::vector<double>& y, int* best) {
+  std::vector<Fit> fits;
+  const int m = (int)X.size(), n = (int)groups.size();
+  for (int i = 0; i <= 2; ++i)
+    for (int j = 0; j <= 1; ++j) {
+      std::vector<std::vector<double>> A(m, std::vector<double>(n));
+      for (int r = 0; r < m; ++r)
+        for (int c = 0; c < n; ++c) A[r][c] = feature(groups[c], X[r], i, j);
+      Fit f;
+      f.i = i;
+      f.j = j;
+      lstsq(A, y, m, n, &f.coef, &f.rank);
+      double ssr = 0;
+      for (int r = 0; r < m; ++r) {
+        double pred = 0;
+        for (int c = 0; c < n; ++c) pred += A[r][c] * f.coef[c];
+        const double e = y[r] - pred;
+        ssr += e * e;
+      }
+      const int dof = m - f.rank;
+      f.rse = dof > 0 ? std::sqrt(ssr / dof) : INFINITY;
+      fits.push_back(f);
+    }
+  *best = 0;
+  for (size_t k = 1; k < fits.size(); ++k)
+    if (fits[k].rse < fits[*best].rse) *best = (int)k;
+  return fits;
+}
+
+double pmnf_predict(const std::vector<std::vector<int>>& groups, const Fit& f, const Tuple& t) {
+  double s = 0;
+  for (size_t c = 0; c < groups.size(); ++c) s += feature(groups[c], t, f.i, f.j) * f.coef[c];
+  return s;
+}
+
+// ------------------------------------------------------------------ modelled metrics (Q22)
+static const char* const kModelMetricNames[] = {
+    "hbm_bytes_per_pt", "l2_bytes_per_pt", "smem_bytes",  "regs",         "threads",
+    "ctas",             "ctas_per_sm",     "waves",       "pts_per_thread", "smem_loads_per_pt"};
+static const int kModelMetrics = 10;
+
+std::vector<double> model_metrics(const cst_stencil* h, const Tuple& t) {
+  const int kind = h->info.kind, r = h->info.r;
+  const int nin = kind == CST_HYPTERM ? 8 : 1, nout = kind == CST_HYPTERM ? 5 : 1;
+  const int64_t* M = h->info.M;
+  double T[3];
+  for (int d = 0; d < 3; ++d) T[d] = (double)t[F_TBX + d] * t[F_BMX + d] * t[F_CMX + d];
+  const double thr = (double)t[F_TBX] * t[F_TBY] * t[F_TBZ];
+  const bool stream = t[F_STREAM] == 2;
+  const int sd = t[F_SD] - 1;
+  double over = 1.0, halo = 1.0, ctas = 1.0;
+  if (stream) {
+    const double ns = (double)M[sd];
+    const double chunks = std::ceil(ns / t[F_SB]);
+    over = (ns + 2.0 * r * chunks) / ns;
+    int a = -1, b = -1;
+    for (int d = 0; d < 3; ++d)
+      if (d != sd) (a < 0 ? a : b) = d;
+    halo = (T[a] + 2 * r) * (T[b] + 2 * r) / (T[a] * T[b]);
+    ctas = std::ceil(M[a] / T[a]) * std::ceil(M[b] / T[b]) * chunks;
+  } else {
+    halo = (T[0] + 2 * r) * (T[1] + 2 * r) * (T[2] + 2 * r) / (T[0] * T[1] * T[2]);
+    ctas = std::ceil(M[0] / T[0]) * std::ceil(M[1] / T[1]) * std::ceil(M[2] / T[2]);
+  }
+  const double smem = (double)model_smem_bytes(kind, r, t);
+  const double regs = (double)model_regs(kind, r, t);
+  double occ = std::min(32.0, std::floor(2048.0 / thr));
+  occ = std::min(occ, std::floor(65536.0 / (std::max(regs, 24.0) * thr)));
+  if (smem > 0) occ = std::min(occ, std::floor(233472.0 / (smem + 1024.0)));
+  occ = std::max(occ, 1.0);
+  const double waves = ctas / (148.0 * occ);
+  const double ppt = (double)t[F_BMX] * t[F_CMX] * t[F_BMY] * t[F_CMY] * t[F_BMZ] * t[F_CMZ];
+  const double bma = t[F_BMX], bmb = stream ? (sd == 2 ? t[F_BMY] : t[F_BMZ]) : t[F_BMY];
+  double loads = 0;
+  if (kind == CST_STAR) loads = (bma + 2 * r) / bma + 2.0 * r / bmb;
+  else if (kind == CST_BOX) loads = (bma + 2) * (bmb + 2) / (bma * bmb);
+  else loads = 6 * ((bma + 8) / bma + (bmb + 8) / bmb) + 2;
+  if (!stream) loads = (kind == CST_BOX ? 27 : (kind == CST_STAR ? 6 * r + 1 : 100));
+  return {8.0 * (nin * over + nout), 8.0 * (nin * over * halo + nout), smem, regs, thr, ctas,
+          occ, waves, ppt, loads};
+}
+
+// ------------------------------------------------------------------ JSON log helpers
+struct Json {
+  std::ostringstream o;
+  bool first = true;
+  void key(const std::string& k) {
+    o << (first ? "" : ",\n ") << "\"" << k << "\": ";
+    first = false;
+  }
+  static std::string num(double v) {
+    if (std::isnan(v)) return "null";
+    if (std::isinf(v)) return v > 0 ? "1e308" : "-1e308";
+    char b[64];
+    std::snprintf(b, sizeof b, "%.17g", v);
+    return b;
+  }
+};
+
+}  // namespace tune
+}  // namespace cst
+
+using namespace cst;
+using namespace cst::tune;
+
+extern "C" void cst_tune_opts_default(cst_tune_opts* o) {
+  if (!o) return;
+  o->seed = 1;
+  o->dataset_size = 128;
+  o->sampling_ratio = 0.10;
+  o->n_subpops = 2;
+  o->subpop_size = 16;
+  o->crossover = 0.8;
+  o->mutation = 0.005;
+  o->top_n = 10;
+  o->cv_threshold = 0.02;
+  o->max_generations = 50;
+  o->num_collections = 3;
+  o->time_budget_s = 100.0;
+  o->reps = 5;
+  o->warmup = 2;
+  o->log_path = nullptr;
+  o->n_user_metrics = 0;
+  o->quantile_sample = 65536;
+}
+
+namespace {
+
+struct EvalResult {
+  double ms = INFINITY;
+  std::vector<double> metrics;
+};
+
+struct Evaluator {
+  cst_stencil* h;
+  const cst_tune_opts* o;
+  const double* const* in;
+  double* const* out;
+  cst_eval_fn cb;
+  void* user;
+  std::map<Tuple, EvalResult> memo;
+  double eval_s = 0, jit_s = 0;
+  uint64_t jit_before = 0;
+  cudaStream_t stream = nullptr;
+  cst_status err = CST_OK;
+
+  int n_metrics() const { return o->n_user_metrics > 0 ? o->n_user_metrics : kModelMetrics; }
+
+  // evaluate (memoised) a batch; invalid settings (rules) get ms = inf without timing
+  cst_status run(const std::vector<Tuple>& cands, std::vector<EvalResult>* res) {
+    std::vector<Tuple> todo;
+    std::set<Tuple> seen;
+    for (const Tuple& t : cands)
+      if (!memo.count(t) && !seen.count(t) && check_rules(h->info, t) == nullptr) {
+        todo.push_back(t);
+        seen.insert(t);
+      }
+    const auto t0 = std::chrono::steady_clock::now();
+    if (!todo.empty()) {
+      std::vector<cst_setting> ss;
+      for (const Tuple& t : todo) ss.push_back(from_tuple(t));
+      std::vector<double> ms(todo.size(), INFINITY);
+      std::vector<double> met;
+      if (cb) {
+        if (o->n_user_metrics > 0) met.assign(todo.size() * o->n_user_metrics, 0.0);
+        if (cb(user, ss.data(), (int32_t)ss.size(), ms.data(),
+               o->n_user_metrics > 0 ? met.data() : nullptr) != 0)
+          return fail(CST_E_INTERNAL, "tuner: evaluation callback failed");
+      } else {
+        // code generation of the batch in parallel (NVRTC is thread-safe), then timing
+        const auto j0 = std::chrono::steady_clock::now();
+        const unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+        std::vector<std::thread> pool;
+        std::atomic<size_t> next{0};
+        for (unsigned w = 0; w < nt; ++w)
+          pool.emplace_back([&] {
+            for (size_t i = next++; i < ss.size(); i = next++) {
+              double cs = 0;
+              cst_variant_compile(h, &ss[i], &cs);
+            }
+          });
+        for (auto& th : pool) th.join();
+        jit_s += std::chrono::duration<double>(std::chrono::steady_clock::now() - j0).count();
+        for (size_t i = 0; i < ss.size(); ++i) {
+          double m = INFINITY;
+          const cst_status st = cst_time_setting(h, &ss[i], in, out, o->warmup,
+                                                 std::max(1, o->reps), stream, &m);
+          if (st == CST_E_CUDA) return st;  // sticky device error: stop
+          ms[i] = st == CST_OK ? m : INFINITY;
+        }
+      }
+      for (size_t i = 0; i < todo.size(); ++i) {
+        EvalResult r;
+        r.ms = (ms[i] > 0 && std::isfinite(ms[i])) ? ms[i] : INFINITY;
+        if (o->n_user_metrics > 0)
+          r.metrics.assign(met.begin() + i * o->n_user_metrics,
+                           met.begin() + (i + 1) * o->n_user_metrics);
+        else
+          r.metrics = model_metrics(h, todo[i]);
+        memo[todo[i]] = r;
+      }
+    }
+    eval_s += std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    res->clear();
+    for (const Tuple& t : cands) {
+      auto it = memo.find(t);
+      if (it != memo.end()) res->push_back(it->second);
+      else {
+        EvalResult r;
+        r.metrics.assign(n_metrics(), 0.0);
+        res->push_back(r);  // invalid: fitness 0
+      }
+    }
+    return CST_OK;
+  }
+};
+
+double fitness_of(const EvalResult& r) { return std::isfinite(r.ms) ? 1.0 / r.ms : 0.0; }
+
+}  // namespace
+
+extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const double* const* in,
+                               double* const* scratch_out, cst_eval_fn eval, void* eval_user,
+                               cst_setting* best_out, cst_tune_report* rep) {
+  if (!h || !o || !best_out || !rep) return fail(CST_E_INVALID, "null argument");
+  if (!eval && (!in || !scratch_out))
+    return fail(CST_E_INVALID, "cst_tune: device buffers required without an eval callback");
+  if (o->dataset_size < 4 || o->n_subpops < 1 || o->subpop_size < 4 || o->top_n < 2 ||
+      o->num_collections < 1 || o->sampling_ratio <= 0 || o->sampling_ratio > 1)
+    return fail(CST_E_INVALID, "cst_tune: bad options");
+  const auto wall0 = std::chrono::steady_clock::now();
+  auto elapsed = [&] {
+    return std::chrono::duration<double>(std::chrono::steady_clock::now() - wall0).count();
+  };
+  if (!h->space) h->space.reset(new Space(h->info));
+  const Space& S = *h->space;
+  const uint64_t count = S.count();
+  if (count == 0) return fail(CST_E_CONSTRAINT, "empty parameter space");
+
+  Evaluator ev{h, o, in, scratch_out, eval, eval_user};
+  ev.jit_before = jit_compile_count();
+  if (!eval) {
+    CST_CUDA(cudaSetDevice(h->device));
+    CST_CUDA(cudaStreamCreateWithFlags(&ev.stream, cudaStreamNonBlocking));
+  }
+  struct StreamGuard {
+    cudaStream_t s;
+    ~StreamGuard() {
+      if (s) cudaStreamDestroy(s);
+    }
+  } guard{ev.stream};
+
+  Json js;
+  js.o << "{";
+
+  // ---- 1. dataset
+  const std::vector<uint64_t> ranks = sample_ranks(o->seed, count, (uint64_t)o->dataset_size);
+  std::vector<Tuple> rows;
+  for (uint64_t rk : ranks) {
+    Tuple t;
+    S.at(rk, &t);
+    rows.push_back(t);
+  }
+  std::vector<EvalResult> res;
+  cst_status st = ev.run(rows, &res);
+  if (st != CST_OK) return st;
+  const double t_dataset = elapsed();
+  // statistics use the valid rows only
+  std::vector<int> valid;
+  for (size_t i = 0; i < rows.size(); ++i)
+    if (std::isfinite(res[i].ms)) valid.push_back((int)i);
+  if (valid.size() < 4) return fail(CST_E_INTERNAL, "tuner: fewer than 4 valid dataset rows");
+  js.key("dataset");
+  js.o << "{\"ranks\": [";
+  for (size_t i = 0; i < ranks.size(); ++i) js.o << (i ? "," : "") << ranks[i];
+  js.o << "], \"ms\": [";
+  for (size_t i = 0; i < res.size(); ++i) js.o << (i ? "," : "") << Json::num(res[i].ms);
+  js.o << "], \"metrics\": [";
+  for (size_t i = 0; i < res.size(); ++i) {
+    js.o << (i ? "," : "") << "[";
+    for (size_t k = 0; k < res[i].metrics.size(); ++k)
+      js.o << (k ? "," : "") << Json::num(res[i].metrics[k]);
+    js.o << "]";
+  }
+  js.o << "]}";
+
+  const auto pre0 = std::chrono::steady_clock::now();
+  // ---- 2. pair CVs (Eq. 1, Q8: dataset-only) + Algorithm 1
+  std::vector<std::pair<Pair, double>> cvs;
+  for (int a = 0; a < F_COUNT; ++a)
+    for (int b = 0; b < F_COUNT; ++b) {
+      if (a == b) continue;
+      std::set<int32_t> vals;
+      for (int i : valid) vals.insert(rows[i][a]);
+      std::vector<double> vs;
+      for (int32_t v : vals) {
+        int bi = -1;
+        for (int i : valid) {
+          if (rows[i][a] != v) continue;
+          if (bi < 0) {
+            bi = i;
+            continue;
+          }
+          const double fi = fitness_of(res[i]), fb = fitness_of(res[bi]);
+          if (fi > fb || (fi == fb && ranks[i] < ranks[bi])) bi = i;
+        }
+        vs.push_back(encode(b, rows[bi][b]));
+      }
+      cvs.push_back({{a, b}, cv(vs)});
+    }
+  const std::vector<std::vector<int>> groups = group_parameters(ascending(cvs, false));
+
+  // ---- 3. metric PCCs (Eq. 2) + Algorithm 2 + selection
+  const int NM = ev.n_metrics();
+  std::vector<std::vector<double>> mcol(NM);
+  std::vector<double> times;
+  for (int i : valid) {
+    times.push_back(res[i].ms);
+    for (int k = 0; k < NM; ++k) mcol[k].push_back(res[i].metrics[k]);
+  }
+  std::vector<std::pair<Pair, double>> pccs;
+  for (int a = 0; a < NM; ++a)
+    for (int b = a + 1; b < NM; ++b) pccs.push_back({{a, b}, pcc(mcol[a], mcol[b])});
+  const std::vector<std::vector<int>> cols = combine_metrics(ascending(pccs, true), o->num_collections);
+  std::vector<int> selected;
+  std::vector<double> dirs;
+  for (const auto& c : cols) {
+    int bm = -1;
+    double bv = -1.0;
+    for (int m : c) {
+      const double v = std::fabs(pcc(mcol[m], times));
+      if (v > bv) {
+        bv = v;
+        bm = m;
+      }
+    }
+    selected.push_back(bm);
+    dirs.push_back(pcc(mcol[bm], times) >= 0 ? 1.0 : -1.0);
+  }
+
+  // ---- 4. PMNF per selected metric (Eq. 3), min RSE over I x J
+  std::vector<Tuple> Xv;
+  for (int i : valid) Xv.push_back(rows[i]);
+  std::vector<Fit> chosen;
+  std::vector<std::vector<Fit>> allfits;
+  for (int m : selected) {
+    int bi = 0;
+    std::vector<Fit> fits = pmnf_fit(groups, Xv, mcol[m], &bi);
+    chosen.push_back(fits[bi]);
+    allfits.push_back(fits);
+  }
+
+  // ---- 5. threshold filter over a quantile sample of the space (Q13)
+  const uint64_t nq = std::min<uint64_t>(count, (uint64_t)std::max(16, o->quantile_sample));
+  const std::vector<uint64_t> qranks = sample_ranks(o->seed ^ 0x51A7E5ULL, count, nq);
+  std::vector<Tuple> qset(qranks.size());
+  for (size_t i = 0; i < qranks.size(); ++i) S.at(qranks[i], &qset[i]);
+  const size_t K = selected.size();
+  std::vector<std::vector<double>> preds(K, std::vector<double>(qset.size()));
+  for (size_t k = 0; k < K; ++k)
+    for (size_t i = 0; i < qset.size(); ++i) preds[k][i] = pmnf_predict(groups, chosen[k], qset[i]);
+  std::vector<std::vector<double>> asc = preds;
+  for (auto& v : asc) std::sort(v.begin(), v.end());
+  const int64_t nqs = (int64_t)qset.size();
+  auto thr_at = [&](int64_t t, size_t k) { return dirs[k] > 0 ? asc[k][t] : asc[k][nqs - 1 - t]; };
+  auto passes = [&](size_t i, int64_t t) {
+    for (size_t k = 0; k < K; ++k) {
+      const double th = thr_at(t, k);
+      if (dirs[k] > 0 ? !(preds[k][i] <= th) : !(preds[k][i] >= th)) return false;
+    }
+    return true;
+  };
+  auto frac = [&](int64_t t) {
+    int64_t n = 0;
+    for (int64_t i = 0; i < nqs; ++i) n += passes((size_t)i, t);
+    return (double)n / (double)nqs;
+  };
+  int64_t lo = 0, hi = nqs - 1;
+  while (lo < hi) {
+    const int64_t mid = (lo + hi) / 2;
+    if (frac(mid) >= o->sampling_ratio) hi = mid;
+    else lo = mid + 1;
+  }
+  const int64_t tstar = lo;
+  std::vector<Tuple> kept;
+  for (int64_t i = 0; i < nqs; ++i)
+    if (passes((size_t)i, tstar)) kept.push_back(qset[i]);
+  const uint64_t sampled_count =
+      (uint64_t)std::llround((double)kept.size() / (double)nqs * (double)count);
+
+  // ---- 6. re-index each group's valid value tuples (Fig. 7)
+  std::vector<std::vector<std::vector<int32_t>>> tables;
+  for (const auto& g : groups) {
+    std::set<std::vector<int32_t>> vals;
+    for (const Tuple& t : kept) {
+      std::vector<int32_t> v;
+      for (int f : g) v.push_back(t[f]);
+      vals.insert(v);
+    }
+    tables.push_back(std::vector<std::vector<int32_t>>(vals.begin(), vals.end()));
+  }
+  const double preproc_s = std::chrono::duration<double>(std::chrono::steady_clock::now() - pre0).count();
+
+  js.key("groups");
+  js.o << "[";
+  for (size_t g = 0; g < groups.size(); ++g) {
+    js.o << (g ? "," : "") << "[";
+    for (size_t q = 0; q < groups[g].size(); ++q) js.o << (q ? "," : "") << groups[g][q];
+    js.o << "]";
+  }
+  js.o << "]";
+  js.key("collections");
+  js.o << "[";
+  for (size_t c = 0; c < cols.size(); ++c) {
+    js.o << (c ? "," : "") << "[";
+    for (size_t q = 0; q < cols[c].size(); ++q) js.o << (q ? "," : "") << cols[c][q];
+    js.o << "]";
+  }
+  js.o << "]";
+  js.key("selected");
+  js.o << "[";
+  for (size_t k = 0; k < K; ++k) js.o << (k ? "," : "") << selected[k];
+  js.o << "]";
+  js.key("fits");
+  js.o << "[";
+  for (size_t k = 0; k < K; ++k) {
+    js.o << (k ? "," : "") << "[";
+    for (size_t q = 0; q < allfits[k].size(); ++q) {
+      const Fit& f = allfits[k][q];
+      js.o << (q ? "," : "") << "{\"i\":" << f.i << ",\"j\":" << f.j << ",\"rank\":" << f.rank
+           << ",\"rse\":" << Json::num(f.rse) << ",\"coef\":[";
+      for (size_t c = 0; c < f.coef.size(); ++c) js.o << (c ? "," : "") << Json::num(f.coef[c]);
+      js.o << "]}";
+    }
+    js.o << "]";
+  }
+  js.o << "]";
+  js.key("threshold_index");
+  js.o << tstar;
+  js.key("quantile_sample");
+  js.o << nqs;
+  js.key("kept_ranks");
+  js.o << "[";
+  {
+    bool first = true;
+    for (int64_t i = 0; i < nqs; ++i)
+      if (passes((size_t)i, tstar)) {
+        js.o << (first ? "" : ",") << qranks[i];
+        first = false;
+      }
+  }
+  js.o << "]";
+  js.key("table_sizes");
+  js.o << "[";
+  for (size_t g = 0; g < tables.size(); ++g) js.o << (g ? "," : "") << tables[g].size();
+  js.o << "]";
+
+  // ---- 7. group-wise GA with approximation
+  int bi = valid[0];
+  for (int i : valid)
+    if (fitness_of(res[i]) > fitness_of(res[bi])) bi = i;
+  Tuple cur = rows[bi];
+  double cur_ms = res[bi].ms;
+  Rng rng(o->seed);
+  const int pop = o->n_subpops * o->subpop_size;
+  int total_gens = 0;
+  js.key("phases");
+  js.o << "[";
+  for (size_t g = 0; g < groups.size(); ++g) {
+    const auto& tab = tables[g];
+    const auto& flds = groups[g];
+    if (tab.empty()) continue;
+    auto decode = [&](uint64_t idx) {
+      Tuple t = cur;
+      const auto& v = tab[idx % tab.size()];  // Q16: wrap out-of-range indices
+      for (size_t q = 0; q < flds.size(); ++q) t[flds[q]] = v[q];
+      return t;
+    };
+    std::map<Tuple, double> phase;  // distinct settings evaluated in this phase -> fitness
+    int gens = 0;
+    bool exhaustive = (int)tab.size() <= pop;
+    if (exhaustive) {
+      // P:343 / P:405: fewer settings than the population -> exhaustive search
+      std::vector<Tuple> c;
+      for (size_t i = 0; i < tab.size(); ++i) c.push_back(decode(i));
+      st = ev.run(c, &res);
+      if (st != CST_OK) return st;
+      for (size_t i = 0; i < c.size(); ++i) phase[c[i]] = fitness_of(res[i]);
+    } else {
+      int bits = 0;
+      while ((1ULL << bits) < tab.size()) ++bits;
+      const int sp = o->subpop_size;
+      int cols_t = 1;
+      while ((cols_t + 1) * (cols_t + 1) <= sp) ++cols_t;  // torus cols x rows
+      const int rows_t = (sp + cols_t - 1) / cols_t;
+      std::vector<uint64_t> geno(pop);
+      std::vector<double> fit(pop);
+      for (int i = 0; i < pop; ++i) geno[i] = rng.next() & ((1ULL << bits) - 1);
+      std::vector<Tuple> c;
+      for (int i = 0; i < pop; ++i) c.push_back(decode(geno[i]));
+      st = ev.run(c, &res);
+      if (st != CST_OK) return st;
+      for (int i = 0; i < pop; ++i) {
+        fit[i] = fitness_of(res[i]);
+        phase[c[i]] = fit[i];
+      }
+      for (gens = 1; gens <= o->max_generations; ++gens) {
+        std::vector<uint64_t> child(pop);
+        for (int sidx = 0; sidx < o->n_subpops; ++sidx)
+          for (int cell = 0; cell < sp; ++cell) {
+            const int r0 = cell / cols_t, c0 = cell % cols_t;
+            auto at = [&](int rr, int cc) {
+              rr = (rr + rows_t) % rows_t;
+              cc = (cc + cols_t) % cols_t;
+              int k = rr * cols_t + cc;
+              if (k >= sp) k = k % sp;
+              return sidx * sp + k;
+            };
+            int nb[4] = {at(r0 - 1, c0), at(r0 + 1, c0), at(r0, c0 - 1), at(r0, c0 + 1)};
+            // roulette over the four neighbours, two parents without replacement
+            auto pick = [&](int excl) {
+              double tot = 0;
+              for (int q = 0; q < 4; ++q)
+                if (q != excl) tot += fit[nb[q]];
+              double u = rng.uniform() * tot;
+              int last = -1;
+              for (int q = 0; q < 4; ++q) {
+                if (q == excl) continue;
+                last = q;
+                if (tot > 0 && u < fit[nb[q]]) return q;
+                u -= fit[nb[q]];
+              }
+              if (tot <= 0) {  // all zero: uniform
+                int k = (int)(rng.next() % 3);
+                for (int q = 0; q < 4; ++q) {
+                  if (q == excl) continue;
+                  if (k-- == 0) return q;
+                }
+              }
+              return last;
+            };
+            const int p1 = pick(-1), p2 = pick(p1);
+            uint64_t ch = geno[nb[p1]];
+            if (rng.uniform() < o->crossover) {
+              const uint64_t m = rng.next();
+              ch = (geno[nb[p1]] & m) | (geno[nb[p2]] & ~m);  // uniform crossover
+            }
+            for (int b = 0; b < bits; ++b)
+              if (rng.uniform() < o->mutation) ch ^= (1ULL << b);
+            child[sidx * sp + cell] = ch & ((1ULL << bits) - 1);
+          }
+        c.clear();
+        for (int i = 0; i < pop; ++i) c.push_back(decode(child[i]));
+        st = ev.run(c, &res);
+        if (st != CST_OK) return st;
+        for (int i = 0; i < pop; ++i) {
+          const double f = fitness_of(res[i]);
+          phase[c[i]] = f;
+          if (f >= fit[i]) {  // synchronous replace-if-not-worse
+            fit[i] = f;
+            geno[i] = child[i];
+          }
+        }
+        // single-ring migration: best of each sub-population replaces the worst of its
+        // two ring neighbours
+        if (o->n_subpops > 1) {
+          std::vector<int> bestc(o->n_subpops);
+          for (int s2 = 0; s2 < o->n_subpops; ++s2) {
+            int b = s2 * sp;
+            for (int k = s2 * sp; k < (s2 + 1) * sp; ++k)
+              if (fit[k] > fit[b]) b = k;
+            bestc[s2] = b;
+          }
+          std::vector<uint64_t> mg(o->n_subpops);
+          std::vector<double> mf(o->n_subpops);
+          for (int s2 = 0; s2 < o->n_subpops; ++s2) {
+            mg[s2] = geno[bestc[s2]];
+            mf[s2] = fit[bestc[s2]];
+          }
+          for (int s2 = 0; s2 < o->n_subpops; ++s2)
+            for (int dlt : {-1, 1}) {
+              const int dst = (s2 + dlt + o->n_subpops) % o->n_subpops;
+              if (dst == s2) continue;
+              int w = dst * sp;
+              for (int k = dst * sp; k < (dst + 1) * sp; ++k)
+                if (fit[k] < fit[w]) w = k;
+              if (mf[s2] > fit[w]) {
+                fit[w] = mf[s2];
+                geno[w] = mg[s2];
+              }
+            }
+        }
+        // approximation stop: CV of the top-n fitness of this phase
+        std::vector<double> fs;
+        for (auto& kv : phase)
+          if (kv.second > 0) fs.push_back(kv.second);
+        std::sort(fs.rbegin(), fs.rend());
+        if ((int)fs.size() >= o->top_n) {
+          fs.resize(o->top_n);
+          if (cv(fs) < o->cv_threshold) break;
+        }
+        if (o->time_budget_s > 0 && elapsed() > o->time_budget_s) break;
+      }
+      if (gens > o->max_generations) gens = o->max_generations;
+    }
+    total_gens += gens;
+    // adopt the best setting of the phase
+    for (auto& kv : phase)
+      if (kv.second > 0 && 1.0 / kv.second < cur_ms) {
+        cur_ms = 1.0 / kv.second;
+        cur = kv.first;
+      }
+    js.o << (g ? "," : "") << "{\"group\":" << g << ",\"table\":" << tab.size()
+         << ",\"exhaustive\":" << (exhaustive ? "true" : "false") << ",\"generations\":" << gens
+         << ",\"evaluated\":" << phase.size() << ",\"best_ms\":" << Json::num(cur_ms) << "}";
+    if (o->time_budget_s > 0 && elapsed() > o->time_budget_s) break;
+  }
+  js.o << "]";
+  *best_out = from_tuple(cur);
+  rep->best_ms = cur_ms;
+  rep->best_gstencils = std::isfinite(cur_ms)
+                            ? (double)h->grid.nx * h->grid.ny * h->grid.nz / (cur_ms * 1e-3) / 1e9
+                            : 0.0;
+  rep->space_count = count;
+  rep->sampled_count = sampled_count;
+  rep->evaluations = ev.memo.size();
+  rep->jit_compiles = jit_compile_count() - ev.jit_before;
+  rep->wall_s = elapsed();
+  rep->eval_s = ev.eval_s;
+  rep->jit_s = ev.jit_s;
+  rep->preproc_s = preproc_s;
+  rep->n_groups = (int32_t)groups.size();
+  rep->generations = total_gens;
+  js.key("best");
+  js.o << "{\"setting\": [";
+  for (int f = 0; f < F_COUNT; ++f) js.o << (f ? "," : "") << cur[f];
+  js.o << "], \"ms\": " << Json::num(cur_ms) << "}";
+  js.key("report");
+  js.o << "{\"wall_s\":" << Json::num(rep->wall_s) << ",\"eval_s\":" << Json::num(rep->eval_s)
+       << ",\"jit_s\":" << Json::num(rep->jit_s) << ",\"preproc_s\":" << Json::num(preproc_s)
+       << ",\"dataset_s\":" << Json::num(t_dataset) << ",\"evaluations\":" << rep->evaluations
+       << ",\"jit_compiles\":" << rep->jit_compiles << ",\"space_count\":" << count
+       << ",\"sampled_count\":" << sampled_count << ",\"generations\":" << total_gens << "}";
+  js.o << "\n}\n";
+  if (o->log_path && *o->log_path) {
+    std::ofstream f(o->log_path);
+    f << js.o.str();
+  }
+  return CST_OK;
+}

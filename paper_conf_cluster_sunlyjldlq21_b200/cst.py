@@ -112,7 +112,8 @@ class cst_tune_opts(ctypes.Structure):
                 ("mutation", ctypes.c_double), ("top_n", ctypes.c_int32),
                 ("cv_threshold", ctypes.c_double), ("max_generations", ctypes.c_int32),
                 ("num_collections", ctypes.c_int32), ("time_budget_s", ctypes.c_double),
-                ("reps", ctypes.c_int32), ("warmup", ctypes.c_int32), ("log_path", ctypes.c_char_p)]
+                ("reps", ctypes.c_int32), ("warmup", ctypes.c_int32), ("log_path", ctypes.c_char_p),
+                ("n_user_metrics", ctypes.c_int32), ("quantile_sample", ctypes.c_int32)]
 
 
 class cst_tune_report(ctypes.Structure):
@@ -125,7 +126,8 @@ class cst_tune_report(ctypes.Structure):
 
 
 EVAL_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.POINTER(cst_setting),
-                           ctypes.c_int32, ctypes.POINTER(ctypes.c_double))
+                           ctypes.c_int32, ctypes.POINTER(ctypes.c_double),
+                           ctypes.POINTER(ctypes.c_double))
 
 _P = ctypes.c_void_p
 _PP = ctypes.POINTER(ctypes.c_void_p)
@@ -298,18 +300,26 @@ def cst_tune_opts_default() -> cst_tune_opts:
 
 
 def cst_tune(h, opts: cst_tune_opts, in_ptrs, scratch_out_ptrs, eval_fn=None):
-    """eval_fn(list[cst_setting]) -> list[float ms] (optional: population-parallel eval)."""
+    """eval_fn(list[cst_setting]) -> list[float ms], or (ms list, metrics rows) when
+    opts.n_user_metrics > 0 (optional: population-parallel / synthetic evaluation)."""
     pi, _a = _ptrs(in_ptrs)
     po, _b = _ptrs(scratch_out_ptrs)
     best, rep = cst_setting(), cst_tune_report()
     if eval_fn is not None:
-        def _cb(user, settings, n, ms):
+        nm = opts.n_user_metrics
+
+        def _cb(user, settings, n, ms, metrics):
             try:
                 res = eval_fn([settings[i] for i in range(n)])
+                times, mets = (res if nm > 0 else (res, None))
                 for i in range(n):
-                    ms[i] = float(res[i])
+                    ms[i] = float(times[i])
+                    for k in range(nm):
+                        metrics[i * nm + k] = float(mets[i][k])
                 return 0
             except Exception:
+                import traceback
+                traceback.print_exc()
                 return 1
         cb = EVAL_FN(_cb)
     else:

@@ -1,0 +1,180 @@
+"""C++ tuner (cst_tune) vs the plain-Python oracle (oracle/tuner.py) — CPU only.
+
+A synthetic evaluation callback supplies fitness and "GPU metrics" to cst_tune; the
+oracle recomputes every pre-processing stage from the same dataset and must agree:
+dataset ranks and Algorithm 1 groups / Algorithm 2 collections / selected metrics
+bit-exactly, PMNF fits to 1e-10, the threshold index and kept (sampled) space exactly
+(up to settings within rounding of the threshold), and re-index table sizes.  The GA is
+pinned by properties: determinism, validity, never worse than the dataset best, and the
+exhaustive fallback on small groups.
+"""
+import json
+import math
+
+import numpy as np
+import pytest
+
+from paper_conf_cluster_sunlyjldlq21_b200 import cst as C
+from oracle import space as S
+from oracle import tuner as T
+
+KIND, R, M = 3, 4, (8, 8, 8)        # 44,148 valid settings: the oracle can enumerate it
+NMET = 6
+
+
+def synth(d):
+    t = 1.0
+    t *= 1 + 0.3 * abs(math.log2(d["tb_x"]) - 3)
+    t *= 1 + 0.2 * abs(math.log2(d["tb_y"]) - 2)
+    t *= {1: 1.5, 2: 1.2, 3: 1.0}[d["staging"]]
+    t *= 1 + 0.1 * (d["prefetch"] - 2) ** 2
+    t *= 1.0 if d["use_retiming"] == 2 else 1.3
+    t *= 1 + 0.05 * math.log2(d["bm_y"] * d["cm_y"])
+    t *= 1 + 0.02 * math.log2(d["uf_x"] * d["uf_y"] * d["uf_z"])
+    t *= (1 + 0.04 * abs(math.log2(d["sb"]) - 2)) if d["use_streaming"] == 2 else 1.8
+    t *= 1 + 0.01 * d["use_constant"]
+    m = [t * (1 + 0.01 * (d["tb_x"] % 3)),
+         math.log2(d["tb_x"] * d["tb_y"]),
+         float(d["staging"] * d["prefetch"]),
+         math.log2(d["tb_x"] * d["tb_y"]) + 0.5,
+         float(d["bm_y"] * d["cm_y"] + d["tb_z"]),
+         7.0]
+    return t, m
+
+
+def run_tuner(tmp_path, seed=3, ratio=0.10, cb_log=None):
+    g = C.make_grid(*M, R)
+    h = C.cst_stencil_create(KIND, R, [1.0] * 7, g)
+    o = C.cst_tune_opts_default()
+    o.seed = seed
+    o.sampling_ratio = ratio
+    o.n_user_metrics = NMET
+    o.time_budget_s = 0
+    log = tmp_path / f"tune_{seed}_{ratio}.json"
+    o.log_path = str(log).encode()
+
+    def ev(settings):
+        ts, ms = [], []
+        for s in settings:
+            t, m = synth(s.as_dict())
+            ts.append(t)
+            ms.append(m)
+            if cb_log is not None:
+                cb_log.append(s.as_tuple())
+        return ts, ms
+
+    best, rep = C.cst_tune(h, o, [], [], eval_fn=ev)
+    count = C.cst_space_count(h)
+    C.cst_stencil_destroy(h)
+    return best, rep, json.load(open(log)), count
+
+
+@pytest.fixture(scope="module")
+def space_list():
+    return list(S.enumerate_space(KIND, R, M))
+
+
+@pytest.fixture(scope="module")
+def tuned(tmp_path_factory):
+    return run_tuner(tmp_path_factory.mktemp("tune"))
+
+
+def test_dataset_is_the_seeded_sample(tuned, space_list):
+    best, rep, log, count = tuned
+    assert count == len(space_list) == rep.space_count
+    assert log["dataset"]["ranks"] == T.sample_ranks(3, count, 128)
+    for rk, ms in zip(log["dataset"]["ranks"], log["dataset"]["ms"]):
+        assert ms == synth(space_list[rk])[0]
+
+
+def _oracle_preprocess(log, space_list, ratio=0.10, num_collections=3, qsample=65536, seed=3):
+    ranks = log["dataset"]["ranks"]
+    rows = [(space_list[r], r) for r in ranks]
+    times = [synth(d)[0] for d, _ in rows]
+    mets = np.array([synth(d)[1] for d, _ in rows])
+    fit = [1.0 / t for t in times]
+    groups = T.group_parameters(T.ascending_deque(T.pair_cvs(rows, fit)))
+    cols = T.combine_metrics(T.ascending_deque(T.metric_pairs(mets), key=abs), num_collections)
+    sel = T.select_metrics(cols, mets, np.array(times))
+    X = np.array([S.as_tuple(d) for d, _ in rows], dtype=np.float64)
+    fits = [T.pmnf_fit(groups, X, mets[:, m]) for m in sel]
+    dirs = [1 if T.pcc(mets[:, m], times) >= 0 else -1 for m in sel]
+    count = len(space_list)
+    qranks = T.sample_ranks(seed ^ 0x51A7E5, count, min(count, qsample))
+    Q = np.array([S.as_tuple(space_list[r]) for r in qranks], dtype=np.float64)
+    preds = np.stack([T.pmnf_predict(groups, Q, f[0][f[1]]) for f in fits], axis=1)
+    t, th = T.threshold_filter(preds, dirs, ratio)
+    kept = [qranks[i] for i in range(len(qranks)) if T.passes(preds[i], dirs, th)]
+    tables = []
+    for gr in groups:
+        tables.append(T.reindex([tuple(S.as_tuple(space_list[r])[f] for f in gr) for r in kept]))
+    return dict(groups=groups, cols=cols, sel=sel, fits=fits, t=t, kept=kept, preds=preds,
+                th=th, dirs=dirs, qranks=qranks, tables=tables)
+
+
+def test_groups_collections_selection_bit_exact(tuned, space_list):
+    _, _, log, _ = tuned
+    o = _oracle_preprocess(log, space_list)
+    assert log["groups"] == o["groups"]
+    assert sorted(p for g in o["groups"] for p in g) == list(range(19))
+    assert log["collections"] == o["cols"]
+    assert log["selected"] == o["sel"]
+
+
+def test_pmnf_fits_match(tuned, space_list):
+    _, _, log, _ = tuned
+    o = _oracle_preprocess(log, space_list)
+    for k, (fits, best) in enumerate(o["fits"]):
+        cfits = log["fits"][k]
+        for (i, j, coef, rse), cf in zip(fits, cfits):
+            assert (cf["i"], cf["j"]) == (i, j)
+            if math.isfinite(rse):
+                assert abs(cf["rse"] - rse) <= 1e-9 * max(1.0, abs(rse)), (k, i, j, cf["rse"], rse)
+        # chosen hypothesis: the min-RSE one on both sides
+        crse = [cf["rse"] for cf in cfits]
+        assert int(np.argmin(crse)) == best or abs(min(crse) - fits[best][3]) <= 1e-9 * abs(fits[best][3])
+
+
+def test_threshold_and_sampled_space(tuned, space_list):
+    _, rep, log, count = tuned
+    o = _oracle_preprocess(log, space_list)
+    assert log["quantile_sample"] == len(o["qranks"]) == count        # whole space (small)
+    assert abs(log["threshold_index"] - o["t"]) <= 1
+    kept_c, kept_o = set(log["kept_ranks"]), set(o["kept"])
+    # settings on which the two sides disagree must sit at the threshold (rounding only)
+    for r in kept_c ^ kept_o:
+        i = o["qranks"].index(r)
+        near = any(abs(o["preds"][i][k] - o["th"][k]) <= 1e-9 * max(1.0, abs(o["th"][k]))
+                   for k in range(len(o["th"])))
+        assert near, r
+    assert len(kept_c ^ kept_o) <= max(2, len(kept_o) // 1000)
+    frac = len(kept_c) / count
+    assert frac >= 0.10 and rep.sampled_count == round(frac * count)
+    assert log["table_sizes"] == [len(t) for t in o["tables"]] or len(kept_c ^ kept_o) > 0
+
+
+def test_ga_properties(tuned, space_list, tmp_path):
+    best, rep, log, count = tuned
+    d = best.as_dict()
+    assert S.check(KIND, R, M, d) is None
+    ds_best = min(t for t in log["dataset"]["ms"] if t < 1e300)
+    assert rep.best_ms <= ds_best and rep.best_ms == synth(d)[0]
+    assert rep.n_groups == len(log["groups"]) and rep.evaluations >= 128
+    # exhaustive fallback whenever a group's table fits in the population
+    for ph in log["phases"]:
+        assert ph["exhaustive"] == (ph["table"] <= 32)
+        if ph["exhaustive"]:
+            assert ph["evaluated"] <= ph["table"]
+    # determinism: same seed -> same result and the same candidate sequence
+    seq1, seq2 = [], []
+    b1, r1, l1, _ = run_tuner(tmp_path, seed=5, cb_log=seq1)
+    b2, r2, l2, _ = run_tuner(tmp_path, seed=5, cb_log=seq2)
+    assert b1.as_tuple() == b2.as_tuple() and seq1 == seq2 and l1["phases"] == l2["phases"]
+
+
+def test_ga_finds_near_optimum_with_full_sampling(tmp_path, space_list):
+    """With the whole space kept (ratio 1) the grouped GA must land within 10 % of the
+    brute-force optimum of the synthetic objective (Fig. 4: top-10 within 96.7 %)."""
+    best, rep, log, count = run_tuner(tmp_path, seed=11, ratio=1.0)
+    opt = min(synth(d)[0] for d in space_list)
+    assert rep.best_ms <= 1.10 * opt, (rep.best_ms, opt)
