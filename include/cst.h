@@ -225,6 +225,20 @@ cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const double* const*
  * slabs all owned by this process on one device, a loopback transport (cudaMemcpyAsync)
  * used to test the decomposition on one GPU. */
 typedef struct cst_dist cst_dist;
+
+/* Halo-exchange plan of rank `rank` in a z-slab decomposition over `nranks` ranks, each
+ * owning `nz` local planes, stencil radius `r`: up to 4 transfers of r contiguous planes
+ * (send local planes [0, r) to rank-1 / [nz-r, nz) to rank+1; receive into halo planes
+ * [-r, 0) from rank-1 / [nz, nz+r) from rank+1).  plane_begin is a LOCAL interior z
+ * (negative = halo).  Used by cst_dist_sweep, the loopback transport and the CPU tests. */
+typedef struct {
+  int32_t peer;          /* rank on the other side                         */
+  int32_t is_send;       /* 1 send, 0 receive                               */
+  int64_t plane_begin;   /* first local plane (interior z coordinate)       */
+  int64_t nplanes;       /* = r                                              */
+} cst_halo_xfer;
+cst_status cst_dist_halo_plan(int32_t nranks, int32_t rank, int64_t nz, int32_t r,
+                              cst_halo_xfer* xfers /* [4] */, int32_t* n_xfers);
 cst_status cst_dist_create(cst_stencil* h, int32_t nranks, int32_t rank,
                            const void* nccl_unique_id, cst_dist** out);
 cst_status cst_dist_nccl_unique_id(void* id128);        /* ncclGetUniqueId */

@@ -379,6 +379,21 @@ __device__ __forceinline__ void load_xwin(const LD& ld, int la0, int lb, double*
       w[2 * q] = v.x;
       w[2 * q + 1] = v.y;
     }
+  } else if constexpr (LD::VEC) {
+    // odd run width: load the 16-B aligned superset with double2 (adjacent lanes then
+    // share 16-B chunks -> broadcast) and select the lane's parity
+    constexpr int NV = (WX + 2) / 2;
+    const int odd = (la0 - XR) & 1;
+    const int e0 = la0 - XR - odd;
+    double raw[2 * NV];
+#pragma unroll
+    for (int q = 0; q < NV; ++q) {
+      const double2 v = ld.at2(e0 + 2 * q, lb);
+      raw[2 * q] = v.x;
+      raw[2 * q + 1] = v.y;
+    }
+#pragma unroll
+    for (int q = 0; q < WX; ++q) w[q] = odd ? raw[q + 1] : raw[q];
   } else {
 #pragma unroll
     for (int q = XR - R; q < WX - (XR - R); ++q) w[q] = ld.at(la0 - XR + q, lb);
@@ -468,6 +483,76 @@ __device__ __forceinline__ void load_centres(const LD& ld, const int* la, const 
         cen[ib][ia] = ld.at(la[ia], lb[ib]);
       }
     }
+}
+
+
+// Retimed star plane update, fully in scatter form: every value loaded from plane p
+// is added straight into the rotating accumulators — s-neighbours (2R per point), x-terms
+// of its row and y-terms of the rows within R — so no per-point temporaries stay live.
+// Logical accumulator m of a point = output plane p - R + m (phys (m + U) % W); the
+// in-plane part belongs to m = R.
+template <int U, class LD>
+__device__ __forceinline__ void star_retimed_plane(const Ctx& C, const LD& ld, const int* la,
+                                                   const int* lb,
+                                                   double (&acc)[NCB][NCA][W]) {
+  constexpr int MR = (R + U) % W;
+#pragma unroll
+  for (int cb = 0; cb < CMB; ++cb) {
+    const int lb0 = lb[cb * BMB];
+#pragma unroll
+    for (int ca = 0; ca < CMA; ++ca) {
+      const int la0 = la[ca * BMA];
+#pragma unroll
+      for (int wr = -R; wr < BMB + R; ++wr) {
+        if (wr >= 0 && wr < BMB) {
+          double w[BMA + 2 * XR];
+          load_xwin(ld, la0, lb0 + wr, w);
+#pragma unroll
+          for (int b = 0; b < BMA; ++b) {
+            double(&A)[W] = acc[cb * BMB + wr][ca * BMA + b];
+            const double c = w[XR + b];
+#pragma unroll
+            for (int m = 0; m < W; ++m)  // s-direction scatter: plane p -> output p-R+m
+              if (m != R) A[(m + U) % W] = fma(C.coef(star_ci(AX_S, R - m)), c, A[(m + U) % W]);
+            double ip = C.coef(0) * c;
+#pragma unroll
+            for (int k = -R; k <= R; ++k)
+              if (k != 0) ip = fma(C.coef(star_ci(AX_A, k)), w[XR + b + k], ip);
+            A[MR] += ip;
+#pragma unroll
+            for (int rb = 0; rb < BMB; ++rb) {  // y-terms of the block rows
+              const int k = wr - rb;
+              if (k == 0 || k < -R || k > R) continue;
+              double& B = acc[cb * BMB + rb][ca * BMA + b][MR];
+              B = fma(C.coef(star_ci(AX_B, k)), c, B);
+            }
+          }
+        } else {
+          double v[BMA];
+          if constexpr (LD::VEC && (BMA % 2 == 0)) {
+#pragma unroll
+            for (int b = 0; b < BMA; b += 2) {
+              const double2 t = ld.at2(la0 + b, lb0 + wr);
+              v[b] = t.x;
+              v[b + 1] = t.y;
+            }
+          } else {
+#pragma unroll
+            for (int b = 0; b < BMA; ++b) v[b] = ld.at(la0 + b, lb0 + wr);
+          }
+#pragma unroll
+          for (int b = 0; b < BMA; ++b)
+#pragma unroll
+            for (int rb = 0; rb < BMB; ++rb) {
+              const int k = wr - rb;
+              if (k < -R || k > R) continue;
+              double& B = acc[cb * BMB + rb][ca * BMA + b][MR];
+              B = fma(C.coef(star_ci(AX_B, k)), v[b], B);
+            }
+        }
+      }
+    }
+  }
 }
 
 // =============================================================================
@@ -602,20 +687,7 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
       if constexpr (KIND == 1 && RETIME) {
         // retiming: plane p adds ws[p-o]*u to outputs o = p-R..p+R, its in-plane
         // part to output p; output p-R is then complete.   logical m -> phys (m+u)%W
-        double ip[NCB][NCA], cen[NCB][NCA];
-        star_inplane(C, plane_ld(slot, p), la, lb, ip, cen);
-#pragma unroll
-        for (int ib = 0; ib < NCB; ++ib)
-#pragma unroll
-          for (int ia = 0; ia < NCA; ++ia) {
-#pragma unroll
-            for (int m = 0; m < W; ++m) {
-              if (m == R) continue;
-              double& a = acc[ib][ia][(m + u) % W];
-              a = fma(C.coef(star_ci(AX_S, R - m)), cen[ib][ia], a);
-            }
-            acc[ib][ia][(R + u) % W] += ip[ib][ia];
-          }
+        star_retimed_plane<u>(C, plane_ld(slot, p), la, lb, acc);
         if (j >= 2 * R) {
 #pragma unroll
           for (int ib = 0; ib < NCB; ++ib)

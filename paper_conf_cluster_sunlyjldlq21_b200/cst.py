@@ -125,6 +125,11 @@ class cst_tune_report(ctypes.Structure):
                 ("generations", ctypes.c_int32)]
 
 
+class cst_halo_xfer(ctypes.Structure):
+    _fields_ = [("peer", ctypes.c_int32), ("is_send", ctypes.c_int32),
+                ("plane_begin", ctypes.c_int64), ("nplanes", ctypes.c_int64)]
+
+
 EVAL_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.POINTER(cst_setting),
                            ctypes.c_int32, ctypes.POINTER(ctypes.c_double),
                            ctypes.POINTER(ctypes.c_double))
@@ -165,6 +170,8 @@ _decl("cst_time_setting", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP, ctypes.
 _decl("cst_tune_opts_default", None, ctypes.POINTER(cst_tune_opts))
 _decl("cst_tune", _S, _P, ctypes.POINTER(cst_tune_opts), _PP, _PP, EVAL_FN, _P,
       ctypes.POINTER(cst_setting), ctypes.POINTER(cst_tune_report))
+_decl("cst_dist_halo_plan", _S, ctypes.c_int32, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32,
+      ctypes.POINTER(cst_halo_xfer), ctypes.POINTER(ctypes.c_int32))
 _decl("cst_dist_create", _S, _P, ctypes.c_int32, ctypes.c_int32, _P, ctypes.POINTER(_P))
 _decl("cst_dist_nccl_unique_id", _S, _P)
 _decl("cst_dist_sweep", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP, ctypes.c_int32, _P)
@@ -327,6 +334,14 @@ def cst_tune(h, opts: cst_tune_opts, in_ptrs, scratch_out_ptrs, eval_fn=None):
     check(_lib.cst_tune(h, ctypes.byref(opts), pi, po, cb, None, ctypes.byref(best),
                         ctypes.byref(rep)))
     return best, rep
+
+
+def cst_dist_halo_plan(nranks: int, rank: int, nz: int, r: int):
+    """[(peer, is_send, plane_begin, nplanes), ...] of this rank's halo exchange."""
+    xs = (cst_halo_xfer * 4)()
+    n = ctypes.c_int32()
+    check(_lib.cst_dist_halo_plan(nranks, rank, nz, r, xs, ctypes.byref(n)))
+    return [(x.peer, x.is_send, x.plane_begin, x.nplanes) for x in xs[:n.value]]
 
 
 def cst_dist_nccl_unique_id() -> bytes:
