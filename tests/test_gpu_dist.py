@@ -32,7 +32,7 @@ SETTINGS = [("tma-retimed", S()), ("tma-gather", S(use_retiming=1, bm_x=1, bm_y=
 @pytest.mark.parametrize("nsteps", [1, 2])
 @pytest.mark.parametrize("name,s", SETTINGS, ids=[x[0] for x in SETTINGS])
 def test_loopback_bit_identical_to_single_grid(nslabs, nsteps, name, s):
-    r, nx, ny, nzl, seed = 4, 48, 40, 8, 23
+    r, nx, ny, nzl, seed = 4, 64, 40, 16, 23
     c = list(H.coeffs(1, r, "random", seed=3))
     gl = C.make_grid(nx, ny, nzl * nslabs, r)
     hg = C.cst_stencil_create(1, r, c, gl)
@@ -67,7 +67,7 @@ def test_loopback_bit_identical_to_single_grid(nslabs, nsteps, name, s):
 
 
 def test_loopback_matches_oracle():
-    r, n, nslabs = 4, (40, 32, 8), 3
+    r, n, nslabs = 4, (40, 32, 12), 3
     c = H.coeffs(1, r)
     G = H.layout((n[0], n[1], n[2] * nslabs), r)
     import cstgen
@@ -81,7 +81,8 @@ def test_loopback_matches_oracle():
           for _ in range(nslabs)]
     for k in range(nslabs):
         C.cst_fill_uniform(ls, us[k].data_ptr(), 5, 0, n[0], n[1], k * n[2])
-    C.cst_dist_sweep_loopback(hl, nslabs, S(), [t.data_ptr() for t in us], [t.data_ptr() for t in vs], 1)
+    C.cst_dist_sweep_loopback(hl, nslabs, S(bm_x=1), [t.data_ptr() for t in us],
+                              [t.data_ptr() for t in vs], 1)
     C.cst_sync(hl)
     wi = H.interior(G, want)
     scale = np.max(np.abs(wi))

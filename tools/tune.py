@@ -1,0 +1,84 @@
+"""Run cst_tune (the csTuner pipeline in libcst) on one GPU for a config and record the
+tuned setting (used by bench.py) plus the tuner's stage-by-stage JSON report.
+
+    python tools/tune.py --config star25      # BASELINE configs[1]: order-4 star, 512^3
+    python tools/tune.py --config box27       # configs[2]
+    python tools/tune.py --config hypterm     # configs[3]
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+from paper_conf_cluster_sunlyjldlq21_b200 import cst as C  # noqa: E402
+
+D2_R4 = [-9, 128, -1008, 8064, -14350, 8064, -1008, 128, -9]
+
+
+def config(name):
+    if name == "star25":
+        w = [v / 5040.0 for v in D2_R4]
+        side = w[:4] + w[5:]
+        return C.CST_STAR, 4, [3 * w[4]] + side * 3, (512, 512, 512), 2
+    if name == "box27":
+        b = [0.25, 0.5, 0.25]
+        return C.CST_BOX, 1, [x * y * z for x in b for y in b for z in b], (512, 512, 512), 3
+    if name == "hypterm":
+        return C.CST_HYPTERM, 4, [4 / 5, -1 / 5, 4 / 105, -1 / 280, 1.0, 1.0, 1.0], (512, 512, 512), 4
+    raise ValueError(name)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="star25")
+    ap.add_argument("--budget", type=float, default=300.0)
+    ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--out", default=None)
+    args = ap.parse_args()
+    kind, r, coeffs, n, seed = config(args.config)
+    g = C.make_grid(*n, r)
+    h = C.cst_stencil_create(kind, r, coeffs, g)
+    ins = [torch.empty(g.numel, dtype=torch.float64, device="cuda") for _ in range(C.N_IN[kind])]
+    outs = [torch.empty(g.numel, dtype=torch.float64, device="cuda") for _ in range(C.N_OUT[kind])]
+    for a, t in enumerate(ins):
+        C.cst_fill_uniform(g, t.data_ptr(), seed, a)
+    torch.cuda.synchronize()
+    o = C.cst_tune_opts_default()
+    o.seed = args.seed
+    o.time_budget_s = args.budget
+    o.reps = args.reps
+    os.makedirs(os.path.join(ROOT, "tuned", "logs"), exist_ok=True)
+    log = os.path.join(ROOT, "tuned", "logs", f"{args.config}_seed{args.seed}.json")
+    o.log_path = log.encode()
+    t0 = time.time()
+    best, rep = C.cst_tune(h, o, [t.data_ptr() for t in ins], [t.data_ptr() for t in outs])
+    wall = time.time() - t0
+    # re-time the winner and the default setting on the same buffers
+    stream = torch.cuda.current_stream().cuda_stream
+    ms_best = C.cst_time_setting(h, best, [t.data_ptr() for t in ins], [t.data_ptr() for t in outs],
+                                 3, 20, stream)
+    dflt = C.cst_setting_default(h)
+    ms_def = C.cst_time_setting(h, dflt, [t.data_ptr() for t in ins], [t.data_ptr() for t in outs],
+                                3, 20, stream)
+    pts = n[0] * n[1] * n[2]
+    res = {"config": args.config, "grid": list(n), "setting": best.as_dict(),
+           "tuned_ms": rep.best_ms, "retimed_ms": ms_best, "gstencils": pts / (ms_best * 1e-3) / 1e9,
+           "default_setting": dflt.as_dict(), "default_ms": ms_def,
+           "report": {f: getattr(rep, f) for f, _ in rep._fields_}, "wall_s": wall,
+           "log": os.path.relpath(log, ROOT), "seed": args.seed, "budget_s": args.budget}
+    out = args.out or os.path.join(ROOT, "tuned", f"{args.config}_512.json")
+    with open(out, "w") as f:
+        json.dump(res, f, indent=1)
+    print(json.dumps(res))
+    C.cst_stencil_destroy(h)
+
+
+if __name__ == "__main__":
+    main()
