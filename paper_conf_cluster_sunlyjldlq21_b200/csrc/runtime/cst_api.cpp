@@ -134,7 +134,10 @@ extern "C" const char* cst_status_str(cst_status s) {
 }
 
 extern "C" const char* cst_last_error(void) { return t_err.c_str(); }
-extern "C" const char* cst_version(void) { return "cst 0.1 (sm_100a)"; }
+extern "C" const char* cst_version(void) {
+  static std::string v = "cst 0.1 (sm_100a; " + nvrtc_description() + ")";
+  return v.c_str();
+}
 
 // ====================================================================== handles
 static int expected_coeffs(int kind, int r) {
@@ -211,26 +214,32 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
     return (int32_t)x;
   };
   const int64_t* M = h->info.M;
+  // measured-good starting points on B200, shrunk to fit small grids:
+  // streaming along z, TMA staging, retimed accumulators; star/box 64x8 tiles of 2x2
+  // register blocks; hypterm 16x8 tiles, one point per thread.
+  const bool hyp = h->info.kind == CST_HYPTERM;
   cst_setting c{};
-  // streaming along z, TMA staging, retimed accumulators, 3-stage pipeline
-  c.tb[0] = p2floor(M[0], 64);
-  c.tb[1] = p2floor(M[1], h->info.kind == CST_HYPTERM ? 4 : 4);
+  c.tb[0] = hyp ? 16 : 32;
+  c.tb[1] = hyp ? 8 : 4;
   c.tb[2] = 1;
   c.staging = 3;
   c.use_constant = 1;
   c.use_streaming = 2;
   c.sd = 3;
-  c.sb = p2floor(M[2], 128);
+  c.sb = p2floor(M[2], hyp ? 256 : 128);
   for (int d = 0; d < 3; ++d) c.uf[d] = c.cm[d] = c.bm[d] = 1;
-  c.bm[1] = p2floor(M[1] / c.tb[1] > 0 ? M[1] / c.tb[1] : 1, 2);
+  c.bm[0] = hyp ? 1 : 2;
+  c.bm[1] = hyp ? 1 : 2;
   c.use_retiming = 2;
-  c.prefetch = 3;
-  if (h->info.kind == CST_HYPTERM) {
-    c.tb[0] = p2floor(M[0], 32);
-    c.tb[1] = p2floor(M[1], 4);
-    c.bm[1] = 1;
-    c.staging = 1;
-    c.prefetch = 1;
+  c.prefetch = h->info.kind == CST_BOX ? 2 : 3;
+  for (int tries = 0; tries < 12 && check_rules(h->info, to_tuple(c)); ++tries) {
+    // shrink the tile until it fits the grid (coverage) and the thread floor
+    if (c.bm[0] > 1 && (int64_t)c.tb[0] * c.bm[0] > M[0]) c.bm[0] /= 2;
+    else if (c.bm[1] > 1 && (int64_t)c.tb[1] * c.bm[1] > M[1]) c.bm[1] /= 2;
+    else if (c.tb[0] > 1 && c.tb[0] > M[0]) { c.tb[0] /= 2; c.tb[1] *= 2; }
+    else if (c.tb[1] > 1 && c.tb[1] > M[1]) { c.tb[1] /= 2; }
+    else if (c.tb[0] * c.bm[0] % 2) { c.staging = 2; }
+    else break;
   }
   if (!check_rules(h->info, to_tuple(c))) {
     *s = c;

@@ -109,6 +109,7 @@ struct Variant {
 cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
                      double* compile_s);
 uint64_t jit_compile_count();
+std::string nvrtc_description();
 
 }  // namespace cst
 

@@ -3,6 +3,7 @@
 // only valid settings are compiled).  NVRTC compiles
 // csrc/kernels/cst_kernels.cuh for sm_100a with the setting as compile-time constants;
 // cubins are cached in memory and on disk ($CST_CACHE_DIR, default ~/.cache/cst).
+#include <dlfcn.h>
 #include <nvrtc.h>
 #include <sys/stat.h>
 #include <unistd.h>
@@ -19,6 +20,57 @@
 
 namespace {
 #include "kernels_src.inc"  // kSrcParams, kSrcPtx, kSrcKernels (generated at build time)
+
+// NVRTC is loaded at run time by absolute path: torch may already have mapped its own
+// (older) libnvrtc.so.12, and binding to that copy through the shared soname silently
+// changes the generated code.  Order: $CST_NVRTC_PATH, $CUDA_HOME/lib64, /usr/local/cuda.
+struct Nvrtc {
+  decltype(&nvrtcCreateProgram) create = nullptr;
+  decltype(&nvrtcCompileProgram) compile = nullptr;
+  decltype(&nvrtcGetProgramLogSize) log_size = nullptr;
+  decltype(&nvrtcGetProgramLog) log = nullptr;
+  decltype(&nvrtcGetCUBINSize) cubin_size = nullptr;
+  decltype(&nvrtcGetCUBIN) cubin = nullptr;
+  decltype(&nvrtcDestroyProgram) destroy = nullptr;
+  decltype(&nvrtcGetErrorString) error = nullptr;
+  decltype(&nvrtcVersion) version = nullptr;
+  std::string path;
+  int major = 0, minor = 0;
+};
+
+const Nvrtc* nvrtc_lib() {
+  static Nvrtc n;
+  static bool ok = false;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    std::vector<std::string> cands;
+    if (const char* e = std::getenv("CST_NVRTC_PATH")) cands.push_back(e);
+    if (const char* c = std::getenv("CUDA_HOME")) cands.push_back(std::string(c) + "/lib64/libnvrtc.so.12");
+    cands.push_back("/usr/local/cuda/lib64/libnvrtc.so.12");
+    cands.push_back("libnvrtc.so.12");
+    for (const std::string& p : cands) {
+      void* h = dlopen(p.c_str(), RTLD_NOW | RTLD_LOCAL);
+      if (!h) continue;
+      n.create = (decltype(n.create))dlsym(h, "nvrtcCreateProgram");
+      n.compile = (decltype(n.compile))dlsym(h, "nvrtcCompileProgram");
+      n.log_size = (decltype(n.log_size))dlsym(h, "nvrtcGetProgramLogSize");
+      n.log = (decltype(n.log))dlsym(h, "nvrtcGetProgramLog");
+      n.cubin_size = (decltype(n.cubin_size))dlsym(h, "nvrtcGetCUBINSize");
+      n.cubin = (decltype(n.cubin))dlsym(h, "nvrtcGetCUBIN");
+      n.destroy = (decltype(n.destroy))dlsym(h, "nvrtcDestroyProgram");
+      n.error = (decltype(n.error))dlsym(h, "nvrtcGetErrorString");
+      n.version = (decltype(n.version))dlsym(h, "nvrtcVersion");
+      if (n.create && n.compile && n.log_size && n.log && n.cubin_size && n.cubin &&
+          n.destroy && n.error && n.version) {
+        n.version(&n.major, &n.minor);
+        n.path = p;
+        ok = true;
+        return;
+      }
+    }
+  });
+  return ok ? &n : nullptr;
+}
 
 std::mutex g_mu;
 std::unordered_map<std::string, std::string> g_mem;  // key -> cubin
@@ -59,6 +111,12 @@ namespace cst {
 
 uint64_t jit_compile_count() { return g_compiles.load(); }
 
+std::string nvrtc_description() {
+  const Nvrtc* N = nvrtc_lib();
+  if (!N) return "nvrtc: not found";
+  return "nvrtc " + std::to_string(N->major) + "." + std::to_string(N->minor) + " (" + N->path + ")";
+}
+
 static std::string prefix_for(const StencilInfo& st, const Tuple& t) {
   std::ostringstream o;
   o << "#define CST_KIND " << st.kind << "\n#define CST_R " << st.r << "\n";
@@ -77,9 +135,9 @@ cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
   static const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo",
                                "--fmad=true", "-default-device", "-DCST_NVRTC=1"};
   const int nopts = sizeof(opts) / sizeof(opts[0]);
-  int nv_major = 0, nv_minor = 0;
-  nvrtcVersion(&nv_major, &nv_minor);
-  std::string keysrc = src + "nvrtc" + std::to_string(nv_major) + "." + std::to_string(nv_minor);
+  const Nvrtc* N = nvrtc_lib();
+  if (!N) return fail(CST_E_NVRTC, "libnvrtc.so.12 not found (set CST_NVRTC_PATH)");
+  std::string keysrc = src + "nvrtc" + std::to_string(N->major) + "." + std::to_string(N->minor);
   for (int i = 0; i < nopts; ++i) keysrc += opts[i];
   uint64_t h = fnv1a(keysrc);
   h = fnv1a(kSrcParams, h);
@@ -114,24 +172,22 @@ cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
   const char* hdr_src[3] = {kSrcParams, kSrcPtx, kSrcKernels};
   const char* hdr_names[3] = {"cst_params.h", "cst_ptx.cuh", "cst_kernels.cuh"};
   nvrtcProgram prog;
-  if (nvrtcCreateProgram(&prog, src.c_str(), "cst_variant.cu", 3, hdr_src, hdr_names) !=
-      NVRTC_SUCCESS)
+  if (N->create(&prog, src.c_str(), "cst_variant.cu", 3, hdr_src, hdr_names) != NVRTC_SUCCESS)
     return fail(CST_E_NVRTC, "nvrtcCreateProgram failed");
-  const nvrtcResult rc = nvrtcCompileProgram(prog, nopts, opts);
+  const nvrtcResult rc = N->compile(prog, nopts, opts);
   if (rc != NVRTC_SUCCESS) {
     size_t n = 0;
-    nvrtcGetProgramLogSize(prog, &n);
+    N->log_size(prog, &n);
     std::string log(n, '\0');
-    if (n) nvrtcGetProgramLog(prog, &log[0]);
-    nvrtcDestroyProgram(&prog);
-    return fail(CST_E_NVRTC, std::string("nvrtc: ") + nvrtcGetErrorString(rc) + "\n" +
-                                 log.substr(0, 4000));
+    if (n) N->log(prog, &log[0]);
+    N->destroy(&prog);
+    return fail(CST_E_NVRTC, std::string("nvrtc: ") + N->error(rc) + "\n" + log.substr(0, 4000));
   }
   size_t n = 0;
-  nvrtcGetCUBINSize(prog, &n);
+  N->cubin_size(prog, &n);
   std::string data(n, '\0');
-  nvrtcGetCUBIN(prog, &data[0]);
-  nvrtcDestroyProgram(&prog);
+  N->cubin(prog, &data[0]);
+  N->destroy(&prog);
   ++g_compiles;
   *compile_s =
       std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
