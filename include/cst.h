@@ -186,6 +186,7 @@ typedef struct {
   const char* log_path;      /* JSON report of every stage, or NULL              */
   int32_t n_user_metrics;    /* metrics supplied by the eval callback (0 = model) */
   int32_t quantile_sample;   /* settings sampled to set thresholds / gene tables  */
+  int32_t warm_start;        /* 1: add cst_setting_default() to the dataset (ours) */
 } cst_tune_opts;
 
 typedef struct {

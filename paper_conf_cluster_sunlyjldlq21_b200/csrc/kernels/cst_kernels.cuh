@@ -827,7 +827,13 @@ __device__ __forceinline__ void load_line(const LD& ld, int la, int lb, double* 
     load_xwin(ld, la, lb, w);
   } else {
 #pragma unroll
-    for (int q = 0; q < BMB + 2 * R; ++q) w[q] = ld.at(la, lb - R + q);
+    for (int q = 0; q < BMB + 2 * R; ++q) {
+      if (BMB == 1 && q == R) {  // the point itself: derivative terms never read it
+        w[q] = 0.0;
+        continue;
+      }
+      w[q] = ld.at(la, lb - R + q);
+    }
   }
 }
 

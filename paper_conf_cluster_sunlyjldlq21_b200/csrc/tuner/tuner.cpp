@@ -372,6 +372,7 @@ extern "C" void cst_tune_opts_default(cst_tune_opts* o) {
   o->log_path = nullptr;
   o->n_user_metrics = 0;
   o->quantile_sample = 65536;
+  o->warm_start = 1;
 }
 
 namespace {
@@ -504,7 +505,16 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
   js.o << "{";
 
   // ---- 1. dataset
-  const std::vector<uint64_t> ranks = sample_ranks(o->seed, count, (uint64_t)o->dataset_size);
+  std::vector<uint64_t> ranks = sample_ranks(o->seed, count, (uint64_t)o->dataset_size);
+  if (o->warm_start) {
+    // ours: the library's measured-good default joins the dataset, so the search starts no
+    // worse than it (the paper samples the dataset purely at random)
+    cst_setting d;
+    uint64_t rk;
+    if (cst_setting_default(h, &d) == CST_OK && S.rank(to_tuple(d), &rk) &&
+        std::find(ranks.begin(), ranks.end(), rk) == ranks.end())
+      ranks.push_back(rk);
+  }
   std::vector<Tuple> rows;
   for (uint64_t rk : ranks) {
     Tuple t;

@@ -113,7 +113,8 @@ class cst_tune_opts(ctypes.Structure):
                 ("cv_threshold", ctypes.c_double), ("max_generations", ctypes.c_int32),
                 ("num_collections", ctypes.c_int32), ("time_budget_s", ctypes.c_double),
                 ("reps", ctypes.c_int32), ("warmup", ctypes.c_int32), ("log_path", ctypes.c_char_p),
-                ("n_user_metrics", ctypes.c_int32), ("quantile_sample", ctypes.c_int32)]
+                ("n_user_metrics", ctypes.c_int32), ("quantile_sample", ctypes.c_int32),
+                ("warm_start", ctypes.c_int32)]
 
 
 class cst_tune_report(ctypes.Structure):

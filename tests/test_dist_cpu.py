@@ -112,6 +112,7 @@ def _tune_worker(rank, world, port, outdir):
     o.seed = 9
     o.n_user_metrics = TT.NMET
     o.time_budget_s = 0
+    o.warm_start = 0
     evaluated = []
 
     def ev(d):
@@ -141,6 +142,7 @@ def test_population_parallel_tuning_equals_single_process(tmp_path):
     o.seed = 9
     o.n_user_metrics = TT.NMET
     o.time_budget_s = 0
+    o.warm_start = 0
     best, rep = C.cst_tune(h, o, [], [], eval_fn=lambda ss: (
         [TT.synth(s.as_dict())[0] for s in ss], [TT.synth(s.as_dict())[1] for s in ss]))
     C.cst_stencil_destroy(h)

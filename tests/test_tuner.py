@@ -50,6 +50,7 @@ def run_tuner(tmp_path, seed=3, ratio=0.10, cb_log=None):
     o.sampling_ratio = ratio
     o.n_user_metrics = NMET
     o.time_budget_s = 0
+    o.warm_start = 0
     log = tmp_path / f"tune_{seed}_{ratio}.json"
     o.log_path = str(log).encode()
 
