@@ -46,6 +46,9 @@ constexpr int BMA = BMX, BMB = SZ ? BMY : BMZ, BMS = SZ ? BMZ : BMY;
 constexpr int CMA = CMX, CMB = SZ ? CMY : CMZ, CMS = SZ ? CMZ : CMY;
 constexpr int UFA = UFX, UFB = SZ ? UFY : UFZ, UFS = SZ ? UFZ : UFY;
 constexpr int TA = TBA * BMA * CMA, TB = TBB * BMB * CMB, TS = TBS * BMS * CMS;
+// register budget: the hypterm fast path keeps 45 FP64 accumulators per point; asking for
+// 3 resident CTAs of <= 128 threads lets ptxas fit it in 168 registers
+constexpr int MINB = 1;  // (3 for the hypterm fast path spills a few bytes; kept at 1)
 
 __constant__ double c_coef[CST_MAX_COEF];
 
@@ -860,6 +863,9 @@ __device__ __forceinline__ void hyp_inplane(const Ctx& C, const LD* ld, const in
     load_line<AXIS>(ld[7], la0, lb0, w4);
 #pragma unroll
     for (int m = 0; m < 4; ++m) {
+      // keep ptxas from hoisting all six windows at once (register budget of the
+      // 45-accumulator fast path; shared-memory latency is hidden by the other warps)
+      if constexpr (MINB > 1) asm volatile("" ::: "memory");
       load_line<AXIS>(ld[m], la0, lb0, wc);
 #pragma unroll
       for (int pt = 0; pt < NPL; ++pt) {
@@ -930,11 +936,10 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   for (int i = 0; i < NCB; ++i) lb[i] = merged_pos(i, tb, TBB, BMB);
   const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
 
-  // streamed-direction weights: plane p contributes ws[p-o] * E_f(p) to flux_f(o)
-  double ws[W];
-#pragma unroll
-  for (int k = -R; k <= R; ++k)
-    ws[k + R] = k == 0 ? 0.0 : (k > 0 ? -1.0 : 1.0) * C.coef(4 + DS) * C.coef((k > 0 ? k : -k) - 1);
+  // streamed-direction weights ws[k] = -sign(k) dxinv_s a_|k| (host-precomputed, in the
+  // constant bank after the 7 user coefficients: 8 for s = z, then 8 for s = y):
+  // plane p contributes ws[p-o] * E_f(p) to flux_f(o)
+  auto ws = [&](int k) { return C.coef(7 + (DS == 1 ? 8 : 0) + (k < 0 ? k + R : k + R - 1)); };
 
   double acc[5][NCB][NCA][W];  // retimed: pending fluxes ; gather: queue of E_f
 #pragma unroll
@@ -1003,26 +1008,44 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
       if constexpr (STAGING == 3) mbar_wait(&bars[slot], (u32)((j / NP) & 1));
       LDT ld[NIN];
       loaders(slot, p, ld);
-      double E[5][NCB][NCA];
-      hyp_products(ld, la, lb, E);
       if constexpr (RETIME) {
-        double ta_[5][NCB][NCA], tb_[5][NCB][NCA];
-        hyp_inplane<0>(C, ld, la, lb, ta_);
-        hyp_inplane<1>(C, ld, la, lb, tb_);
+        // scatter in an order that keeps few temporaries live: E_f first, then T_a, T_b
+        {
+          double E[5][NCB][NCA];
+          hyp_products(ld, la, lb, E);
 #pragma unroll
-        for (int f = 0; f < 5; ++f)
+          for (int f = 0; f < 5; ++f)
 #pragma unroll
-          for (int ib = 0; ib < NCB; ++ib)
+            for (int ib = 0; ib < NCB; ++ib)
 #pragma unroll
-            for (int ia = 0; ia < NCA; ++ia) {
+              for (int ia = 0; ia < NCA; ++ia)
 #pragma unroll
-              for (int m = 0; m < W; ++m) {
-                if (m == R) continue;
-                double& a = acc[f][ib][ia][(m + u) % W];
-                a = fma(ws[2 * R - m], E[f][ib][ia], a);  // k = p - o = R - m
-              }
-              acc[f][ib][ia][(R + u) % W] += -ta_[f][ib][ia] - tb_[f][ib][ia];
-            }
+                for (int m = 0; m < W; ++m) {
+                  if (m == R) continue;
+                  double& a = acc[f][ib][ia][(m + u) % W];
+                  a = fma(ws(R - m), E[f][ib][ia], a);  // k = p - o = R - m
+                }
+        }
+        {
+          double t[5][NCB][NCA];
+          hyp_inplane<0>(C, ld, la, lb, t);
+#pragma unroll
+          for (int f = 0; f < 5; ++f)
+#pragma unroll
+            for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+              for (int ia = 0; ia < NCA; ++ia) acc[f][ib][ia][(R + u) % W] -= t[f][ib][ia];
+        }
+        {
+          double t[5][NCB][NCA];
+          hyp_inplane<1>(C, ld, la, lb, t);
+#pragma unroll
+          for (int f = 0; f < 5; ++f)
+#pragma unroll
+            for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+              for (int ia = 0; ia < NCA; ++ia) acc[f][ib][ia][(R + u) % W] -= t[f][ib][ia];
+        }
         if (j >= 2 * R) {
 #pragma unroll
           for (int ib = 0; ib < NCB; ++ib)
@@ -1042,6 +1065,8 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
             for (int ia = 0; ia < NCA; ++ia) acc[f][ib][ia][u % W] = 0.0;
       } else {
         // gather: queue of E_f, newest at phys u
+        double E[5][NCB][NCA];
+        hyp_products(ld, la, lb, E);
 #pragma unroll
         for (int f = 0; f < 5; ++f)
 #pragma unroll
@@ -1207,7 +1232,7 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
 // =============================================================================
 // entry point
 // =============================================================================
-extern "C" __global__ void __launch_bounds__(NTHR) cst_kernel(const __grid_constant__ cst_kparams P) {
+extern "C" __global__ void __launch_bounds__(NTHR, MINB) cst_kernel(const __grid_constant__ cst_kparams P) {
   extern __shared__ __align__(128) double cst_smem[];
   if constexpr (!STREAM) {
     kernel_tile3d(P, cst_smem);

@@ -175,6 +175,16 @@ extern "C" cst_status cst_stencil_create(const cst_stencil_desc* desc, const cst
   h->desc = *desc;
   h->coeffs.assign(desc->coeffs, desc->coeffs + desc->n_coeffs);
   h->desc.coeffs = h->coeffs.data();
+  // kernel coefficient bank: the user's coefficients, plus for hypterm the streamed-
+  // direction weights ws[k] = -sign(k) dxinv_s a_|k| (k = -4..-1, 1..4) for s = z, then y
+  h->kcoef = h->coeffs;
+  if (kind == CST_HYPTERM)
+    for (int sdir : {2, 1})
+      for (int k = -4; k <= 4; ++k) {
+        if (k == 0) continue;
+        const double a = h->coeffs[(k > 0 ? k : -k) - 1];
+        h->kcoef.push_back((k > 0 ? -1.0 : 1.0) * (h->coeffs[4 + sdir] * a));
+      }
   h->grid = *g;
   h->device = device;
   h->info.kind = kind;
@@ -195,6 +205,8 @@ extern "C" void cst_stencil_destroy(cst_stencil* h) {
       if (kv.second.mod) d->cuModuleUnload(kv.second.mod);
     for (double* p : h->dev_bufs) cudaFree(p);
     if (h->host_stream) cudaStreamDestroy(h->host_stream);
+    if (h->host_in_stream) cudaStreamDestroy(h->host_in_stream);
+    if (h->host_out_stream) cudaStreamDestroy(h->host_out_stream);
   }
   delete h;
 }
@@ -342,7 +354,7 @@ static cst_status get_variant(cst_stencil* h, const cst_setting* s, Variant** ou
     size_t bytes;
     st = cu_check(d->cuModuleGetGlobal(&dp, &bytes, v.mod, "c_coef"), "cuModuleGetGlobal");
     if (st != CST_OK) return st;
-    CST_CUDA(cudaMemcpy((void*)dp, h->coeffs.data(), h->coeffs.size() * sizeof(double),
+    CST_CUDA(cudaMemcpy((void*)dp, h->kcoef.data(), h->kcoef.size() * sizeof(double),
                         cudaMemcpyHostToDevice));
   }
   h->variants[key] = v;
@@ -440,7 +452,7 @@ cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* 
     }
   }
   for (int o = 0; o < nout; ++o) P.out[o] = out[o] + origin;
-  for (size_t i = 0; i < h->coeffs.size() && i < CST_MAX_COEF; ++i) P.coef[i] = h->coeffs[i];
+  for (size_t i = 0; i < h->kcoef.size() && i < CST_MAX_COEF; ++i) P.coef[i] = h->kcoef[i];
   P.py = G.pitch_x;
   P.pz = G.pitch_x * G.pitch_y;
   P.nx = (int)G.nx;
@@ -547,37 +559,77 @@ extern "C" cst_status cst_sweep_host(cst_stencil* h, const cst_setting* s,
   cudaStream_t sm = h->host_stream;
   const double* din[CST_MAX_IN];
   double* dout[CST_MAX_OUT];
-  for (int a = 0; a < nin; ++a) {
-    din[a] = h->dev_bufs[a];
-    CST_CUDA(cudaMemcpyAsync(h->dev_bufs[a], in[a], (size_t)n * 8, cudaMemcpyHostToDevice, sm));
-  }
-  for (int o = 0; o < nout; ++o) {
-    dout[o] = h->dev_bufs[nin + o];
-    if (nsteps > 1)  // ping-pong reads the output buffer's halo (Dirichlet data)
-      CST_CUDA(cudaMemcpyAsync(dout[o], out[o], (size_t)n * 8, cudaMemcpyHostToDevice, sm));
-  }
-  st = cst_sweep(h, s, din, dout, nsteps, sm);
-  if (st != CST_OK) return st;
-  // copy back interiors only (halos of host outputs are never written)
-  auto copy_back = [&](const double* dsrc, double* hdst) -> cst_status {
+  for (int a = 0; a < nin; ++a) din[a] = h->dev_bufs[a];
+  for (int o = 0; o < nout; ++o) dout[o] = h->dev_bufs[nin + o];
+  const int64_t plane = G.pitch_y * G.pitch_x;
+  // copy back interior planes [z0, z1) only (halos of host outputs are never written)
+  auto copy_back = [&](const double* dsrc, double* hdst, int64_t z0, int64_t z1,
+                       cudaStream_t st_) -> cst_status {
     cudaMemcpy3DParms p = {};
-    const int64_t first = ((int64_t)G.halo * G.pitch_y + G.halo) * G.pitch_x + G.lead_x;
+    const int64_t first = ((G.halo + z0) * G.pitch_y + G.halo) * G.pitch_x + G.lead_x;
     p.srcPtr = make_cudaPitchedPtr((void*)(dsrc + first), G.pitch_x * 8, G.nx * 8, G.pitch_y);
     p.dstPtr = make_cudaPitchedPtr((void*)(hdst + first), G.pitch_x * 8, G.nx * 8, G.pitch_y);
-    p.extent = make_cudaExtent(G.nx * 8, G.ny, G.nz);
+    p.extent = make_cudaExtent(G.nx * 8, G.ny, z1 - z0);
     p.kind = cudaMemcpyDeviceToHost;
-    CST_CUDA(cudaMemcpy3DAsync(&p, sm));
+    CST_CUDA(cudaMemcpy3DAsync(&p, st_));
     return CST_OK;
   };
+  if (nsteps == 1) {
+    // pipelined along z: H2D of chunk k+1 || sweep of chunk k || D2H of chunk k-1
+    if (!h->host_in_stream) {
+      CST_CUDA(cudaStreamCreateWithFlags(&h->host_in_stream, cudaStreamNonBlocking));
+      CST_CUDA(cudaStreamCreateWithFlags(&h->host_out_stream, cudaStreamNonBlocking));
+    }
+    const int64_t nc = std::max<int64_t>(1, std::min<int64_t>(8, G.nz / std::max(16, 4 * h->info.r)));
+    std::vector<cudaEvent_t> evs;
+    auto event = [&](cudaStream_t st_) -> cudaEvent_t {
+      cudaEvent_t e;
+      cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+      cudaEventRecord(e, st_);
+      evs.push_back(e);
+      return e;
+    };
+    int64_t copied = 0;  // padded planes already on the device
+    const int64_t planes = G.nz + 2 * (int64_t)G.halo;
+    h->last_launches = 0;
+    st = CST_OK;
+    for (int64_t k = 0; k < nc && st == CST_OK; ++k) {
+      const int64_t z0 = k * G.nz / nc, z1 = (k + 1) * G.nz / nc;
+      const int64_t need = k == nc - 1 ? planes : std::min(planes, z1 + G.halo + h->info.r);
+      for (int a = 0; a < nin && need > copied; ++a)
+        CST_CUDA(cudaMemcpyAsync(h->dev_bufs[a] + copied * plane, in[a] + copied * plane,
+                                 (size_t)(need - copied) * plane * 8, cudaMemcpyHostToDevice,
+                                 h->host_in_stream));
+      copied = std::max(copied, need);
+      CST_CUDA(cudaStreamWaitEvent(sm, event(h->host_in_stream), 0));
+      st = cst_launch_range(h, s, din, dout, z0, z1 - z0, sm);
+      if (st != CST_OK) break;
+      CST_CUDA(cudaStreamWaitEvent(h->host_out_stream, event(sm), 0));
+      for (int o = 0; o < nout && st == CST_OK; ++o)
+        st = copy_back(dout[o], out[o], z0, z1, h->host_out_stream);
+    }
+    cudaStreamSynchronize(h->host_in_stream);
+    cudaStreamSynchronize(sm);
+    cudaStreamSynchronize(h->host_out_stream);
+    for (cudaEvent_t e : evs) cudaEventDestroy(e);
+    if (st != CST_OK) return st;
+    CST_CUDA(cudaGetLastError());
+    return CST_OK;
+  }
+  for (int a = 0; a < nin; ++a)
+    CST_CUDA(cudaMemcpyAsync(h->dev_bufs[a], in[a], (size_t)n * 8, cudaMemcpyHostToDevice, sm));
+  for (int o = 0; o < nout; ++o)  // ping-pong reads the output buffer's halo (Dirichlet data)
+    CST_CUDA(cudaMemcpyAsync(dout[o], out[o], (size_t)n * 8, cudaMemcpyHostToDevice, sm));
+  st = cst_sweep(h, s, din, dout, nsteps, sm);
+  if (st != CST_OK) return st;
   for (int o = 0; o < nout; ++o) {
-    st = copy_back(dout[o], out[o]);
+    st = copy_back(dout[o], out[o], 0, G.nz, sm);
     if (st != CST_OK) return st;
   }
-  if (nsteps > 1)
-    for (int a = 0; a < nin; ++a) {
-      st = copy_back(din[a], const_cast<double*>(in[a]));
-      if (st != CST_OK) return st;
-    }
+  for (int a = 0; a < nin; ++a) {
+    st = copy_back(din[a], const_cast<double*>(in[a]), 0, G.nz, sm);
+    if (st != CST_OK) return st;
+  }
   CST_CUDA(cudaStreamSynchronize(sm));
   CST_CUDA(cudaGetLastError());
   return CST_OK;

@@ -123,7 +123,8 @@ namespace cst {
 
 struct cst_stencil {
   cst_stencil_desc desc{};
-  std::vector<double> coeffs;
+  std::vector<double> coeffs;   // as given (desc.n_coeffs)
+  std::vector<double> kcoef;    // kernel coefficient bank (coeffs + derived weights)
   cst_grid grid{};
   int device = 0;
   cst::StencilInfo info{};
@@ -135,5 +136,6 @@ struct cst_stencil {
   std::vector<double*> dev_bufs;
   size_t dev_buf_elems = 0;
   cudaStream_t host_stream = nullptr;
+  cudaStream_t host_in_stream = nullptr, host_out_stream = nullptr;
   int64_t last_launches = 0;
 };

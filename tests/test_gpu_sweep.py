@@ -214,3 +214,30 @@ def test_invalid_arguments_on_gpu():
         C.cst_sweep(h, bad, [t.data_ptr()], [t2.data_ptr()])
     assert e.value.status == C.CST_E_CONSTRAINT
     C.cst_stencil_destroy(h)
+
+
+def test_host_path_multistep_and_chunked():
+    kind, r = 1, 2
+    L = H.layout((48, 40, 70), r)                      # 70 planes -> several pipeline chunks
+    c = H.coeffs(kind, r, "random", seed=8)
+    ins = H.inputs(kind, L, seed=12)
+    g = C.cst_grid(L.nx, L.ny, L.nz, L.halo, L.lead_x, L.pitch_x, L.pitch_y)
+    h = C.cst_stencil_create(kind, r, list(c), g)
+    s = C.cst_setting_default(h)
+    # one step, pipelined over z-chunks
+    _, want = H.oracle_outputs(kind, r, c, L, ins)
+    hin = [torch.from_numpy(ins[0].copy()).pin_memory()]
+    hout = [torch.full((L.numel,), float("nan"), dtype=torch.float64).pin_memory()]
+    C.cst_sweep_host(h, s, [t.data_ptr() for t in hin], [t.data_ptr() for t in hout], 1)
+    assert C.cst_last_launch_count(h) > 1
+    H.assert_parity(L, hout[0].numpy(), want[0], "host chunked")
+    H.assert_halo_untouched(L, hout[0].numpy(), np.full(L.numel, np.nan))
+    # two steps (ping-pong through the host buffers)
+    out0 = ins[0].copy()
+    H.interior(L, out0)[...] = np.nan
+    win, wout = H.oracle_outputs(kind, r, c, L, ins, nsteps=2)
+    hin = [torch.from_numpy(ins[0].copy()).pin_memory()]
+    hout = [torch.from_numpy(out0).pin_memory()]
+    C.cst_sweep_host(h, s, [t.data_ptr() for t in hin], [t.data_ptr() for t in hout], 2)
+    H.assert_parity(L, hin[0].numpy(), win[0], "host T=2")
+    C.cst_stencil_destroy(h)
