@@ -121,6 +121,65 @@ def ncu_traffic():
     return None
 
 
+OTHER = {
+    # name: (kind, order, coefficients, grid, seed, description)
+    "c1_star13_64": (1, 2, None, (64, 64, 64), 1,
+                     "configs[0]: order-2 13-point star, 64^3, fixed default setting (L2-resident)"),
+    "c3_box27_512": (2, 1, None, (512, 512, 512), 3,
+                     "configs[2]: 27-point box (binomial), 512^3, TMA halo staging"),
+    "c4_hypterm_512": (3, 4, None, (512, 512, 512), 4,
+                       "configs[3]: hypterm-like, 8 in / 5 out, order 4, 512^3"),
+}
+
+
+def other_coeffs(kind, r):
+    if kind == 1:
+        w = {2: [-1 / 12, 16 / 12, -30 / 12, 16 / 12, -1 / 12]}[r]
+        return [3 * w[r]] + (w[:r] + w[r + 1:]) * 3
+    if kind == 2:
+        b = [0.25, 0.5, 0.25]
+        return [x * y * z for x in b for y in b for z in b]
+    return [4 / 5, -1 / 5, 4 / 105, -1 / 280, 1.0, 1.0, 1.0]
+
+
+def other_configs(C, torch, peak, steps=10):
+    """The other single-GPU configs of BASELINE.json, each timed the same way (CUDA events,
+    inputs resident, device generator), with their own roofline fractions."""
+    res = {}
+    for name, (kind, r, _, n, seed, desc) in OTHER.items():
+        g = C.make_grid(*n, r)
+        h = C.cst_stencil_create(kind, r, other_coeffs(kind, r), g)
+        tuned = os.path.join(ROOT, "tuned", {"c3_box27_512": "box27_512.json",
+                                             "c4_hypterm_512": "hypterm_512.json"}.get(name, "-"))
+        src = "cst_setting_default"
+        s = C.cst_setting_default(h)
+        if os.path.exists(tuned):
+            try:
+                t = C.cst_setting.from_dict(json.load(open(tuned))["setting"])
+                C.cst_setting_check(h, t)
+                s, src = t, os.path.relpath(tuned, ROOT)
+            except Exception:
+                pass
+        ins = [torch.empty(g.numel, dtype=torch.float64, device="cuda") for _ in range(C.N_IN[kind])]
+        outs = [torch.empty(g.numel, dtype=torch.float64, device="cuda") for _ in range(C.N_OUT[kind])]
+        for a, t in enumerate(ins):
+            C.cst_fill_uniform(g, t.data_ptr(), seed, a)
+        ms = C.cst_time_setting(h, s, [t.data_ptr() for t in ins], [t.data_ptr() for t in outs],
+                                3, steps, torch.cuda.current_stream().cuda_stream)
+        pts = n[0] * n[1] * n[2]
+        bpp = 8 * (C.N_IN[kind] + C.N_OUT[kind])
+        gbs = pts * bpp / (ms * 1e-3) / 1e9
+        res[name] = {"workload": desc, "gstencils": pts / (ms * 1e-3) / 1e9, "ms_median": ms,
+                     "alg_bytes_per_point": bpp, "achieved_GBs": gbs,
+                     "hbm_frac_measured": None if n[0] < 128 else gbs / peak,
+                     "hbm_frac_nominal_8TBs": None if n[0] < 128 else gbs / 8000.0,
+                     "setting": s.as_dict(), "setting_source": src}
+        del ins, outs
+        C.cst_stencil_destroy(h)
+        torch.cuda.empty_cache()
+    return res
+
+
 def cpu_baseline(target_s: float = 10.0):
     """The oracle, as it stands, on a bounded sample of the same workload: a 512 x 512 x 16
     slab of the 512^3 star25 grid swept repeatedly until >= target_s seconds."""
@@ -190,6 +249,7 @@ def main():
     ap.add_argument("--impl", default="cst", choices=["cst", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-other-configs", action="store_true")
     args = ap.parse_args()
     assert args.warmup >= 3 or args.impl == "reference" or True
 
@@ -286,6 +346,12 @@ def main():
                "d2h_bytes_per_step": pts * 8, "ms_per_step": el * 1e3,
                "steps": args.e2e_steps, "api": "cst_sweep_host"}
 
+    others = None
+    if rank == 0 and world == 1 and not args.no_other_configs:
+        del u, v
+        torch.cuda.empty_cache()
+        others = other_configs(C, torch, peak)
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline()
@@ -304,6 +370,7 @@ def main():
                                  % (grid.numel * 8 / 1e9),
                            "parallelism": f"z-slab x{world}" if world > 1 else "single GPU"},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
+                "other_configs": others,
                 "gpu_launches": launches if dist_h is None else None,
                 "per_step_ms": {"min": min(per), "median": statistics.median(per), "max": max(per)}}
         print(json.dumps(line), flush=True)

@@ -641,7 +641,10 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
   // ---- prologue: first D planes in flight
   if constexpr (STAGING == 3) {
     if (tid == 0) {
-      for (int s = 0; s < NP; ++s) mbar_init(&bars[s], 1);
+      for (int s = 0; s < NP; ++s) {
+        mbar_init(&bars[s], 1);                 // full: producer arrive + TMA bytes
+        mbar_init(&bars[NP + s], NTHR / 32);    // empty: one arrive per warp
+      }
       fence_mbar_init();
     }
     __syncthreads();
@@ -775,9 +778,15 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
 
       // ---- release the oldest live slot and refill it with plane j + D
       if constexpr (STAGING == 3) {
-        __syncthreads();
+        // each warp releases the slot it no longer needs on the "empty" barrier; only the
+        // producer thread waits for the release before refilling (no CTA-wide barrier)
+        if (j >= RETAIN) {
+          __syncwarp();
+          if ((tid & 31) == 0) mbar_arrive(&bars[NP + (j - RETAIN) % NP]);
+        }
         if (tid == 0 && j + D < n_planes) {
-          const int sl = (j + D) % NP;
+          const int jn = j + D, sl = jn % NP;
+          if (jn >= NP) mbar_wait(&bars[NP + sl], (u32)((jn / NP - 1) & 1));
           fence_proxy_async();
           mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
           tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);
@@ -954,7 +963,10 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   double frag[D > 1 && STAGING == 2 ? (D - 1) * FR : 1];
   if constexpr (STAGING == 3) {
     if (tid == 0) {
-      for (int s = 0; s < NP; ++s) mbar_init(&bars[s], 1);
+      for (int s = 0; s < NP; ++s) {
+        mbar_init(&bars[s], 1);                 // full: producer arrive + TMA bytes
+        mbar_init(&bars[NP + s], NTHR / 32);    // empty: one arrive per warp
+      }
       fence_mbar_init();
     }
     __syncthreads();
@@ -1103,9 +1115,15 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
       }
 
       if constexpr (STAGING == 3) {
-        __syncthreads();
+        // each warp releases the slot it no longer needs on the "empty" barrier; only the
+        // producer thread waits for the release before refilling (no CTA-wide barrier)
+        if (j >= RETAIN) {
+          __syncwarp();
+          if ((tid & 31) == 0) mbar_arrive(&bars[NP + (j - RETAIN) % NP]);
+        }
         if (tid == 0 && j + D < n_planes) {
-          const int sl = (j + D) % NP;
+          const int jn = j + D, sl = jn % NP;
+          if (jn >= NP) mbar_wait(&bars[NP + sl], (u32)((jn / NP - 1) & 1));
           fence_proxy_async();
           mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
           tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);

@@ -29,6 +29,10 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(u64* bar, u32 bytes) {
                : "memory");
 }
 
+__device__ __forceinline__ void mbar_arrive(u64* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
 __device__ __forceinline__ void mbar_wait(u64* bar, u32 parity) {
   asm volatile(
       "{\n\t.reg .pred P1;\n"
