@@ -19,6 +19,10 @@
 #include "cst_params.h"
 #include "cst_ptx.cuh"
 
+#ifndef CST_EMPTY_BARRIERS
+#define CST_EMPTY_BARRIERS 0
+#endif
+
 // ------------------------------------------------------------------ configuration
 constexpr int KIND = CST_KIND;  // 1 star, 2 box, 3 hypterm
 constexpr int R = CST_R;
@@ -46,9 +50,10 @@ constexpr int BMA = BMX, BMB = SZ ? BMY : BMZ, BMS = SZ ? BMZ : BMY;
 constexpr int CMA = CMX, CMB = SZ ? CMY : CMZ, CMS = SZ ? CMZ : CMY;
 constexpr int UFA = UFX, UFB = SZ ? UFY : UFZ, UFS = SZ ? UFZ : UFY;
 constexpr int TA = TBA * BMA * CMA, TB = TBB * BMB * CMB, TS = TBS * BMS * CMS;
-// register budget: the hypterm fast path keeps 45 FP64 accumulators per point; asking for
-// 3 resident CTAs of <= 128 threads lets ptxas fit it in 168 registers
-constexpr int MINB = 1;  // (3 for the hypterm fast path spills a few bytes; kept at 1)
+// minimum resident CTAs requested from ptxas (__launch_bounds__); 3 would fit the
+// 45-accumulator hypterm path in 168 registers but spills a few bytes, so it stays 0
+// (= no request, ptxas' own heuristic, which measured best)
+constexpr int MINB = 0;
 
 __constant__ double c_coef[CST_MAX_COEF];
 
@@ -642,8 +647,10 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
   if constexpr (STAGING == 3) {
     if (tid == 0) {
       for (int s = 0; s < NP; ++s) {
-        mbar_init(&bars[s], 1);                 // full: producer arrive + TMA bytes
-        mbar_init(&bars[NP + s], NTHR / 32);    // empty: one arrive per warp
+        mbar_init(&bars[s], 1);  // full: producer arrive + TMA bytes
+#if CST_EMPTY_BARRIERS
+        mbar_init(&bars[NP + s], NTHR / 32);  // empty: one arrive per warp
+#endif
       }
       fence_mbar_init();
     }
@@ -778,8 +785,8 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
 
       // ---- release the oldest live slot and refill it with plane j + D
       if constexpr (STAGING == 3) {
-        // each warp releases the slot it no longer needs on the "empty" barrier; only the
-        // producer thread waits for the release before refilling (no CTA-wide barrier)
+#if CST_EMPTY_BARRIERS
+        // per-warp release on an "empty" mbarrier; only the producer waits (experimental)
         if (j >= RETAIN) {
           __syncwarp();
           if ((tid & 31) == 0) mbar_arrive(&bars[NP + (j - RETAIN) % NP]);
@@ -787,6 +794,13 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
         if (tid == 0 && j + D < n_planes) {
           const int jn = j + D, sl = jn % NP;
           if (jn >= NP) mbar_wait(&bars[NP + sl], (u32)((jn / NP - 1) & 1));
+#else
+        // CTA barrier: every warp is done with the slot of plane j - RETAIN, which is then
+        // refilled with plane j + D
+        __syncthreads();
+        if (tid == 0 && j + D < n_planes) {
+          const int sl = (j + D) % NP;
+#endif
           fence_proxy_async();
           mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
           tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);
@@ -964,8 +978,10 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   if constexpr (STAGING == 3) {
     if (tid == 0) {
       for (int s = 0; s < NP; ++s) {
-        mbar_init(&bars[s], 1);                 // full: producer arrive + TMA bytes
-        mbar_init(&bars[NP + s], NTHR / 32);    // empty: one arrive per warp
+        mbar_init(&bars[s], 1);  // full: producer arrive + TMA bytes
+#if CST_EMPTY_BARRIERS
+        mbar_init(&bars[NP + s], NTHR / 32);  // empty: one arrive per warp
+#endif
       }
       fence_mbar_init();
     }
@@ -1115,8 +1131,8 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
       }
 
       if constexpr (STAGING == 3) {
-        // each warp releases the slot it no longer needs on the "empty" barrier; only the
-        // producer thread waits for the release before refilling (no CTA-wide barrier)
+#if CST_EMPTY_BARRIERS
+        // per-warp release on an "empty" mbarrier; only the producer waits (experimental)
         if (j >= RETAIN) {
           __syncwarp();
           if ((tid & 31) == 0) mbar_arrive(&bars[NP + (j - RETAIN) % NP]);
@@ -1124,6 +1140,13 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
         if (tid == 0 && j + D < n_planes) {
           const int jn = j + D, sl = jn % NP;
           if (jn >= NP) mbar_wait(&bars[NP + sl], (u32)((jn / NP - 1) & 1));
+#else
+        // CTA barrier: every warp is done with the slot of plane j - RETAIN, which is then
+        // refilled with plane j + D
+        __syncthreads();
+        if (tid == 0 && j + D < n_planes) {
+          const int sl = (j + D) % NP;
+#endif
           fence_proxy_async();
           mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
           tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);
@@ -1250,7 +1273,7 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
 // =============================================================================
 // entry point
 // =============================================================================
-extern "C" __global__ void __launch_bounds__(NTHR, MINB) cst_kernel(const __grid_constant__ cst_kparams P) {
+extern "C" __global__ void __launch_bounds__(NTHR) cst_kernel(const __grid_constant__ cst_kparams P) {
   extern __shared__ __align__(128) double cst_smem[];
   if constexpr (!STREAM) {
     kernel_tile3d(P, cst_smem);

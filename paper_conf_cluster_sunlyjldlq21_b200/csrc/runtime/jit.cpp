@@ -132,9 +132,18 @@ static std::string prefix_for(const StencilInfo& st, const Tuple& t) {
 cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
                      double* compile_s) {
   const std::string src = prefix_for(st, t);
-  static const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo",
-                               "--fmad=true", "-default-device", "-DCST_NVRTC=1"};
-  const int nopts = sizeof(opts) / sizeof(opts[0]);
+  std::vector<std::string> optv = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo",
+                                   "--fmad=true", "-default-device", "-DCST_NVRTC=1"};
+  // experiment hook: extra -D options (e.g. "-DCST_EMPTY_BARRIERS=1"), part of the cache key
+  if (const char* e = std::getenv("CST_NVRTC_DEFINES")) {
+    std::stringstream ss(e);
+    std::string tok;
+    while (ss >> tok) optv.push_back(tok);
+  }
+  std::vector<const char*> optp;
+  for (const std::string& o : optv) optp.push_back(o.c_str());
+  const char* const* opts = optp.data();
+  const int nopts = (int)optp.size();
   const Nvrtc* N = nvrtc_lib();
   if (!N) return fail(CST_E_NVRTC, "libnvrtc.so.12 not found (set CST_NVRTC_PATH)");
   std::string keysrc = src + "nvrtc" + std::to_string(N->major) + "." + std::to_string(N->minor);

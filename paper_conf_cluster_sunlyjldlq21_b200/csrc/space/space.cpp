@@ -111,7 +111,7 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
       NP = D * T[sd] + 2 * r;
   }
   const int64_t plane = (plane_elems * 8 + 127) / 128 * 128;
-  const int64_t bars = t[F_STAGING] == 3 ? 2 * NP * 8 : 0;  // full + empty mbarriers
+  const int64_t bars = t[F_STAGING] == 3 ? 2 * NP * 8 : 0;  // full (+ optional empty) mbarriers
   return n_arrays(kind) * NP * plane + bars;
 }
 
