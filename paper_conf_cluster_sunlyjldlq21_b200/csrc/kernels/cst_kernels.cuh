@@ -22,6 +22,9 @@
 #ifndef CST_EMPTY_BARRIERS
 #define CST_EMPTY_BARRIERS 0
 #endif
+#ifndef CST_HYP_SCALAR
+#define CST_HYP_SCALAR 0
+#endif
 
 // ------------------------------------------------------------------ configuration
 constexpr int KIND = CST_KIND;  // 1 star, 2 box, 3 hypterm
@@ -875,6 +878,35 @@ __device__ __forceinline__ void hyp_inplane(const Ctx& C, const LD* ld, const in
   constexpr int NL = AXIS == 0 ? NCB * CMA : NCA * CMB;  // lines
   constexpr int NPL = AXIS == 0 ? BMA : BMB;             // points per line
   const double dxi = C.coef(4 + DIR);
+#if CST_HYP_SCALAR
+  // experimental: no windows, 12 scalar loads per k (fewer live registers)
+#pragma unroll
+  for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+    for (int ia = 0; ia < NCA; ++ia) {
+      auto at = [&](int arr, int kk) {
+        return AXIS == 0 ? ld[arr].at(la[ia] + kk, lb[ib]) : ld[arr].at(la[ia], lb[ib] + kk);
+      };
+      double sum[5];
+#pragma unroll
+      for (int k = 1; k <= 4; ++k) {
+        const double qp = at(QD, k), qm = at(QD, -k), p4 = at(7, k), m4 = at(7, -k);
+        const double a = C.coef(k - 1);
+#pragma unroll
+        for (int m = 0; m < 4; ++m) {
+          const double cp = at(m, k), cm = at(m, -k);
+          if (m == DIR) sum[0] = (k == 1) ? a * (cp - cm) : fma(a, cp - cm, sum[0]);
+          double e = fma(cp, qp, -(cm * qm));
+          if (m == 3) e = e + fma(p4, qp, -(m4 * qm));
+          else if (m == DIR) e = e + (p4 - m4);
+          sum[m + 1] = (k == 1) ? a * e : fma(a, e, sum[m + 1]);
+        }
+      }
+#pragma unroll
+      for (int f = 0; f < 5; ++f) t[f][ib][ia] = dxi * sum[f];
+    }
+  return;
+#endif
 #pragma unroll
   for (int line = 0; line < NL; ++line) {
     // line -> (run start la0, lb0) and point (ib, ia) of its t-th point
