@@ -306,7 +306,7 @@ def main():
     evs[0].record(stream)
     for i in range(args.steps):
         step()
-        launches += C.cst_last_launch_count(h) if dist_h is None else 0
+        launches += C.cst_last_launch_count(h)
         evs[i + 1].record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -371,7 +371,7 @@ def main():
                            "parallelism": f"z-slab x{world}" if world > 1 else "single GPU"},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
                 "other_configs": others,
-                "gpu_launches": launches if dist_h is None else None,
+                "gpu_launches": launches,
                 "per_step_ms": {"min": min(per), "median": statistics.median(per), "max": max(per)}}
         print(json.dumps(line), flush=True)
     if dist_h is not None:

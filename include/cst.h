@@ -162,6 +162,15 @@ cst_status cst_time_setting(cst_stencil* h, const cst_setting* s, const double* 
                             double* const* out, int32_t warmup, int32_t reps, void* stream,
                             double* ms);
 
+/* Hardware counters of one sweep (CUPTI range profiler, user range + user replay: the
+ * sweep is re-run once per counter pass).  names: metric names as ncu / CUPTI spell them
+ * (e.g. "dram__bytes_read.sum"); values[n] receives their GPU values.  CST_E_UNSUPPORTED
+ * when libcupti is missing or counters are not permitted.  (the paper
+ * collects its dataset's GPU metrics with Nsight.) */
+cst_status cst_collect_metrics(cst_stencil* h, const cst_setting* s, const double* const* in,
+                               double* const* out, const char* const* names, int32_t n,
+                               double* values);
+
 /* ------------------------------------------------------------------------ tuner */
 /* csTuner method: dataset, CV + Algorithm 1 grouping
  * (P:155-230), PCC + Algorithm 2 metric combination, PMNF surrogate + RSE
@@ -187,6 +196,8 @@ typedef struct {
   int32_t n_user_metrics;    /* metrics supplied by the eval callback (0 = model) */
   int32_t quantile_sample;   /* settings sampled to set thresholds / gene tables  */
   int32_t warm_start;        /* 1: add cst_setting_default() to the dataset (ours) */
+  int32_t metrics_mode;      /* 0: CUPTI counters for the dataset if available, else
+                                modelled features; 1: modelled features only        */
 } cst_tune_opts;
 
 typedef struct {

@@ -289,6 +289,22 @@ static const char* const kModelMetricNames[] = {
     "ctas",             "ctas_per_sm",     "waves",       "pts_per_thread", "smem_loads_per_pt"};
 static const int kModelMetrics = 10;
 
+// Hardware counters of the dataset (SURVEY Q22 default set; PM counters only).
+static const char* const kHwMetricNames[] = {
+    "dram__bytes_read.sum",
+    "dram__bytes_write.sum",
+    "lts__t_bytes.sum",
+    "lts__t_sector_hit_rate.pct",
+    "l1tex__t_bytes.sum",
+    "l1tex__throughput.avg.pct_of_peak_sustained_active",
+    "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum",
+    "l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum",
+    "sm__throughput.avg.pct_of_peak_sustained_elapsed",
+    "sm__warps_active.avg.pct_of_peak_sustained_active",
+    "sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active",
+    "smsp__inst_executed.sum"};
+static const int kHwMetrics = 12;
+
 std::vector<double> model_metrics(const cst_stencil* h, const Tuple& t) {
   const int kind = h->info.kind, r = h->info.r;
   const int nin = kind == CST_HYPTERM ? 8 : 1, nout = kind == CST_HYPTERM ? 5 : 1;
@@ -373,6 +389,7 @@ extern "C" void cst_tune_opts_default(cst_tune_opts* o) {
   o->n_user_metrics = 0;
   o->quantile_sample = 65536;
   o->warm_start = 1;
+  o->metrics_mode = 0;
 }
 
 namespace {
@@ -394,8 +411,14 @@ struct Evaluator {
   uint64_t jit_before = 0;
   cudaStream_t stream = nullptr;
   cst_status err = CST_OK;
+  bool use_hw = false;      // collect CUPTI counters for the rows evaluated now (dataset)
+  bool hw_ok = true;        // cleared on the first CUPTI failure -> modelled features
+  std::string metrics_source = "model";
 
-  int n_metrics() const { return o->n_user_metrics > 0 ? o->n_user_metrics : kModelMetrics; }
+  int n_metrics() const {
+    if (o->n_user_metrics > 0) return o->n_user_metrics;
+    return metrics_source == "cupti" ? kHwMetrics : kModelMetrics;
+  }
 
   // evaluate (memoised) a batch; invalid settings (rules) get ms = inf without timing
   cst_status run(const std::vector<Tuple>& cands, std::vector<EvalResult>* res) {
@@ -440,12 +463,28 @@ struct Evaluator {
           ms[i] = st == CST_OK ? m : INFINITY;
         }
       }
+      // dataset rows: hardware counters through the CUPTI range profiler when possible
+      std::vector<std::vector<double>> hw(todo.size());
+      if (!cb && use_hw && hw_ok) {
+        for (size_t i = 0; i < todo.size() && hw_ok; ++i) {
+          if (!(ms[i] > 0 && std::isfinite(ms[i]))) continue;
+          std::vector<double> v(kHwMetrics);
+          const cst_status cs_ = cst_collect_metrics(h, &ss[i], in, out, kHwMetricNames,
+                                                     kHwMetrics, v.data());
+          if (cs_ == CST_OK) hw[i] = v;
+          else if (cs_ == CST_E_CUDA) return cs_;
+          else hw_ok = false;
+        }
+        metrics_source = hw_ok ? "cupti" : "model";
+      }
       for (size_t i = 0; i < todo.size(); ++i) {
         EvalResult r;
         r.ms = (ms[i] > 0 && std::isfinite(ms[i])) ? ms[i] : INFINITY;
         if (o->n_user_metrics > 0)
           r.metrics.assign(met.begin() + i * o->n_user_metrics,
                            met.begin() + (i + 1) * o->n_user_metrics);
+        else if (metrics_source == "cupti")
+          r.metrics = hw[i].empty() ? std::vector<double>(kHwMetrics, 0.0) : hw[i];
         else
           r.metrics = model_metrics(h, todo[i]);
         memo[todo[i]] = r;
@@ -522,14 +561,20 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
     rows.push_back(t);
   }
   std::vector<EvalResult> res;
+  ev.use_hw = (o->metrics_mode == 0);
   cst_status st = ev.run(rows, &res);
+  ev.use_hw = false;
   if (st != CST_OK) return st;
+  if (!eval && ev.metrics_source == "model")  // CUPTI unavailable: recompute uniformly
+    for (size_t i = 0; i < rows.size(); ++i) res[i].metrics = model_metrics(h, rows[i]);
   const double t_dataset = elapsed();
   // statistics use the valid rows only
   std::vector<int> valid;
   for (size_t i = 0; i < rows.size(); ++i)
     if (std::isfinite(res[i].ms)) valid.push_back((int)i);
   if (valid.size() < 4) return fail(CST_E_INTERNAL, "tuner: fewer than 4 valid dataset rows");
+  js.key("metrics_source");
+  js.o << "\"" << (o->n_user_metrics > 0 ? "callback" : ev.metrics_source) << "\"";
   js.key("dataset");
   js.o << "{\"ranks\": [";
   for (size_t i = 0; i < ranks.size(); ++i) js.o << (i ? "," : "") << ranks[i];

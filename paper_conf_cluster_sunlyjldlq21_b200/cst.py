@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(_HERE, "libcst.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(
-        f"{LIB_PATH} is missing: build it with `python -m paper_conf_cluster_sunlyjldlq21_b200.build`"
+        f"{LIB_PATH} is missing: build it with `python paper_conf_cluster_sunlyjldlq21_b200/build.py`"
         " (there is no fallback implementation)")
 
 _lib = ctypes.CDLL(LIB_PATH)
@@ -114,7 +114,7 @@ class cst_tune_opts(ctypes.Structure):
                 ("num_collections", ctypes.c_int32), ("time_budget_s", ctypes.c_double),
                 ("reps", ctypes.c_int32), ("warmup", ctypes.c_int32), ("log_path", ctypes.c_char_p),
                 ("n_user_metrics", ctypes.c_int32), ("quantile_sample", ctypes.c_int32),
-                ("warm_start", ctypes.c_int32)]
+                ("warm_start", ctypes.c_int32), ("metrics_mode", ctypes.c_int32)]
 
 
 class cst_tune_report(ctypes.Structure):
@@ -168,6 +168,8 @@ _decl("cst_fill_uniform", _S, ctypes.POINTER(cst_grid), _P, ctypes.c_uint64, cty
       ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_double, _P)
 _decl("cst_time_setting", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP, ctypes.c_int32,
       ctypes.c_int32, _P, ctypes.POINTER(ctypes.c_double))
+_decl("cst_collect_metrics", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP,
+      ctypes.POINTER(ctypes.c_char_p), ctypes.c_int32, ctypes.POINTER(ctypes.c_double))
 _decl("cst_tune_opts_default", None, ctypes.POINTER(cst_tune_opts))
 _decl("cst_tune", _S, _P, ctypes.POINTER(cst_tune_opts), _PP, _PP, EVAL_FN, _P,
       ctypes.POINTER(cst_setting), ctypes.POINTER(cst_tune_report))
@@ -299,6 +301,16 @@ def cst_time_setting(h, s: cst_setting, in_ptrs, out_ptrs, warmup=2, reps=5, str
     check(_lib.cst_time_setting(h, ctypes.byref(s), pi, po, warmup, reps, ctypes.c_void_p(stream),
                                 ctypes.byref(ms)))
     return ms.value
+
+
+def cst_collect_metrics(h, s: cst_setting, in_ptrs, out_ptrs, names):
+    """{metric name: value} of one sweep from the CUPTI range profiler."""
+    pi, _a = _ptrs(in_ptrs)
+    po, _b = _ptrs(out_ptrs)
+    arr = (ctypes.c_char_p * len(names))(*[n.encode() for n in names])
+    vals = (ctypes.c_double * len(names))()
+    check(_lib.cst_collect_metrics(h, ctypes.byref(s), pi, po, arr, len(names), vals))
+    return dict(zip(names, list(vals)))
 
 
 def cst_tune_opts_default() -> cst_tune_opts:
