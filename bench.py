@@ -154,7 +154,11 @@ OTHER = {
                      "configs[2]: 27-point box (binomial), 512^3, TMA halo staging"),
     "c4_hypterm_512": (3, 4, None, (512, 512, 512), 4,
                        "configs[3]: hypterm-like, 8 in / 5 out, order 4, 512^3"),
+    "next1_rhs4_320": (4, 2, None, (320, 320, 320), 6,
+                       "SURVEY NEXT-1: rhs4center-like (5 in / 3 out, order 2, 666 FLOPs/pt), "
+                       "320^3 as in Table III — FP64-bound"),
 }
+FLOPS_PER_POINT = {1: None, 2: 53, 3: 358, 4: 666}
 
 
 def other_coeffs(kind, r):
@@ -164,10 +168,12 @@ def other_coeffs(kind, r):
     if kind == 2:
         b = [0.25, 0.5, 0.25]
         return [x * y * z for x in b for y in b for z in b]
+    if kind == 4:
+        return [1.0, 1.0, 1.0]
     return [4 / 5, -1 / 5, 4 / 105, -1 / 280, 1.0, 1.0, 1.0]
 
 
-def other_configs(C, torch, peak, steps=10):
+def other_configs(C, torch, peak, steps=10, fp64_peak=None):
     """The other single-GPU configs of BASELINE.json, each timed the same way (CUDA events,
     inputs resident, device generator), with their own roofline fractions."""
     res = {}
@@ -175,7 +181,8 @@ def other_configs(C, torch, peak, steps=10):
         g = C.make_grid(*n, r)
         h = C.cst_stencil_create(kind, r, other_coeffs(kind, r), g)
         tuned = os.path.join(ROOT, "tuned", {"c3_box27_512": "box27_512.json",
-                                             "c4_hypterm_512": "hypterm_512.json"}.get(name, "-"))
+                                             "c4_hypterm_512": "hypterm_512.json",
+                                             "next1_rhs4_320": "rhs4_320.json"}.get(name, "-"))
         src = "cst_setting_default"
         s = C.cst_setting_default(h)
         if os.path.exists(tuned):
@@ -199,6 +206,11 @@ def other_configs(C, torch, peak, steps=10):
                      "hbm_frac_measured": None if n[0] < 128 else gbs / peak,
                      "hbm_frac_nominal_8TBs": None if n[0] < 128 else gbs / 8000.0,
                      "setting": s.as_dict(), "setting_source": src}
+        fpp = FLOPS_PER_POINT.get(kind)
+        if fpp and fp64_peak:
+            tf = pts * fpp / (ms * 1e-3) / 1e12
+            res[name].update({"flops_per_point_as_written": fpp, "achieved_TFLOPs": tf,
+                              "fp64_frac_measured": tf / fp64_peak})
         del ins, outs
         C.cst_stencil_destroy(h)
         torch.cuda.empty_cache()
@@ -386,7 +398,12 @@ def main():
     if rank == 0 and world == 1 and not args.no_other_configs:
         del u, v
         torch.cuda.empty_cache()
-        others = other_configs(C, torch, peak)
+        try:
+            fp64_peak, _ = C.cst_fp64_peak(local)
+        except Exception:
+            fp64_peak = None
+        others = other_configs(C, torch, peak, fp64_peak=fp64_peak)
+        others["fp64_peak_TFLOPs_measured"] = fp64_peak
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

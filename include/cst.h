@@ -45,7 +45,7 @@ const char* cst_last_error(void);           /* thread-local detail of the last f
 const char* cst_version(void);
 
 /* ------------------------------------------------------------------ stencil + grid */
-typedef enum { CST_STAR = 1, CST_BOX = 2, CST_HYPTERM = 3 } cst_kind;
+typedef enum { CST_STAR = 1, CST_BOX = 2, CST_HYPTERM = 3, CST_RHS4 = 4 } cst_kind;
 
 /* Stencil spec "with order, coefficients and input grids" (north_star; P:13 order = the
  * neighbour extent along each dimension = radius r; Table III shapes).
@@ -55,6 +55,9 @@ typedef enum { CST_STAR = 1, CST_BOX = 2, CST_HYPTERM = 3 } cst_kind;
  *   HYPTERM order 4, 8 in (cons1..4, q1..4) / 5 out (flux0..4), coeffs
  *           [a1, a2, a3, a4, dxinv_x, dxinv_y, dxinv_z] (7 values); Table III "hypterm"
  *           (358 FLOPs, 13 I/O arrays) — definition in DESIGN.md §2.
+ *   RHS4    order 2, 5 in (u1, u2, u3, mu, lambda) / 3 out (r1..r3), coeffs
+ *           [s_x, s_y, s_z]: rhs4center-like variable-coefficient elastic operator
+ *           (Table III "rhs4center", 666 FLOPs; SW4 [1]) — DESIGN.md §2 O7.
  * The coefficient array is copied at create time. */
 typedef struct {
   int32_t kind;
@@ -170,6 +173,10 @@ cst_status cst_time_setting(cst_stencil* h, const cst_setting* s, const double* 
 cst_status cst_collect_metrics(cst_stencil* h, const cst_setting* s, const double* const* in,
                                double* const* out, const char* const* names, int32_t n,
                                double* values);
+
+/* FP64 FMA throughput of the device (TFLOP/s, 2 FLOPs per DFMA), measured by a DFMA-chain
+ * microbenchmark: the FP64 roofline denominator.  *sm_clock_ghz = the device's max clock. */
+cst_status cst_fp64_peak(int device, double* tflops, double* sm_clock_ghz);
 
 /* ------------------------------------------------------------------------ tuner */
 /* csTuner method: dataset, CV + Algorithm 1 grouping

@@ -23,7 +23,7 @@
 
 namespace {
 
-enum Kind { STAR = 1, BOX = 2, HYPTERM = 3 };
+enum Kind { STAR = 1, BOX = 2, HYPTERM = 3, RHS4 = 4 };
 
 struct Grid {
   int64_t nx, ny, nz, halo, lead_x, pitch_x, pitch_y;
@@ -114,6 +114,77 @@ void hypterm_point(const Acc& U, const double* c, T* flux) {
   }
 }
 
+// NEXT-1 rhs4center-like (Table III "rhs4center": order 2, 666 FLOPs, 8 I/O arrays, P:339;
+// SW4 [1]; DESIGN.md §2 O7).  Inputs 0..4 = u1, u2, u3, mu, lambda; outputs r1..r3;
+// coefficients [s_x, s_y, s_z] (direction scales).  The variable-coefficient elastic
+// operator  r_i = sum_j d_j(mu (d_j u_i + d_i u_j)) + d_i(lambda div u)  with radius-2,
+// 4th-order operators:
+//   D_d[f]     = (f(-2) - 8 f(-1) + 8 f(+1) - f(+2)) / 12                (first derivative)
+//   V_d[a](f)  = ( m1 (f(-2)-f(0)) + m2 (f(-1)-f(0)) + m3 (f(+1)-f(0)) + m4 (f(+2)-f(0)) ) / 6
+//     m1 = a(-1) - 3/4 (a(0) + a(-2)),   m2 = a(-2) + a(+1) + 3 (a(0) + a(-1)),
+//     m3 = a(-1) + a(+2) + 3 (a(+1) + a(0)),   m4 = a(+1) - 3/4 (a(0) + a(+2))
+//   r_i = sum_d s_d^2 V_d[mu + delta_id (mu + lambda)](u_i)
+//       + sum_{d != i} s_d s_i ( D_d[mu * D_i u_d] + D_i[lambda * D_d u_d] )
+// summed in that order (d ascending); products are pointwise at the outer stencil's points.
+template <class T, class Acc>
+void rhs4_point(const Acc& U, const double* c, T* r) {
+  enum { U1 = 0, U2, U3, MU, LA };
+  auto sh = [](int d, int k, int* o) { o[0] = o[1] = o[2] = 0; o[d] = k; };
+  for (int i = 0; i < 3; ++i) {
+    T acc = T(0.0);
+    for (int d = 0; d < 3; ++d) {
+      // a(k) = mu(k) (+ mu(k) + lambda(k) on the diagonal d == i), along e_d
+      auto a = [&](int k) {
+        int o[3];
+        sh(d, k, o);
+        T m = U(MU, o[0], o[1], o[2]);
+        if (d == i) return m + (m + U(LA, o[0], o[1], o[2]));
+        return m;
+      };
+      auto f = [&](int k) {
+        int o[3];
+        sh(d, k, o);
+        return U(U1 + i, o[0], o[1], o[2]);
+      };
+      const T am2 = a(-2), am1 = a(-1), a0 = a(0), ap1 = a(1), ap2 = a(2);
+      const T m1 = am1 - T(0.75) * (a0 + am2);
+      const T m2 = am2 + ap1 + T(3.0) * (a0 + am1);
+      const T m3 = am1 + ap2 + T(3.0) * (ap1 + a0);
+      const T m4 = ap1 - T(0.75) * (a0 + ap2);
+      const T f0 = f(0);
+      const T v = (m1 * (f(-2) - f0) + m2 * (f(-1) - f0) + m3 * (f(1) - f0) + m4 * (f(2) - f0)) *
+                  T(1.0 / 6.0);
+      const T term = (T(c[d]) * T(c[d])) * v;
+      acc = (d == 0) ? term : acc + term;
+    }
+    for (int d = 0; d < 3; ++d) {
+      if (d == i) continue;
+      // D along `outer` of (coef array) * (D along `inner` of u_comp), products at the
+      // outer stencil's points
+      auto mixed = [&](int outer, int inner, int coef, int comp) {
+        auto inner_d = [&](int ko) {
+          auto at = [&](int ki) {
+            int o[3] = {0, 0, 0};
+            o[outer] += ko;
+            o[inner] += ki;
+            return U(comp, o[0], o[1], o[2]);
+          };
+          int o[3] = {0, 0, 0};
+          o[outer] += ko;
+          const T g = ((at(-2) - at(2)) + T(8.0) * (at(1) - at(-1))) * T(1.0 / 12.0);
+          return U(coef, o[0], o[1], o[2]) * g;
+        };
+        return ((inner_d(-2) - inner_d(2)) + T(8.0) * (inner_d(1) - inner_d(-1))) *
+               T(1.0 / 12.0);
+      };
+      const T sdi = T(c[d]) * T(c[i]);
+      acc = acc + sdi * mixed(d, i, MU, U1 + d);   // d_d (mu d_i u_d)
+      acc = acc + sdi * mixed(i, d, LA, U1 + d);   // d_i (lambda d_d u_d)
+    }
+    r[i] = acc;
+  }
+}
+
 // FLOP-counting number type: counts + - * between counted values (negation is a sign
 // flip, not a FLOP, matching Table III's convention as reconstructed in SURVEY §8(c)).
 struct Flop {
@@ -127,20 +198,22 @@ struct Flop {
   Flop operator-() const { return Flop(-v); }
 };
 
-int n_inputs(int kind) { return kind == HYPTERM ? 8 : 1; }
-int n_outputs(int kind) { return kind == HYPTERM ? 5 : 1; }
+int n_inputs(int kind) { return kind == HYPTERM ? 8 : (kind == RHS4 ? 5 : 1); }
+int n_outputs(int kind) { return kind == HYPTERM ? 5 : (kind == RHS4 ? 3 : 1); }
 
 template <class Acc>
 void point(int kind, int r, const double* c, const Acc& U, double* out) {
   if (kind == STAR) star_point<double>(U, r, c, out);
   else if (kind == BOX) box_point<double>(U, r, c, out);
-  else hypterm_point<double>(U, c, out);
+  else if (kind == HYPTERM) hypterm_point<double>(U, c, out);
+  else rhs4_point<double>(U, c, out);
 }
 
 bool valid_kind(int kind, int r) {
   if (kind == STAR) return r >= 1 && r <= 4;
   if (kind == BOX) return r == 1;
   if (kind == HYPTERM) return r == 4;
+  if (kind == RHS4) return r == 2;
   return false;
 }
 
@@ -166,7 +239,7 @@ int oracle_sweep(int kind, int order, const double* coeffs, int64_t nx, int64_t 
   for (int step = 0; step < nsteps; ++step) {
 #pragma omp parallel for schedule(static) num_threads(nthreads > 0 ? nthreads : 1)
     for (int64_t z = 0; z < nz; ++z) {
-      double res[5];
+      double res[5];  // up to 5 outputs
       for (int64_t y = 0; y < ny; ++y)
         for (int64_t x = 0; x < nx; ++x) {
           auto U = [&](int a, int dx, int dy, int dz) {
@@ -189,7 +262,7 @@ int oracle_point_gen(int kind, int order, const double* coeffs, uint64_t seed,
                      int array_id0, int64_t nx, int64_t ny, int64_t halo, int64_t x,
                      int64_t y, int64_t z, double* out) {
   if (!valid_kind(kind, order)) return 1;
-  uint64_t keys[8];
+  uint64_t keys[8];  // up to 8 inputs
   for (int a = 0; a < n_inputs(kind); ++a) keys[a] = cstgen_key(seed, (uint64_t)(array_id0 + a));
   auto U = [&](int a, int dx, int dy, int dz) {
     return cstgen_value(keys[a], cstgen_index(nx, ny, halo, x + dx, y + dy, z + dz));
@@ -206,6 +279,15 @@ int64_t oracle_hypterm_flops(void) {
   auto U = [](int, int, int, int) { return Flop(1.0); };
   Flop f[5];
   hypterm_point<Flop>(U, c, f);
+  return Flop::count;
+}
+
+int64_t oracle_rhs4_flops(void) {
+  Flop::count = 0;
+  const double c[3] = {1, 1, 1};
+  auto U = [](int, int, int, int) { return Flop(1.0); };
+  Flop f[3];
+  rhs4_point<Flop>(U, c, f);
   return Flop::count;
 }
 

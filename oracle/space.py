@@ -35,7 +35,7 @@ FIELDS = ("tb_x", "tb_y", "tb_z", "staging", "use_constant", "use_streaming", "s
           "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z", "bm_x", "bm_y", "bm_z",
           "use_retiming", "prefetch")
 
-STAR, BOX, HYPTERM = 1, 2, 3
+STAR, BOX, HYPTERM, RHS4 = 1, 2, 3, 4
 SMEM_LIMIT = 227 * 1024 - 1024      # data bytes; 1 KiB kept for mbarriers / alignment
 REG_LIMIT = 255
 
@@ -50,11 +50,11 @@ def p2(lo: int, hi: int):
 
 
 def n_arrays(kind: int) -> int:
-    return 8 if kind == HYPTERM else 1
+    return {HYPTERM: 8, RHS4: 5}.get(kind, 1)
 
 
 def live_doubles_per_point(kind: int, r: int) -> int:
-    return {STAR: 2 * r + 2, BOX: 12, HYPTERM: 50}[kind]
+    return {STAR: 2 * r + 2, BOX: 12, HYPTERM: 50, RHS4: 24}[kind]
 
 
 def retention(kind: int, r: int) -> int:

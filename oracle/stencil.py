@@ -16,9 +16,9 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
-STAR, BOX, HYPTERM = 1, 2, 3
-N_IN = {STAR: 1, BOX: 1, HYPTERM: 8}
-N_OUT = {STAR: 1, BOX: 1, HYPTERM: 5}
+STAR, BOX, HYPTERM, RHS4 = 1, 2, 3, 4
+N_IN = {STAR: 1, BOX: 1, HYPTERM: 8, RHS4: 5}
+N_OUT = {STAR: 1, BOX: 1, HYPTERM: 5, RHS4: 3}
 
 _DP = ctypes.POINTER(ctypes.c_double)
 
@@ -46,7 +46,7 @@ def lib():
         L.oracle_point_gen.argtypes = [ctypes.c_int, ctypes.c_int, _DP, ctypes.c_uint64,
                                        ctypes.c_int, i64, i64, i64, i64, i64, i64, _DP]
         L.oracle_point_gen.restype = ctypes.c_int
-        for f in ("oracle_hypterm_flops",):
+        for f in ("oracle_hypterm_flops", "oracle_rhs4_flops"):
             getattr(L, f).restype = i64
             getattr(L, f).argtypes = []
         for f in ("oracle_star_flops", "oracle_box_flops"):
@@ -93,6 +93,10 @@ def hypterm_flops() -> int:
     return int(lib().oracle_hypterm_flops())
 
 
+def rhs4_flops() -> int:
+    return int(lib().oracle_rhs4_flops())
+
+
 def star_flops(r: int) -> int:
     return int(lib().oracle_star_flops(r))
 
@@ -134,3 +138,7 @@ HYPTERM_A_INT = (672.0, -168.0, 32.0, -3.0)
 def hypterm_coeffs(integer: bool = False, dxinv=(1.0, 1.0, 1.0)) -> np.ndarray:
     a = HYPTERM_A_INT if integer else HYPTERM_A
     return np.array(list(a) + list(dxinv), dtype=np.float64)
+
+
+def rhs4_coeffs(scales=(1.0, 1.0, 1.0)) -> np.ndarray:
+    return np.array(scales, dtype=np.float64)

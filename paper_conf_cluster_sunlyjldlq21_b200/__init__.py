@@ -6,6 +6,6 @@ space (Table I of Sun et al., CLUSTER'21), plus the host C++ tuner and the z-sla
 distributed sweep.  This package is the thin ctypes binding (cst.py) and a small
 torch-tensor convenience layer (stencil.py).
 """
-from .cst import (CST_BOX, CST_HYPTERM, CST_STAR, CstError, cst_grid, cst_setting,  # noqa: F401
+from .cst import (CST_BOX, CST_HYPTERM, CST_RHS4, CST_STAR, CstError, cst_grid, cst_setting,  # noqa: F401
                   make_grid, version)
 from .stencil import Stencil  # noqa: F401

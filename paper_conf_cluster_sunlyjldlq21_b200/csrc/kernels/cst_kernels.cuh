@@ -27,7 +27,7 @@
 #endif
 
 // ------------------------------------------------------------------ configuration
-constexpr int KIND = CST_KIND;  // 1 star, 2 box, 3 hypterm
+constexpr int KIND = CST_KIND;  // 1 star, 2 box, 3 hypterm, 4 rhs4center-like
 constexpr int R = CST_R;
 constexpr int TBX = CST_TBX, TBY = CST_TBY, TBZ = CST_TBZ;
 constexpr int STAGING = CST_STAGING;  // 1 none, 2 smem ld/st, 3 TMA
@@ -41,8 +41,8 @@ constexpr int BMX = CST_BMX, BMY = CST_BMY, BMZ = CST_BMZ;
 constexpr bool RETIME = CST_RET == 2;
 constexpr int PF = CST_PF;  // pipeline stages (1 = no prefetch)
 
-constexpr int NIN = KIND == 3 ? 8 : 1;
-constexpr int NOUT = KIND == 3 ? 5 : 1;
+constexpr int NIN = KIND == 3 ? 8 : (KIND == 4 ? 5 : 1);
+constexpr int NOUT = KIND == 3 ? 5 : (KIND == 4 ? 3 : 1);
 constexpr int NTHR = TBX * TBY * TBZ;
 constexpr int TX = TBX * BMX * CMX, TY = TBY * BMY * CMY, TZ = TBZ * BMZ * CMZ;
 
@@ -185,11 +185,68 @@ __device__ __forceinline__ void hypterm_point(const Ctx& C, const Acc& U, double
   }
 }
 
+// rhs4center-like (NEXT-1; Table III "rhs4center"): inputs u1, u2, u3, mu, lambda,
+// outputs r1..r3, coefficients [s_x, s_y, s_z]; same terms and order as the oracle:
+//   r_i = sum_d s_d^2 V_d[mu + delta_id (mu + la)](u_i)
+//       + sum_{d != i} s_d s_i (D_d[mu D_i u_d] + D_i[la D_d u_d])
+template <class Acc>
+__device__ __forceinline__ void rhs4_point(const Ctx& C, const Acc& U, double* r) {
+  auto at = [&](int arr, int d, int k, int d2, int k2) {
+    int o[3] = {0, 0, 0};
+    o[d] += k;
+    o[d2] += k2;
+    return U(arr, o[0], o[1], o[2]);
+  };
+#pragma unroll
+  for (int i = 0; i < 3; ++i) {
+    double acc = 0.0;
+#pragma unroll
+    for (int d = 0; d < 3; ++d) {
+      auto a = [&](int k) {
+        const double m = at(3, d, k, d, 0);
+        return d == i ? m + (m + at(4, d, k, d, 0)) : m;
+      };
+      auto f = [&](int k) { return at(i, d, k, d, 0); };
+      const double am2 = a(-2), am1 = a(-1), a0 = a(0), ap1 = a(1), ap2 = a(2);
+      const double m1 = fma(-0.75, a0 + am2, am1);
+      const double m2 = fma(3.0, a0 + am1, am2 + ap1);
+      const double m3 = fma(3.0, ap1 + a0, am1 + ap2);
+      const double m4 = fma(-0.75, a0 + ap2, ap1);
+      const double f0 = f(0);
+      double v = m1 * (f(-2) - f0);
+      v = fma(m2, f(-1) - f0, v);
+      v = fma(m3, f(1) - f0, v);
+      v = fma(m4, f(2) - f0, v);
+      const double sd = C.coef(d);
+      const double term = (sd * sd) * (v * (1.0 / 6.0));
+      acc = d == 0 ? term : acc + term;
+    }
+#pragma unroll
+    for (int d = 0; d < 3; ++d) {
+      if (d == i) continue;
+      auto mixed = [&](int outer, int inner, int coef, int comp) {
+        auto inner_d = [&](int ko) {
+          const double g = ((at(comp, outer, ko, inner, -2) - at(comp, outer, ko, inner, 2)) +
+                            8.0 * (at(comp, outer, ko, inner, 1) - at(comp, outer, ko, inner, -1))) *
+                           (1.0 / 12.0);
+          return at(coef, outer, ko, outer, 0) * g;
+        };
+        return ((inner_d(-2) - inner_d(2)) + 8.0 * (inner_d(1) - inner_d(-1))) * (1.0 / 12.0);
+      };
+      const double sdi = C.coef(d) * C.coef(i);
+      acc = fma(sdi, mixed(d, i, 3, d), acc);
+      acc = fma(sdi, mixed(i, d, 4, d), acc);
+    }
+    r[i] = acc;
+  }
+}
+
 template <class Acc>
 __device__ __forceinline__ void point(const Ctx& C, const Acc& U, double* o) {
   if constexpr (KIND == 1) star_point(C, U, o);
   else if constexpr (KIND == 2) box_point(C, U, o);
-  else hypterm_point(C, U, o);
+  else if constexpr (KIND == 3) hypterm_point(C, U, o);
+  else rhs4_point(C, U, o);
 }
 
 // =============================================================================
@@ -1309,7 +1366,7 @@ extern "C" __global__ void __launch_bounds__(NTHR) cst_kernel(const __grid_const
   extern __shared__ __align__(128) double cst_smem[];
   if constexpr (!STREAM) {
     kernel_tile3d(P, cst_smem);
-  } else if constexpr (KIND != 3 && TS == 1) {
+  } else if constexpr ((KIND == 1 || KIND == 2) && TS == 1) {
     kernel_stream1(P, cst_smem);
   } else if constexpr (KIND == 3 && TS == 1) {
     kernel_hyp_stream1(P, cst_smem);

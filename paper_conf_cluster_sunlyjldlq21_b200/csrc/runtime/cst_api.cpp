@@ -143,6 +143,7 @@ extern "C" const char* cst_version(void) {
 static int expected_coeffs(int kind, int r) {
   if (kind == CST_STAR) return 6 * r + 1;
   if (kind == CST_BOX) return (2 * r + 1) * (2 * r + 1) * (2 * r + 1);
+  if (kind == CST_RHS4) return 3;
   return 7;
 }
 
@@ -151,10 +152,12 @@ extern "C" cst_status cst_stencil_create(const cst_stencil_desc* desc, const cst
   if (!desc || !g || !out) return fail(CST_E_INVALID, "null argument");
   const int kind = desc->kind, r = desc->order;
   const bool supported = (kind == CST_STAR && r >= 1 && r <= 4) ||
-                         (kind == CST_BOX && r == 1) || (kind == CST_HYPTERM && r == 4);
-  if (kind < 1 || kind > 3) return fail(CST_E_INVALID, "desc.kind");
+                         (kind == CST_BOX && r == 1) || (kind == CST_HYPTERM && r == 4) ||
+                         (kind == CST_RHS4 && r == 2);
+  if (kind < 1 || kind > 4) return fail(CST_E_INVALID, "desc.kind");
   if (!supported) return fail(CST_E_UNSUPPORTED, "(kind, order) not supported");
-  const int nin = kind == CST_HYPTERM ? 8 : 1, nout = kind == CST_HYPTERM ? 5 : 1;
+  const int nin = kind == CST_HYPTERM ? 8 : (kind == CST_RHS4 ? 5 : 1);
+  const int nout = kind == CST_HYPTERM ? 5 : (kind == CST_RHS4 ? 3 : 1);
   if (desc->n_inputs != nin || desc->n_outputs != nout)
     return fail(CST_E_INVALID, "desc.n_inputs / n_outputs do not match the kind");
   if (!desc->coeffs || desc->n_coeffs != expected_coeffs(kind, r))
@@ -229,7 +232,7 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
   // measured-good starting points on B200, shrunk to fit small grids:
   // streaming along z, TMA staging, retimed accumulators; star/box 64x8 tiles of 2x2
   // register blocks; hypterm 16x8 tiles, one point per thread.
-  const bool hyp = h->info.kind == CST_HYPTERM;
+  const bool hyp = h->info.kind == CST_HYPTERM || h->info.kind == CST_RHS4;
   cst_setting c{};
   c.tb[0] = hyp ? 16 : 32;
   c.tb[1] = hyp ? 8 : 4;

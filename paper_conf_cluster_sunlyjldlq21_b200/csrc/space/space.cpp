@@ -50,9 +50,12 @@ std::string setting_key(const cst_setting& s) {
 static const int64_t SMEM_LIMIT = 227 * 1024 - 1024;
 static const int64_t REG_LIMIT = 255;
 
-static int n_arrays(int kind) { return kind == CST_HYPTERM ? 8 : 1; }
+static int n_arrays(int kind) {
+  return kind == CST_HYPTERM ? 8 : (kind == CST_RHS4 ? 5 : 1);
+}
 static int live_doubles(int kind, int r) {
-  return kind == CST_STAR ? 2 * r + 2 : (kind == CST_BOX ? 12 : 50);
+  return kind == CST_STAR ? 2 * r + 2
+                          : (kind == CST_BOX ? 12 : (kind == CST_HYPTERM ? 50 : 24));
 }
 static int retention(int kind, int r) { return kind == CST_BOX ? 2 * r : r; }
 
@@ -105,9 +108,9 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
     const int b = sd == 2 ? 1 : 2;
     plane_elems = (T[0] + 2 * XR) * (T[b] + 2 * r);
     const int64_t D = t[F_PF];
-    if (T[sd] == 1)
+    if (T[sd] == 1 && kind != CST_RHS4)  // fast streaming paths
       NP = D + (t[F_RET] == 2 ? 0 : retention(kind, r));
-    else
+    else                                 // generic ring
       NP = D * T[sd] + 2 * r;
   }
   const int64_t plane = (plane_elems * 8 + 127) / 128 * 128;

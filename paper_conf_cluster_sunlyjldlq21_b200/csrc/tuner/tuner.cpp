@@ -307,7 +307,8 @@ static const int kHwMetrics = 12;
 
 std::vector<double> model_metrics(const cst_stencil* h, const Tuple& t) {
   const int kind = h->info.kind, r = h->info.r;
-  const int nin = kind == CST_HYPTERM ? 8 : 1, nout = kind == CST_HYPTERM ? 5 : 1;
+  const int nin = kind == CST_HYPTERM ? 8 : (kind == CST_RHS4 ? 5 : 1);
+  const int nout = kind == CST_HYPTERM ? 5 : (kind == CST_RHS4 ? 3 : 1);
   const int64_t* M = h->info.M;
   double T[3];
   for (int d = 0; d < 3; ++d) T[d] = (double)t[F_TBX + d] * t[F_BMX + d] * t[F_CMX + d];
@@ -340,8 +341,10 @@ std::vector<double> model_metrics(const cst_stencil* h, const Tuple& t) {
   double loads = 0;
   if (kind == CST_STAR) loads = (bma + 2 * r) / bma + 2.0 * r / bmb;
   else if (kind == CST_BOX) loads = (bma + 2) * (bmb + 2) / (bma * bmb);
-  else loads = 6 * ((bma + 8) / bma + (bmb + 8) / bmb) + 2;
-  if (!stream) loads = (kind == CST_BOX ? 27 : (kind == CST_STAR ? 6 * r + 1 : 100));
+  else if (kind == CST_HYPTERM) loads = 6 * ((bma + 8) / bma + (bmb + 8) / bmb) + 2;
+  else loads = 150;  // rhs4 generic path: every operand from the smem ring
+  if (!stream)
+    loads = (kind == CST_BOX ? 27 : (kind == CST_STAR ? 6 * r + 1 : (kind == CST_HYPTERM ? 100 : 150)));
   return {8.0 * (nin * over + nout), 8.0 * (nin * over * halo + nout), smem, regs, thr, ctas,
           occ, waves, ppt, loads};
 }

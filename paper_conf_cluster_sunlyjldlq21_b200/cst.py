@@ -24,9 +24,9 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 CST_OK, CST_E_INVALID, CST_E_UNSUPPORTED, CST_E_CONSTRAINT, CST_E_CUDA, CST_E_NVRTC, \
     CST_E_NCCL, CST_E_OOM, CST_E_INTERNAL = range(9)
-CST_STAR, CST_BOX, CST_HYPTERM = 1, 2, 3
-N_IN = {CST_STAR: 1, CST_BOX: 1, CST_HYPTERM: 8}
-N_OUT = {CST_STAR: 1, CST_BOX: 1, CST_HYPTERM: 5}
+CST_STAR, CST_BOX, CST_HYPTERM, CST_RHS4 = 1, 2, 3, 4
+N_IN = {CST_STAR: 1, CST_BOX: 1, CST_HYPTERM: 8, CST_RHS4: 5}
+N_OUT = {CST_STAR: 1, CST_BOX: 1, CST_HYPTERM: 5, CST_RHS4: 3}
 
 FIELDS = ("tb_x", "tb_y", "tb_z", "staging", "use_constant", "use_streaming", "sd", "sb",
           "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z", "bm_x", "bm_y", "bm_z",
@@ -170,6 +170,8 @@ _decl("cst_time_setting", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP, ctypes.
       ctypes.c_int32, _P, ctypes.POINTER(ctypes.c_double))
 _decl("cst_collect_metrics", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP,
       ctypes.POINTER(ctypes.c_char_p), ctypes.c_int32, ctypes.POINTER(ctypes.c_double))
+_decl("cst_fp64_peak", _S, ctypes.c_int, ctypes.POINTER(ctypes.c_double),
+      ctypes.POINTER(ctypes.c_double))
 _decl("cst_tune_opts_default", None, ctypes.POINTER(cst_tune_opts))
 _decl("cst_tune", _S, _P, ctypes.POINTER(cst_tune_opts), _PP, _PP, EVAL_FN, _P,
       ctypes.POINTER(cst_setting), ctypes.POINTER(cst_tune_report))
@@ -311,6 +313,13 @@ def cst_collect_metrics(h, s: cst_setting, in_ptrs, out_ptrs, names):
     vals = (ctypes.c_double * len(names))()
     check(_lib.cst_collect_metrics(h, ctypes.byref(s), pi, po, arr, len(names), vals))
     return dict(zip(names, list(vals)))
+
+
+def cst_fp64_peak(device: int = 0):
+    """(TFLOP/s, max SM clock GHz) from the DFMA-chain microbenchmark."""
+    t, g = ctypes.c_double(), ctypes.c_double()
+    check(_lib.cst_fp64_peak(device, ctypes.byref(t), ctypes.byref(g)))
+    return t.value, g.value
 
 
 def cst_tune_opts_default() -> cst_tune_opts:

@@ -17,7 +17,7 @@ def main():
                    "ranks": T.sample_ranks(12345, 1220000000, 16)}, f, indent=1)
     spaces = []
     for M in [(4, 4, 4), (8, 8, 8)]:
-        for kind, r in [(1, 2), (1, 4), (2, 1), (3, 4)]:
+        for kind, r in [(1, 2), (1, 4), (2, 1), (3, 4), (4, 2)]:
             n, h = S.fnv1a64_stream(S.enumerate_space(kind, r, M))
             spaces.append({"M": list(M), "kind": kind, "order": r, "count": n, "fnv1a64": hex(h)})
     with open(os.path.join(HERE, "space.json"), "w") as f:

@@ -12,15 +12,19 @@ TOL = 1e-12   # north_star: 1e-12 relative max-norm (covers FMA contraction + re
 def coeffs(kind, r, variant="config", seed=0):
     if variant == "random":
         rng = np.random.default_rng(1000 + seed)
-        n = {1: 6 * r + 1, 2: 27, 3: 7}[kind]
+        n = {1: 6 * r + 1, 2: 27, 3: 7, 4: 3}[kind]
         c = rng.uniform(-1, 1, n)
         if kind == 3:
             c[4:] = rng.uniform(0.5, 2.0, 3)
+        if kind == 4:
+            c = rng.uniform(0.5, 2.0, 3)
         return c
     if kind == 1:
         return ost.star_laplacian_coeffs(r)
     if kind == 2:
         return ost.box_binomial_coeffs()
+    if kind == 4:
+        return ost.rhs4_coeffs()
     return ost.hypterm_coeffs()
 
 

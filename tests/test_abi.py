@@ -32,7 +32,8 @@ def test_exports_every_declared_symbol():
 
 
 def coeffs_for(kind, r):
-    return {C.CST_STAR: [1.0] * (6 * r + 1), C.CST_BOX: [1.0] * 27, C.CST_HYPTERM: [1.0] * 7}[kind]
+    return {C.CST_STAR: [1.0] * (6 * r + 1), C.CST_BOX: [1.0] * 27, C.CST_HYPTERM: [1.0] * 7,
+            C.CST_RHS4: [1.0] * 3}[kind]
 
 
 def handle(kind, r, n=(8, 8, 8), halo=None):
@@ -59,7 +60,7 @@ def test_create_validation():
     C.cst_stencil_destroy(h)
 
 
-@pytest.mark.parametrize("kind,r", [(1, 2), (1, 4), (2, 1), (3, 4)])
+@pytest.mark.parametrize("kind,r", [(1, 2), (1, 4), (2, 1), (3, 4), (4, 2)])
 def test_space_4cubed_matches_oracle_stream(kind, r):
     gold = json.load(open(os.path.join(GOLD, "space.json")))["spaces"]
     g = [e for e in gold if e["M"] == [4, 4, 4] and e["kind"] == kind and e["order"] == r][0]
@@ -110,7 +111,8 @@ def test_rank_unrank_roundtrip_512():
 def test_rules_agree_with_oracle_on_random_tuples():
     rng = random.Random(3)
     p2 = lambda hi: [1 << k for k in range(hi.bit_length()) if (1 << k) <= hi]
-    for kind, r, M in [(1, 4, (64, 32, 128)), (2, 1, (32, 64, 16)), (3, 4, (64, 64, 64))]:
+    for kind, r, M in [(1, 4, (64, 32, 128)), (2, 1, (32, 64, 16)), (3, 4, (64, 64, 64)),
+                       (4, 2, (32, 32, 64))]:
         h = handle(kind, r, M)
         agree_valid = 0
         for _ in range(3000):
@@ -147,14 +149,15 @@ def test_rules_agree_with_oracle_on_random_tuples():
 
 def test_default_setting_valid():
     for kind, r, n in [(1, 2, (64, 64, 64)), (1, 4, (512, 512, 512)), (2, 1, (512, 512, 512)),
-                       (3, 4, (512, 512, 512)), (1, 2, (4, 4, 4)), (3, 4, (8, 8, 8))]:
+                       (3, 4, (512, 512, 512)), (1, 2, (4, 4, 4)), (3, 4, (8, 8, 8)),
+                       (4, 2, (320, 320, 320))]:
         h = handle(kind, r, n)
         s = C.cst_setting_default(h)
         C.cst_setting_check(h, s)
         C.cst_stencil_destroy(h)
 
 
-@pytest.mark.parametrize("kind,r", [(1, 4), (1, 2), (2, 1), (3, 4)])
+@pytest.mark.parametrize("kind,r", [(1, 4), (1, 2), (2, 1), (3, 4), (4, 2)])
 def test_variants_compile_without_gpu(kind, r, tmp_path, monkeypatch):
     """Code generation + NVRTC for sm_100a of the default setting and random valid settings
     drawn from the canonical space (every path: streaming fast/generic, 3-D tiles)."""

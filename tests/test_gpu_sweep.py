@@ -94,7 +94,7 @@ def test_star_r2_paths_ragged(name, setting):
 
 @pytest.mark.parametrize("kind,r,n", [(1, 4, (64, 48, 40)), (1, 1, (33, 20, 17)),
                                       (1, 3, (40, 24, 30)), (2, 1, (50, 33, 27)),
-                                      (3, 4, (40, 24, 20))])
+                                      (3, 4, (40, 24, 20)), (4, 2, (36, 28, 20))])
 def test_random_space_settings(kind, r, n):
     """Property-style: random valid settings drawn from the canonical space."""
     L = H.layout(n, r)
@@ -121,7 +121,7 @@ def test_random_space_settings(kind, r, n):
     assert ran >= len(picks) // 2
 
 
-@pytest.mark.parametrize("kind,r", [(1, 2), (1, 4), (2, 1), (3, 4)])
+@pytest.mark.parametrize("kind,r", [(1, 2), (1, 4), (2, 1), (3, 4), (4, 2)])
 def test_config_coefficients_default_setting(kind, r):
     L = H.layout((64, 64, 64) if kind != 3 else (64, 32, 32), r)
     c = H.coeffs(kind, r)

@@ -284,3 +284,88 @@ def test_invalid_arguments_rejected():
         ost.sweep(ost.STAR, 2, ost.star_laplacian_coeffs(2), L, [u], [u.copy()])  # halo < order
     with pytest.raises(ValueError):
         ost.sweep(ost.BOX, 2, np.zeros(125), L, [u], [u.copy()])                   # box r != 1
+
+
+# ------------------------------------------------------------------ rhs4center-like (NEXT-1)
+def test_rhs4_flop_count_matches_table3():
+    assert ost.rhs4_flops() == 666          # Table III "rhs4center": 666 FLOPs
+
+
+def _rhs4_run(fields, n=5, scales=(1.0, 1.0, 1.0)):
+    X, Y, Z = sp.symbols("x y z")
+    ins = []
+    for f in fields:
+        fn = sp.lambdify((X, Y, Z), f, "numpy")
+        L, b = grid_from(lambda x, y, z: fn(x, y, z) + 0 * x, n, 2)
+        ins.append(b)
+    return L, run(ost.RHS4, 2, ost.rhs4_coeffs(scales), L, ins)
+
+
+def _elastic(u, mu, la, X, Y, Z, scales=(1, 1, 1)):
+    """Continuum d_j(mu (d_j u_i + d_i u_j)) + d_i(la div u) with x_d scaled by s_d."""
+    xs = (X, Y, Z)
+    D = lambda f, d: scales[d] * sp.diff(f, xs[d])
+    div = sum(D(u[j], j) for j in range(3))
+    return [sum(D(mu * (D(u[i], j) + D(u[j], i)), j) for j in range(3)) + D(la * div, i)
+            for i in range(3)]
+
+
+def test_rhs4_constant_fields_zero():
+    L, outs = _rhs4_run([sp.Integer(3), sp.Integer(-2), sp.Integer(5), sp.Integer(2),
+                         sp.Integer(7)])
+    for o in outs:
+        assert np.all(interior(L, o) == 0.0)
+
+
+@pytest.mark.parametrize("seed,scales", [(1, (1, 1, 1)), (2, (1, 2, 0.5)), (3, (0.5, 1, 2))])
+def test_rhs4_constant_coefficients_polynomial_exact(seed, scales):
+    """Constant mu, lambda and displacements of total degree <= 4: the 4th-order operators
+    reproduce mu lap u + (mu + la) grad div u up to rounding (closed form via sympy)."""
+    rng = np.random.default_rng(seed)
+    X, Y, Z = sp.symbols("x y z")
+    mons = [X ** a * Y ** b * Z ** c for a in range(5) for b in range(5) for c in range(5)
+            if a + b + c <= 4]
+    u = [sum(int(rng.integers(-3, 4)) * m for m in rng.choice(mons, 8, replace=False))
+         for _ in range(3)]
+    mu, la = sp.Integer(3), sp.Integer(2)
+    L, outs = _rhs4_run(u + [mu, la], scales=scales)
+    want = _elastic(u, mu, la, X, Y, Z, scales)
+    t = np.arange(5, dtype=np.float64)
+    Zg, Yg, Xg = np.meshgrid(t, t, t, indexing="ij")
+    for o, w in zip(outs, want):
+        ref = sp.lambdify((X, Y, Z), w, "numpy")(Xg, Yg, Zg) + 0 * Xg
+        got = interior(L, o)
+        assert np.max(np.abs(got - ref)) <= 1e-12 * max(1.0, np.max(np.abs(ref)))
+
+
+def test_rhs4_degree_bound_is_tight():
+    """The mixed terms use 4th-order first derivatives: degree 5 in the inner direction
+    is no longer reproduced."""
+    X, Y, Z = sp.symbols("x y z")
+    u = [sp.Integer(0), X ** 5, sp.Integer(0)]            # u2 = x^5: d_y(mu d_x u2) ... and
+    mu, la = sp.Integer(1), sp.Integer(1)                  # d_x(la d_y u2) = 0; d_x(mu d_x u2)
+    L, outs = _rhs4_run(u + [mu, la])                      # is a 2nd derivative (exact to 5)
+    t = np.arange(5, dtype=np.float64)
+    Zg, Yg, Xg = np.meshgrid(t, t, t, indexing="ij")
+    want = _elastic(u, mu, la, X, Y, Z)
+    ref1 = sp.lambdify((X, Y, Z), want[1], "numpy")(Xg, Yg, Zg) + 0 * Xg
+    assert np.max(np.abs(interior(L, outs[1]) - ref1)) <= 1e-9 * np.max(np.abs(ref1))
+    u = [X * Y ** 5, sp.Integer(0), sp.Integer(0)]         # d_x(la d_x u1) ok, d_y(mu d_x u1)
+    L, outs = _rhs4_run(u + [mu, la])                      # needs D_y of y^5 -> inexact
+    want = _elastic(u, mu, la, X, Y, Z)
+    ref1 = sp.lambdify((X, Y, Z), want[1], "numpy")(Xg, Yg, Zg) + 0 * Xg
+    assert np.max(np.abs(interior(L, outs[1]) - ref1)) > 1e-6 * np.max(np.abs(ref1))
+
+
+def test_rhs4_variable_coefficient_second_derivative():
+    """Linear mu and quadratic u: d(mu du) is reproduced (the SW4 4th-order variable-
+    coefficient operator is exact there); lambda = 0 so only the V and mu-mixed terms act."""
+    X, Y, Z = sp.symbols("x y z")
+    mu = 5 + X + 2 * Y - Z
+    u = [X * X + Y * Z, Y * Y - X * Z, Z * Z + X * Y]
+    L, outs = _rhs4_run(u + [mu, sp.Integer(0)], n=6)
+    t = np.arange(6, dtype=np.float64)
+    Zg, Yg, Xg = np.meshgrid(t, t, t, indexing="ij")
+    for o, w in zip(outs, _elastic(u, mu, sp.Integer(0), X, Y, Z)):
+        ref = sp.lambdify((X, Y, Z), w, "numpy")(Xg, Yg, Zg) + 0 * Xg
+        assert np.max(np.abs(interior(L, o) - ref)) <= 1e-12 * max(1.0, np.max(np.abs(ref)))

@@ -31,6 +31,8 @@ def config(name):
         return C.CST_BOX, 1, [x * y * z for x in b for y in b for z in b], (512, 512, 512), 3
     if name == "hypterm":
         return C.CST_HYPTERM, 4, [4 / 5, -1 / 5, 4 / 105, -1 / 280, 1.0, 1.0, 1.0], (512, 512, 512), 4
+    if name == "rhs4":
+        return C.CST_RHS4, 2, [1.0, 1.0, 1.0], (320, 320, 320), 6
     raise ValueError(name)
 
 
@@ -73,7 +75,7 @@ def main():
            "default_setting": dflt.as_dict(), "default_ms": ms_def,
            "report": {f: getattr(rep, f) for f, _ in rep._fields_}, "wall_s": wall,
            "log": os.path.relpath(log, ROOT), "seed": args.seed, "budget_s": args.budget}
-    out = args.out or os.path.join(ROOT, "tuned", f"{args.config}_512.json")
+    out = args.out or os.path.join(ROOT, "tuned", f"{args.config}_{n[0]}.json")
     with open(out, "w") as f:
         json.dump(res, f, indent=1)
     print(json.dumps(res))
