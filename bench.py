@@ -76,6 +76,7 @@ class ClockSampler:
         self.thread = None
         self.proc = None
         self.rows = []
+        self.poll_s = float(os.environ.get("CST_BENCH_CLOCK_POLL_MS", "20")) / 1e3
 
     def start(self):
         try:
@@ -94,7 +95,7 @@ class ClockSampler:
                                 self.reasons.add(n)
                     except Exception:
                         pass
-                    time.sleep(0.002)
+                    time.sleep(self.poll_s)
             self.thread = threading.Thread(target=poll, daemon=True)
             self.thread.start()
             self.source = "nvml"
@@ -425,7 +426,10 @@ def main():
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
                 "other_configs": others,
                 "gpu_launches": launches,
-                "per_step_ms": {"min": min(per), "median": statistics.median(per), "max": max(per)}}
+                "per_step_ms": {"min": min(per), "median": statistics.median(per), "max": max(per),
+                                "p90": sorted(per)[int(0.9 * (len(per) - 1))],
+                                "slow_steps_gt_1.1x_median":
+                                    sum(1 for x in per if x > 1.1 * statistics.median(per))}}
         print(json.dumps(line), flush=True)
     if dist_h is not None:
         C.cst_dist_destroy(dist_h)

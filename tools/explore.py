@@ -29,7 +29,7 @@ def main():
     ap.add_argument("--reps", type=int, default=10)
     args = ap.parse_args()
     kind, r = args.kind, args.order
-    nc = {1: 6 * r + 1, 2: 27, 3: 7}[kind]
+    nc = {1: 6 * r + 1, 2: 27, 3: 7, 4: 3}[kind]
     coeffs = [0.1] * nc
     g = C.make_grid(*args.n, r)
     h = C.cst_stencil_create(kind, r, coeffs, g)
