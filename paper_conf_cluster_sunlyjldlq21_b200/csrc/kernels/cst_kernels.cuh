@@ -186,9 +186,12 @@ __device__ __forceinline__ void hypterm_point(const Ctx& C, const Acc& U, double
 }
 
 // rhs4center-like (NEXT-1; Table III "rhs4center"): inputs u1, u2, u3, mu, lambda,
-// outputs r1..r3, coefficients [s_x, s_y, s_z]; same terms and order as the oracle:
+// outputs r1..r3, coefficients [s_x, s_y, s_z]; the oracle's terms in the oracle's order,
 //   r_i = sum_d s_d^2 V_d[mu + delta_id (mu + la)](u_i)
-//       + sum_{d != i} s_d s_i (D_d[mu D_i u_d] + D_i[la D_d u_d])
+//       + sum_{d != i} s_d s_i (D_d[mu D_i u_d] + D_i[la D_d u_d]),
+// with the constant factors folded (host-precomputed in the coefficient bank):
+// kcoef[3 + d] = s_d^2 / 6 scales the unscaled V sum, kcoef[6 + pair(d, i)] = s_d s_i / 144
+// scales the unscaled outer(inner) difference of each mixed term.
 template <class Acc>
 __device__ __forceinline__ void rhs4_point(const Ctx& C, const Acc& U, double* r) {
   auto at = [&](int arr, int d, int k, int d2, int k2) {
@@ -204,7 +207,7 @@ __device__ __forceinline__ void rhs4_point(const Ctx& C, const Acc& U, double* r
     for (int d = 0; d < 3; ++d) {
       auto a = [&](int k) {
         const double m = at(3, d, k, d, 0);
-        return d == i ? m + (m + at(4, d, k, d, 0)) : m;
+        return d == i ? fma(2.0, m, at(4, d, k, d, 0)) : m;
       };
       auto f = [&](int k) { return at(i, d, k, d, 0); };
       const double am2 = a(-2), am1 = a(-1), a0 = a(0), ap1 = a(1), ap2 = a(2);
@@ -217,25 +220,22 @@ __device__ __forceinline__ void rhs4_point(const Ctx& C, const Acc& U, double* r
       v = fma(m2, f(-1) - f0, v);
       v = fma(m3, f(1) - f0, v);
       v = fma(m4, f(2) - f0, v);
-      const double sd = C.coef(d);
-      const double term = (sd * sd) * (v * (1.0 / 6.0));
-      acc = d == 0 ? term : acc + term;
+      acc = d == 0 ? C.coef(3 + d) * v : fma(C.coef(3 + d), v, acc);
     }
 #pragma unroll
     for (int d = 0; d < 3; ++d) {
       if (d == i) continue;
       auto mixed = [&](int outer, int inner, int coef, int comp) {
         auto inner_d = [&](int ko) {
-          const double g = ((at(comp, outer, ko, inner, -2) - at(comp, outer, ko, inner, 2)) +
-                            8.0 * (at(comp, outer, ko, inner, 1) - at(comp, outer, ko, inner, -1))) *
-                           (1.0 / 12.0);
+          const double g = fma(8.0, at(comp, outer, ko, inner, 1) - at(comp, outer, ko, inner, -1),
+                               at(comp, outer, ko, inner, -2) - at(comp, outer, ko, inner, 2));
           return at(coef, outer, ko, outer, 0) * g;
         };
-        return ((inner_d(-2) - inner_d(2)) + 8.0 * (inner_d(1) - inner_d(-1))) * (1.0 / 12.0);
+        return fma(8.0, inner_d(1) - inner_d(-1), inner_d(-2) - inner_d(2));
       };
-      const double sdi = C.coef(d) * C.coef(i);
-      acc = fma(sdi, mixed(d, i, 3, d), acc);
-      acc = fma(sdi, mixed(i, d, 4, d), acc);
+      const double w = C.coef(6 + (d + i - 1));  // pair (0,1) -> 6, (0,2) -> 7, (1,2) -> 8
+      acc = fma(w, mixed(d, i, 3, d), acc);
+      acc = fma(w, mixed(i, d, 4, d), acc);
     }
     r[i] = acc;
   }

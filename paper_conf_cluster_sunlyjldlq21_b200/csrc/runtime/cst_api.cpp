@@ -181,6 +181,13 @@ extern "C" cst_status cst_stencil_create(const cst_stencil_desc* desc, const cst
   // kernel coefficient bank: the user's coefficients, plus for hypterm the streamed-
   // direction weights ws[k] = -sign(k) dxinv_s a_|k| (k = -4..-1, 1..4) for s = z, then y
   h->kcoef = h->coeffs;
+  if (kind == CST_RHS4) {
+    // s_d^2 / 6 for the V terms, s_d s_i / 144 for the mixed pairs (0,1), (0,2), (1,2)
+    for (int d = 0; d < 3; ++d) h->kcoef.push_back(h->coeffs[d] * h->coeffs[d] / 6.0);
+    h->kcoef.push_back(h->coeffs[0] * h->coeffs[1] / 144.0);
+    h->kcoef.push_back(h->coeffs[0] * h->coeffs[2] / 144.0);
+    h->kcoef.push_back(h->coeffs[1] * h->coeffs[2] / 144.0);
+  }
   if (kind == CST_HYPTERM)
     for (int sdir : {2, 1})
       for (int k = -4; k <= 4; ++k) {
