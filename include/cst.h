@@ -83,7 +83,8 @@ typedef struct {
 } cst_grid;
 
 /* Parameter setting: Table I with the B200 extensions of DESIGN.md §3.
- * Encoding (Q14): bool/enum start at 1 with unit stride; numerics are powers of 2. */
+ * Encoding (Q14): bool/enum start at 1 with unit stride; numerics are powers of 2.
+ * A zero-initialised struct is NOT valid: start from cst_setting_default or cst_space_at. */
 typedef struct {
   int32_t tb[3];          /* TB_x, TB_y, TB_z: CTA shape */
   int32_t staging;        /* 1 none (L1/L2), 2 smem ld/st, 3 smem via TMA */
@@ -96,6 +97,11 @@ typedef struct {
   int32_t bm[3];          /* block merging (adjacent points) */
   int32_t use_retiming;   /* 1 gather form, 2 retimed scatter accumulation */
   int32_t prefetch;       /* 1 off, 2..4 pipeline stages in flight */
+  int32_t bt;             /* temporal blocking degree {1,2,4}: sweeps fused per kernel
+                           * pass (B200 extension, "more
+                           * optimization parameters").  Rule R14: bt > 1 needs star/box,
+                           * z streaming with T_z = 1, TMA staging, retiming, CM = UF = 1,
+                           * BM_x, BM_y <= 2.  Only matters for nsteps > 1 (cst_sweep). */
 } cst_setting;
 
 typedef struct cst_stencil cst_stencil;     /* opaque: JIT modules, TMA descriptors, space */
@@ -112,8 +118,9 @@ cst_status cst_setting_check(const cst_stencil* h, const cst_setting* s);
 /* A good default setting for the handle's stencil (valid by construction). */
 cst_status cst_setting_default(const cst_stencil* h, cst_setting* s);
 
-/* Canonical valid space: lexicographic order of the 19 fields (Table I row order, values
- * ascending) restricted to valid tuples; rank = position (bit-exact with oracle/space.py). */
+/* Canonical valid space: lexicographic order of the 20 fields (Table I row order, then bt;
+ * values ascending) restricted to valid tuples; rank = position (bit-exact with
+ * oracle/space.py). */
 cst_status cst_space_count(cst_stencil* h, uint64_t* n);
 cst_status cst_space_at(cst_stencil* h, uint64_t rank, cst_setting* s);
 cst_status cst_space_rank(cst_stencil* h, const cst_setting* s, uint64_t* rank);
@@ -134,10 +141,14 @@ cst_status cst_kernel_info_get(cst_stencil* h, const cst_setting* s, cst_kernel_
 cst_status cst_variant_compile(const cst_stencil* h, const cst_setting* s, double* compile_s);
 
 /* One sweep (nsteps = 1) or nsteps ping-pong sweeps over DEVICE buffers, asynchronous on
- * `stream`.  in[n_inputs], out[n_outputs].  Only interior points are written; output
- * halos are never touched.  nsteps > 1 requires n_inputs == n_outputs (ping-pong: the
- * interior of in[] is overwritten; result in out if nsteps is odd, else in in).
- * Inputs must not overlap outputs (CST_E_INVALID).  Allocates nothing after first use. */
+ * `stream`.  in[n_inputs], out[n_outputs].  nsteps = 1: only interior points of out[] are
+ * written, output halos are never touched.  nsteps > 1 requires n_inputs == n_outputs
+ * (ping-pong: the interior of in[] is overwritten; result in out if nsteps is odd, else in
+ * in); in[]'s halo is the boundary condition of every step and is first copied into
+ * out[]'s halo (reading Q23).  With s->bt > 1 the steps run as kernel passes of
+ * up to bt fused sweeps (temporal blocking); the pass count keeps nsteps' parity, so the
+ * result placement is the same for every bt.  Inputs must not overlap outputs
+ * (CST_E_INVALID).  Allocates nothing after first use. */
 cst_status cst_sweep(cst_stencil* h, const cst_setting* s, const double* const* in,
                      double* const* out, int32_t nsteps, void* stream);
 /* Same computation over HOST buffers (end-to-end path): copies the inputs host->device,
@@ -159,11 +170,12 @@ cst_status cst_fill_uniform(const cst_grid* g, double* dev, uint64_t seed, uint6
                             int64_t nx_global, int64_t ny_global, int64_t z0,
                             double pad_value, void* stream);
 
-/* Time a setting: `warmup` untimed sweeps then the median of `reps` CUDA-event timed
- * sweeps on `stream` (fitness of P:351 / Q20).  *ms = median milliseconds per sweep. */
+/* Time a setting: `warmup` untimed cst_sweep calls of `nsteps` steps, then the median of
+ * `reps` CUDA-event timed calls on `stream` (fitness of P:351 / Q20).  *ms = median
+ * milliseconds PER STEP (call time / nsteps).  nsteps > 1 overwrites in[] (ping-pong). */
 cst_status cst_time_setting(cst_stencil* h, const cst_setting* s, const double* const* in,
-                            double* const* out, int32_t warmup, int32_t reps, void* stream,
-                            double* ms);
+                            double* const* out, int32_t nsteps, int32_t warmup, int32_t reps,
+                            void* stream, double* ms);
 
 /* Hardware counters of one sweep (CUPTI range profiler, user range + user replay: the
  * sweep is re-run once per counter pass).  names: metric names as ncu / CUPTI spell them
@@ -205,6 +217,10 @@ typedef struct {
   int32_t warm_start;        /* 1: add cst_setting_default() to the dataset (ours) */
   int32_t metrics_mode;      /* 0: CUPTI counters for the dataset if available, else
                                 modelled features; 1: modelled features only        */
+  int32_t nsteps;            /* steps per cst_sweep call of the tuned workload (1); the
+                                fitness is ms per step.  With nsteps = 1 a setting is
+                                timed as its bt = 1 twin; with nsteps > 1 the built-in
+                                evaluator times ping-pong on its own device copies   */
 } cst_tune_opts;
 
 typedef struct {

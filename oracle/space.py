@@ -19,13 +19,19 @@ Space (readings Q14/Q15 of SURVEY.md §8(c)):
   15-17 BM_x,y,z     p2[1, M_d]
   18  use_retiming   {1,2}
   19  prefetch       {1 off, 2, 3, 4 stages}        usePrefetching {1,2} + depth
+  20  bt             {1, 2, 4}                      temporal blocking degree: sweeps fused
+                                                    per pass (B200 extension, SURVEY §8(f)
+                                                    NEXT-2; "more optimization parameters",
+                                                    P:127 / P:419)
 
 Rules: paper R1 prod TB <= 1024; R2 SD=SB=1 when streaming off; R3 UF_SD <= SB when
 streaming on.  Ours (Q15): R4 prod TB >= 32; R5 T_d = TB_d*BM_d*CM_d <= E_d (E_d = M_d,
 E_SD = SB when streaming); R6 UF_d <= trip_d (trip_d = BM_d*CM_d; trip_SD = SB / T_SD when
 streaming); R7 prod(BM*CM) <= 16; R8 streaming => SD != 1; R9 prefetch > 1 => streaming;
 R10 modelled smem <= SMEM_LIMIT; R11 modelled registers <= 255; R12 TMA box: T_x even and
-every box extent <= 256.
+every box extent <= 256; R14 bt > 1 only for the temporally blocked path: star / box,
+streaming along z with T_SD = 1, TMA staging, retimed accumulators, no cyclic merging,
+BM_x, BM_y <= 2, every UF = 1 (reading Q23).
 """
 from __future__ import annotations
 
@@ -33,7 +39,7 @@ import math
 
 FIELDS = ("tb_x", "tb_y", "tb_z", "staging", "use_constant", "use_streaming", "sd", "sb",
           "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z", "bm_x", "bm_y", "bm_z",
-          "use_retiming", "prefetch")
+          "use_retiming", "prefetch", "bt")
 
 STAR, BOX, HYPTERM, RHS4 = 1, 2, 3, 4
 SMEM_LIMIT = 227 * 1024 - 1024      # data bytes; 1 KiB kept for mbarriers / alignment
@@ -67,6 +73,25 @@ def tiles(s: dict):
             s["tb_z"] * s["bm_z"] * s["cm_z"]]
 
 
+def xr(r: int) -> int:
+    """x half-width of a staged halo: r rounded up to even (16-B aligned TMA box rows)."""
+    return r + (r & 1)
+
+
+def tb_extent(r: int, s: dict, level: int):
+    """(x, y) extents of level `level` of a temporally blocked CTA (level 0 = the TMA input
+    box, level bt = the output tile): T + 2 (bt - level) * halo per side."""
+    T = tiles(s)
+    k = s["bt"] - level
+    return T[0] + 2 * xr(r) * k, T[1] + 2 * r * k
+
+
+def tb_blocks_per_thread(r: int, s: dict, level: int) -> int:
+    ex, ey = tb_extent(r, s, level)
+    nthr = s["tb_x"] * s["tb_y"] * s["tb_z"]
+    return -(-((ex // s["bm_x"]) * (ey // s["bm_y"])) // nthr)
+
+
 def plane_geometry(kind: int, r: int, s: dict):
     """(in-plane elements P, ring planes NP) of the smem staging for a streaming setting;
     (box elements, 1) for a non-streaming one."""
@@ -87,12 +112,24 @@ def plane_geometry(kind: int, r: int, s: dict):
 def smem_bytes(kind: int, r: int, s: dict) -> int:
     if s["staging"] == 1:
         return 0
+    if s["bt"] > 1:
+        # prefetch ring of input planes + two slots per intermediate level
+        rnd = lambda e: -(-(e * 8) // 128) * 128
+        e0 = tb_extent(r, s, 0)
+        e1 = tb_extent(r, s, 1)
+        return s["prefetch"] * rnd(e0[0] * e0[1]) + (s["bt"] - 1) * 2 * rnd(e1[0] * e1[1])
     P, NP = plane_geometry(kind, r, s)
     plane = -(-(P * 8) // 128) * 128
     return n_arrays(kind) * NP * plane
 
 
 def est_regs(kind: int, r: int, s: dict) -> int:
+    if s["bt"] > 1:
+        # 2r+1 rotating accumulators per point of every level + one operand window
+        pts = sum(tb_blocks_per_thread(r, s, lv) for lv in range(1, s["bt"] + 1))
+        pts *= s["bm_x"] * s["bm_y"]
+        win = (s["bm_y"] + 2 * r) * (s["bm_x"] + 2 * xr(r))
+        return 32 + 2 * ((2 * r + 1) * pts + win)
     ppt = 1
     for d in "xyz":
         ppt *= s["bm_" + d] * s["cm_" + d]
@@ -110,6 +147,8 @@ def tma_ok(r: int, s: dict) -> bool:
     T = tiles(s)
     if T[0] % 2:
         return False
+    if s["bt"] > 1:
+        return all(e <= 256 for e in tb_extent(r, s, 0))
     if s["use_streaming"] == 1:
         ext = [t + 2 * r for t in T]
     else:
@@ -149,6 +188,8 @@ def check(kind: int, r: int, M, s: dict):
         return "R7"
     if s["prefetch"] > 1 and not stream:
         return "R9"
+    if s["bt"] > 1 and not tb_path_ok(kind, s):
+        return "R14"
     if smem_bytes(kind, r, s) > SMEM_LIMIT:
         return "R10"
     if est_regs(kind, r, s) > REG_LIMIT:
@@ -156,6 +197,16 @@ def check(kind: int, r: int, M, s: dict):
     if s["staging"] == 3 and not tma_ok(r, s):
         return "R12"
     return None
+
+
+def tb_path_ok(kind: int, s: dict) -> bool:
+    """R14: the temporally blocked kernel's structural requirements."""
+    return (kind in (STAR, BOX) and s["use_streaming"] == 2 and s["sd"] == 3
+            and s["staging"] == 3 and s["use_retiming"] == 2
+            and s["tb_z"] == 1 and s["bm_z"] == 1
+            and s["cm_x"] == 1 and s["cm_y"] == 1 and s["cm_z"] == 1
+            and s["bm_x"] <= 2 and s["bm_y"] <= 2
+            and s["uf_x"] == 1 and s["uf_y"] == 1 and s["uf_z"] == 1)
 
 
 def enumerate_space(kind: int, r: int, M):
@@ -215,12 +266,14 @@ def _inner(kind, r, M, s):
                                     for ufz in p2(1, bnd[2]):
                                         for ret in (1, 2):
                                             for pf in (1, 2, 3, 4):
-                                                t = dict(s, uf_x=ufx, uf_y=ufy, uf_z=ufz,
-                                                         cm_x=cmx, cm_y=cmy, cm_z=cmz,
-                                                         bm_x=bmx, bm_y=bmy, bm_z=bmz,
-                                                         use_retiming=ret, prefetch=pf)
-                                                if check(kind, r, M, t) is None:
-                                                    found.append(t)
+                                                for bt in (1, 2, 4):
+                                                    t = dict(s, uf_x=ufx, uf_y=ufy, uf_z=ufz,
+                                                             cm_x=cmx, cm_y=cmy, cm_z=cmz,
+                                                             bm_x=bmx, bm_y=bmy, bm_z=bmz,
+                                                             use_retiming=ret, prefetch=pf,
+                                                             bt=bt)
+                                                    if check(kind, r, M, t) is None:
+                                                        found.append(t)
     found.sort(key=as_tuple)
     yield from found
 

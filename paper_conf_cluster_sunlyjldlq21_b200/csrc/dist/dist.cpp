@@ -151,6 +151,14 @@ extern "C" cst_status cst_dist_sweep(cst_dist* D, const cst_setting* s, const do
     cin[a] = in[a];
     cout[a] = out[a];
   }
+  if (s->bt > 1)
+    return fail(CST_E_UNSUPPORTED, "temporal blocking (bt > 1) needs bt*order halo planes; "
+                                   "cst_dist_sweep exchanges order planes per step");
+  if (nsteps > 1)  // boundary condition of every step = in[]'s halo (as cst_sweep)
+    for (int a = 0; a < nio; ++a) {
+      st = copy_halo(G, in[a], out[a], sc);
+      if (st != CST_OK) return st;
+    }
   h->last_launches = 0;  // cst_launch_range counts every launch
   for (int step = 0; step < nsteps; ++step) {
     // 1. boundary planes first
@@ -231,6 +239,9 @@ extern "C" cst_status cst_dist_sweep_loopback(cst_stencil* h, int32_t nslabs, co
     cin[i] = in_slabs[i];
     cout[i] = out_slabs[i];
   }
+  if (s->bt > 1) st = fail(CST_E_UNSUPPORTED, "temporal blocking (bt > 1) is not supported by z-slab sweeps");
+  if (nsteps > 1)  // boundary condition of every step = in[]'s halo (as cst_sweep)
+    for (int i = 0; i < nslabs * nio && st == CST_OK; ++i) st = copy_halo(G, in_slabs[i], out_slabs[i], sc);
   h->last_launches = 0;  // cst_launch_range counts every launch
   for (int step = 0; step < nsteps && st == CST_OK; ++step) {
     for (int k = 0; k < nslabs && st == CST_OK; ++k) {

@@ -1360,11 +1360,264 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
 }
 
 // =============================================================================
+// temporal blocking, bt > 1 (B200 extension):
+// BT sweeps of a star / box stencil fused into one pass over HBM.
+//   level 0   input planes, TMA ring, extent (TA + 2 BT XR) x (TB + 2 BT R)
+//   level s   sweep s over the tile grown by BT - s halos, two smem slots per level
+//   level BT  the output tile, stored to HBM
+// Every level runs the retimed scatter: 2R+1 rotating accumulators per point, one
+// plane in, one completed plane out.  The pipeline is skewed — level s consumes the plane
+// level s-1 emitted in the previous iteration — so one __syncthreads per plane orders all
+// levels.  Points outside the interior keep their input value: the input halo is the
+// boundary condition of every fused step (cst_sweep copies it into the output halo, so
+// unfused ping-pong steps see the same values).  Intermediate planes never reach HBM.
+// =============================================================================
+constexpr int BT = CST_BT;
+__host__ __device__ constexpr int tb_wa(int s) { return TA + 2 * XR * (BT - s); }
+__host__ __device__ constexpr int tb_wb(int s) { return TB + 2 * R * (BT - s); }
+__host__ __device__ constexpr int tb_nba(int s) { return tb_wa(s) / BMA; }
+__host__ __device__ constexpr int tb_nblk(int s) { return tb_nba(s) * (tb_wb(s) / BMB); }
+__host__ __device__ constexpr int tb_kb(int s) { return (tb_nblk(s) + NTHR - 1) / NTHR; }
+constexpr int TB_NPB = BMA * BMB;  // points per register block
+constexpr int TB_SLOT0 = round_slot(tb_wa(0) * tb_wb(0));
+constexpr int TB_SLOTI = round_slot(tb_wa(1) * tb_wb(1));
+
+template <int S>
+struct TbAcc {
+  double v[tb_kb(S) * TB_NPB][W];
+  TbAcc<S + 1> next;
+};
+template <>
+struct TbAcc<BT + 1> {};
+
+template <int S, int L>
+__device__ __forceinline__ auto& tb_acc(TbAcc<L>& a) {
+  if constexpr (S == L) return a.v;
+  else return tb_acc<S>(a.next);
+}
+
+// One level-S step of the skewed pipeline: plane q of level S-1 (src, row width
+// tb_wa(S-1)) is scattered into the level-S accumulators; level-S plane q - R is then
+// complete and goes to dst (level-S slot) or, for S == BT, to HBM.
+template <int S, int U>
+__device__ __forceinline__ void tb_stage(const Ctx& C, const cst_kparams& P, const SGeo& g,
+                                         const double* __restrict__ src,
+                                         double* __restrict__ dst,
+                                         double (&acc)[tb_kb(S) * TB_NPB][W], int q) {
+  constexpr int WA = tb_wa(S), SWA = tb_wa(S - 1);
+  constexpr int NBA = tb_nba(S), NBLK = tb_nblk(S), KB = tb_kb(S);
+  constexpr int HX = XR * (BT - S), HY = R * (BT - S);
+  constexpr int WX = BMA + 2 * XR;   // x-window of a block row (src cols ex0 .. ex0 + WX)
+  constexpr int ES = (U - R + W) % W;  // slot of the completed plane q - R
+  // contribution d of plane q belongs to plane q - (d - R); only interior planes compute
+  bool zin[W];
+#pragma unroll
+  for (int d = 0; d < W; ++d) {
+    const int m = q - (d - R);
+    zin[d] = m >= 0 && m < P.nz;
+  }
+  const int o = q - R;
+#pragma unroll
+  for (int kb = 0; kb < KB; ++kb) {
+    const int blk = (int)threadIdx.x + kb * NTHR;
+    if (KB * NTHR > NBLK && blk >= NBLK) continue;
+    const int ex0 = (blk % NBA) * BMA, ey0 = (blk / NBA) * BMB;
+    // level-S point (ex, ey) reads src at (ex + XR + dx, ey + R + dy)
+    const double* base = src + ey0 * SWA + ex0;
+    // contribution chains start from the accumulator they land in (no extra add);
+    // points outside the interior restart from it below and keep their input value
+    double c[BMB][BMA][W], ctr[BMB][BMA];
+    auto accum = [&](int ib, int ia, int d) -> double& {
+      return acc[kb * TB_NPB + ib * BMA + ia][(U - (d - R) + 2 * W) % W];
+    };
+    auto load_row = [&](int row, double* w) {
+      if constexpr (BMA % 2 == 0) {
+#pragma unroll
+        for (int t = 0; t < WX / 2; ++t) {
+          const double2 v = *reinterpret_cast<const double2*>(base + row * SWA + 2 * t);
+          w[2 * t] = v.x;
+          w[2 * t + 1] = v.y;
+        }
+      } else {
+#pragma unroll
+        for (int t = 0; t < WX; ++t) w[t] = base[row * SWA + t];
+      }
+    };
+    if constexpr (KIND == 1) {
+#pragma unroll
+      for (int ib = 0; ib < BMB; ++ib) {
+        double w[WX];
+        load_row(R + ib, w);
+#pragma unroll
+        for (int ia = 0; ia < BMA; ++ia) {
+          const double u0 = w[XR + ia];
+          ctr[ib][ia] = u0;
+          double ip = fma(C.coef(0), u0, accum(ib, ia, R));
+#pragma unroll
+          for (int k = -R; k <= R; ++k)
+            if (k != 0) ip = fma(C.coef(star_ci(0, k)), w[XR + ia + k], ip);
+          c[ib][ia][R] = ip;
+#pragma unroll
+          for (int d = 0; d < W; ++d)
+            if (d != R) c[ib][ia][d] = fma(C.coef(star_ci(2, d - R)), u0, accum(ib, ia, d));
+        }
+      }
+#pragma unroll
+      for (int wr = -R; wr < BMB + R; ++wr) {  // y-neighbour rows of the block
+        double v[BMA];
+        if (wr >= 0 && wr < BMB) {
+#pragma unroll
+          for (int ia = 0; ia < BMA; ++ia) v[ia] = ctr[wr][ia];
+        } else if constexpr (BMA % 2 == 0) {
+#pragma unroll
+          for (int ia = 0; ia < BMA; ia += 2) {
+            const double2 t = *reinterpret_cast<const double2*>(base + (R + wr) * SWA + XR + ia);
+            v[ia] = t.x;
+            v[ia + 1] = t.y;
+          }
+        } else {
+#pragma unroll
+          for (int ia = 0; ia < BMA; ++ia) v[ia] = base[(R + wr) * SWA + XR + ia];
+        }
+#pragma unroll
+        for (int ib = 0; ib < BMB; ++ib) {
+          const int k = wr - ib;
+          if (k == 0 || k < -R || k > R) continue;
+#pragma unroll
+          for (int ia = 0; ia < BMA; ++ia)
+            c[ib][ia][R] = fma(C.coef(star_ci(1, k)), v[ia], c[ib][ia][R]);
+        }
+      }
+    } else {  // box: slices dz of plane q, (dy, dx) ascending within each slice
+#pragma unroll
+      for (int ib = 0; ib < BMB; ++ib)
+#pragma unroll
+        for (int ia = 0; ia < BMA; ++ia)
+#pragma unroll
+          for (int d = 0; d < W; ++d) c[ib][ia][d] = accum(ib, ia, d);
+#pragma unroll
+      for (int wr = 0; wr < BMB + 2 * R; ++wr) {
+        double w[WX];
+        load_row(wr, w);
+#pragma unroll
+        for (int ib = 0; ib < BMB; ++ib) {
+          const int dy = wr - R - ib;
+          if (dy == 0) {
+#pragma unroll
+            for (int ia = 0; ia < BMA; ++ia) ctr[ib][ia] = w[XR + ia];
+          }
+          if (dy < -R || dy > R) continue;
+#pragma unroll
+          for (int ia = 0; ia < BMA; ++ia)
+#pragma unroll
+            for (int dx = -R; dx <= R; ++dx)
+#pragma unroll
+              for (int d = 0; d < W; ++d)
+                c[ib][ia][d] = fma(C.coef(box_ci(d - R, dy, dx)), w[XR + ia + dx], c[ib][ia][d]);
+        }
+      }
+    }
+    // scatter into the rotating accumulators, emit plane q - R, clear its slot
+#pragma unroll
+    for (int ib = 0; ib < BMB; ++ib)
+#pragma unroll
+      for (int ia = 0; ia < BMA; ++ia) {
+        double(&A)[W] = acc[kb * TB_NPB + ib * BMA + ia];
+        const int gx = g.a0 - HX + ex0 + ia, gy = g.b0 - HY + ey0 + ib;
+        const bool inxy = gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny;
+#pragma unroll
+        for (int d = 0; d < W; ++d) {
+          const int sl = (U - (d - R) + 2 * W) % W;
+          if (inxy && zin[d]) A[sl] = c[ib][ia][d];
+          else if (d == R) A[sl] += ctr[ib][ia];  // outside: keep the input value
+        }
+        const double val = A[ES];
+        A[ES] = 0.0;
+        if constexpr (S < BT) {
+          dst[(ey0 + ib) * WA + ex0 + ia] = val;
+        } else {
+          if (o >= g.s_start && o < g.s_end && gx < P.nx && gy < P.ny)
+            P.out[0][gx + (long long)gy * P.py + (long long)o * P.pz] = val;
+        }
+      }
+  }
+}
+
+template <int S, int L>
+__device__ __forceinline__ void tb_zero(TbAcc<L>& a) {
+  if constexpr (S <= BT) {
+    auto& v = tb_acc<S>(a);
+#pragma unroll
+    for (int k = 0; k < tb_kb(S) * TB_NPB; ++k)
+#pragma unroll
+      for (int m = 0; m < W; ++m) v[k][m] = 0.0;
+    tb_zero<S + 1>(a);
+  }
+}
+
+template <int DUMMY>
+__device__ __forceinline__ void kernel_tblock(const cst_kparams& P, double* smem) {
+  Ctx C{P};
+  constexpr int D = PF, NP = PF;
+  constexpr unsigned BYTES0 = (unsigned)(tb_wa(0) * tb_wb(0) * 8);
+  const SGeo g = stream_geo(P);
+  const int tid = threadIdx.x;
+  const int n_load = (g.s_end - g.s_start) + 2 * BT * R;  // input planes of this chunk
+  const int n_it = n_load + BT - 1;                       // + pipeline skew
+  const int p0 = g.s_start - BT * R;
+  double* lvl = smem + NP * TB_SLOT0;  // level s slot t at lvl + ((s-1)*2 + t) * TB_SLOTI
+  u64* bars = (u64*)(lvl + (BT - 1) * 2 * TB_SLOTI);
+  TbAcc<1> acc;
+  tb_zero<1>(acc);
+  if (tid == 0) {
+    for (int s = 0; s < NP; ++s) mbar_init(&bars[s], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  auto issue = [&](int j) {  // input plane p0 + j -> ring slot j % NP
+    const int sl = j % NP;
+    mbar_arrive_expect_tx(&bars[sl], BYTES0);
+    tma_load_3d(smem + sl * TB_SLOT0, &P.tma[0], &bars[sl], P.tox + g.a0 - XR * BT,
+                P.toy + g.b0 - R * BT, P.toz + p0 + j);
+  };
+  if (tid == 0)
+    for (int j = 0; j < D && j < n_load; ++j) issue(j);
+
+  for (int i0 = 0; i0 < n_it; i0 += W) {
+    static_for<0, W>([&](auto UU) {
+      constexpr int u = decltype(UU)::value;
+      const int i = i0 + u;
+      if (i >= n_it) return;  // CTA-uniform
+      const int p = p0 + i;
+      // levels BT..2 consume last iteration's planes while the TMA of plane p lands
+      static_for<2, BT + 1>([&](auto SS) {
+        constexpr int S = BT + 2 - decltype(SS)::value;
+        const double* src = lvl + ((S - 2) * 2 + ((i - 1) & 1)) * TB_SLOTI;
+        double* dst = S < BT ? lvl + ((S - 1) * 2 + (i & 1)) * TB_SLOTI : nullptr;
+        tb_stage<S, u>(C, P, g, src, dst, tb_acc<S>(acc), p - (S - 1) * (R + 1));
+      });
+      if (i < n_load) {
+        mbar_wait(&bars[i % NP], (u32)((i / NP) & 1));
+        tb_stage<1, u>(C, P, g, smem + (i % NP) * TB_SLOT0, lvl + (i & 1) * TB_SLOTI,
+                       tb_acc<1>(acc), p);
+      }
+      __syncthreads();
+      if (tid == 0 && i + D < n_load) {
+        fence_proxy_async();
+        issue(i + D);
+      }
+    });
+  }
+}
+
+// =============================================================================
 // entry point
 // =============================================================================
 extern "C" __global__ void __launch_bounds__(NTHR) cst_kernel(const __grid_constant__ cst_kparams P) {
   extern __shared__ __align__(128) double cst_smem[];
-  if constexpr (!STREAM) {
+  if constexpr (BT > 1) {
+    kernel_tblock<0>(P, cst_smem);
+  } else if constexpr (!STREAM) {
     kernel_tile3d(P, cst_smem);
   } else if constexpr ((KIND == 1 || KIND == 2) && TS == 1) {
     kernel_stream1(P, cst_smem);

@@ -94,7 +94,11 @@ static Geometry geometry(const StencilInfo& st, const Tuple& t, int64_t nx, int6
     g.grid_x = (unsigned)(g.tiles_a * (int64_t)g.tiles_b);
     g.grid_y = (unsigned)g.chunks;
     g.box[0] = (int)T[0] + 2 * xr;
-    if (sz) {
+    if (t[F_BT] > 1) {  // temporally blocked: the input box carries bt halos per side
+      g.box[0] = (int)T[0] + 2 * xr * t[F_BT];
+      g.box[1] = (int)T[1] + 2 * r * t[F_BT];
+      g.box[2] = 1;
+    } else if (sz) {
       g.box[1] = (int)T[1] + 2 * r;
       g.box[2] = 1;
     } else {
@@ -254,6 +258,7 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
   c.bm[0] = hyp ? 1 : 2;
   c.bm[1] = hyp ? 1 : 2;
   c.use_retiming = 2;
+  c.bt = 1;
   c.prefetch = (h->info.kind == CST_BOX || h->info.kind == CST_RHS4) ? 2 : 3;
   for (int tries = 0; tries < 12 && check_rules(h->info, to_tuple(c)); ++tries) {
     // shrink the tile until it fits the grid (coverage) and the thread floor
@@ -485,6 +490,30 @@ cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* 
   return CST_OK;
 }
 
+namespace cst {
+std::vector<int> pass_schedule(int nsteps, int bt) {
+  std::vector<int> v;
+  if (bt < 1) bt = 1;
+  for (int rem = nsteps; rem > 0;) {
+    int b = bt;
+    while (b > rem) b /= 2;
+    v.push_back(b);
+    rem -= b;
+  }
+  if ((int)(v.size() & 1) != (nsteps & 1)) {
+    // one pass more: split the last pass of >= 2 steps in halves (exists: an all-ones
+    // schedule has nsteps passes)
+    for (int k = (int)v.size() - 1; k >= 0; --k)
+      if (v[k] >= 2) {
+        v[k] /= 2;
+        v.insert(v.begin() + k + 1, v[k]);
+        break;
+      }
+  }
+  return v;
+}
+}  // namespace cst
+
 static bool overlaps(const double* a, const double* b, int64_t n) {
   return a < b + n && b < a + n;
 }
@@ -515,13 +544,26 @@ extern "C" cst_status cst_sweep(cst_stencil* h, const cst_setting* s, const doub
     for (int q = 0; q < o; ++q)
       if (overlaps(out[q], out[o], n)) return fail(CST_E_INVALID, "outputs overlap");
   }
+  {
+    const char* rule = check_rules(h->info, to_tuple(*s));
+    if (rule) return fail(CST_E_CONSTRAINT, std::string("setting violates ") + rule);
+  }
   h->last_launches = 0;
   const double* cur_in[CST_MAX_IN];
   double* cur_out[CST_MAX_OUT];
   for (int a = 0; a < nin; ++a) cur_in[a] = in[a];
   for (int o = 0; o < nout; ++o) cur_out[o] = out[o];
-  for (int step = 0; step < nsteps; ++step) {
-    cst_status st = cst_launch_range(h, s, cur_in, cur_out, 0, h->grid.nz, (cudaStream_t)stream);
+  if (nsteps > 1) {
+    // boundary condition of every step = in[]'s halo (reading Q23)
+    cst_status st = copy_halo(h->grid, in[0], out[0], (cudaStream_t)stream);
+    if (st != CST_OK) return st;
+    ++h->last_launches;
+  }
+  // temporal blocking: passes of b <= bt fused steps (bt = 1: one launch per step)
+  for (int b : pass_schedule(nsteps, s->bt)) {
+    cst_setting sp = *s;
+    sp.bt = b;
+    cst_status st = cst_launch_range(h, &sp, cur_in, cur_out, 0, h->grid.nz, (cudaStream_t)stream);
     if (st != CST_OK) return st;
     if (nsteps > 1) {
       const double* tmp = cur_in[0];
@@ -586,6 +628,8 @@ extern "C" cst_status cst_sweep_host(cst_stencil* h, const cst_setting* s,
     return CST_OK;
   };
   if (nsteps == 1) {
+    cst_setting s1 = *s;  // one step: no temporal blocking
+    s1.bt = 1;
     // pipelined along z: H2D of chunk k+1 || sweep of chunk k || D2H of chunk k-1
     if (!h->host_in_stream) {
       CST_CUDA(cudaStreamCreateWithFlags(&h->host_in_stream, cudaStreamNonBlocking));
@@ -613,7 +657,7 @@ extern "C" cst_status cst_sweep_host(cst_stencil* h, const cst_setting* s,
                                  h->host_in_stream));
       copied = std::max(copied, need);
       CST_CUDA(cudaStreamWaitEvent(sm, event(h->host_in_stream), 0));
-      st = cst_launch_range(h, s, din, dout, z0, z1 - z0, sm);
+      st = cst_launch_range(h, &s1, din, dout, z0, z1 - z0, sm);
       if (st != CST_OK) break;
       CST_CUDA(cudaStreamWaitEvent(h->host_out_stream, event(sm), 0));
       for (int o = 0; o < nout && st == CST_OK; ++o)
@@ -629,8 +673,7 @@ extern "C" cst_status cst_sweep_host(cst_stencil* h, const cst_setting* s,
   }
   for (int a = 0; a < nin; ++a)
     CST_CUDA(cudaMemcpyAsync(h->dev_bufs[a], in[a], (size_t)n * 8, cudaMemcpyHostToDevice, sm));
-  for (int o = 0; o < nout; ++o)  // ping-pong reads the output buffer's halo (Dirichlet data)
-    CST_CUDA(cudaMemcpyAsync(dout[o], out[o], (size_t)n * 8, cudaMemcpyHostToDevice, sm));
+  // (no copy of out[]: cst_sweep gives the output buffer in[]'s halo, the boundary condition)
   st = cst_sweep(h, s, din, dout, nsteps, sm);
   if (st != CST_OK) return st;
   for (int o = 0; o < nout; ++o) {
@@ -648,22 +691,23 @@ extern "C" cst_status cst_sweep_host(cst_stencil* h, const cst_setting* s,
 
 extern "C" cst_status cst_time_setting(cst_stencil* h, const cst_setting* s,
                                        const double* const* in, double* const* out,
-                                       int32_t warmup, int32_t reps, void* stream, double* ms) {
-  if (!h || !s || !ms || reps < 1) return fail(CST_E_INVALID, "bad argument");
+                                       int32_t nsteps, int32_t warmup, int32_t reps,
+                                       void* stream, double* ms) {
+  if (!h || !s || !ms || reps < 1 || nsteps < 1) return fail(CST_E_INVALID, "bad argument");
   const Driver* d = nullptr;
   cst_status st = driver(&d);
   if (st != CST_OK) return st;
   CST_CUDA(cudaSetDevice(h->device));
   cudaStream_t sm = (cudaStream_t)stream;
   for (int i = 0; i < warmup; ++i) {
-    st = cst_sweep(h, s, in, out, 1, sm);
+    st = cst_sweep(h, s, in, out, nsteps, sm);
     if (st != CST_OK) return st;
   }
   std::vector<cudaEvent_t> ev(reps + 1);
   for (auto& e : ev) CST_CUDA(cudaEventCreate(&e));
   CST_CUDA(cudaEventRecord(ev[0], sm));
   for (int i = 0; i < reps; ++i) {
-    st = cst_sweep(h, s, in, out, 1, sm);
+    st = cst_sweep(h, s, in, out, nsteps, sm);
     if (st != CST_OK) break;
     CST_CUDA(cudaEventRecord(ev[i + 1], sm));
   }
@@ -682,6 +726,6 @@ extern "C" cst_status cst_time_setting(cst_stencil* h, const cst_setting* s,
   for (auto& e : ev) cudaEventDestroy(e);
   if (ke != cudaSuccess) return fail(CST_E_CUDA, std::string("kernel: ") + cudaGetErrorString(ke));
   std::sort(t.begin(), t.end());
-  *ms = reps % 2 ? t[reps / 2] : 0.5 * (t[reps / 2 - 1] + t[reps / 2]);
+  *ms = (reps % 2 ? t[reps / 2] : 0.5 * (t[reps / 2 - 1] + t[reps / 2])) / nsteps;
   return CST_OK;
 }

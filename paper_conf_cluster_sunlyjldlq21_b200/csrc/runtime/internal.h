@@ -29,10 +29,11 @@ cst_status fail(cst_status s, const std::string& msg);
   } while (0)
 
 // ------------------------------------------------------------------ settings
-// The 19 fields in canonical order (Table I row order).
+// The 20 fields in canonical order: Table I row order, then the temporal
+// blocking degree (B200 extension, NEXT-2).
 enum Field {
   F_TBX, F_TBY, F_TBZ, F_STAGING, F_CONST, F_STREAM, F_SD, F_SB, F_UFX, F_UFY, F_UFZ,
-  F_CMX, F_CMY, F_CMZ, F_BMX, F_BMY, F_BMZ, F_RET, F_PF, F_COUNT
+  F_CMX, F_CMY, F_CMZ, F_BMX, F_BMY, F_BMZ, F_RET, F_PF, F_BT, F_COUNT
 };
 using Tuple = std::array<int32_t, F_COUNT>;
 Tuple to_tuple(const cst_setting& s);
@@ -45,7 +46,7 @@ struct StencilInfo {
   int64_t M[3];  // nx, ny, nz
 };
 
-// Rule check (R1..R12).  Returns nullptr if valid else the rule id.
+// Rule check (R1..R12, R14).  Returns nullptr if valid else the rule id.
 const char* check_rules(const StencilInfo& st, const Tuple& t);
 int64_t model_smem_bytes(int kind, int r, const Tuple& t);
 int64_t model_regs(int kind, int r, const Tuple& t);
@@ -61,8 +62,8 @@ class Space {
   bool rank(const Tuple& t, uint64_t* out) const;
 
  private:
-  struct Core {  // (CM x3, BM x3, ret, pf) and its per-dim UF bounds (counts)
-    int32_t cm[3], bm[3], ret, pf;
+  struct Core {  // (CM x3, BM x3, ret, pf, bt) and its per-dim UF bounds (counts)
+    int32_t cm[3], bm[3], ret, pf, bt;
     int32_t nuf[3];
   };
   struct Prefix {
@@ -76,6 +77,14 @@ class Space {
   uint64_t total_ = 0;
   std::vector<int32_t> p2_[3];  // powers of two <= M_d
 };
+
+// Copy the logical halo of one array (fill.cu).  Multi-step sweeps use in[]'s halo as the
+// boundary condition of every step.
+cst_status copy_halo(const cst_grid& g, const double* src, double* dst, cudaStream_t stream);
+
+// Temporal-blocking pass schedule: step counts per kernel pass (powers of two <= bt)
+// summing to nsteps, with as many passes as nsteps has parity (ping-pong placement).
+std::vector<int> pass_schedule(int nsteps, int bt);
 
 // ------------------------------------------------------------------ driver entry points
 struct Driver {

@@ -1,9 +1,10 @@
 // space.cpp — the parameter space of Table I with the rules of DESIGN.md §3:
 // explicit rules of P:149 (R1-R3), our semantics rules (R4-R9) and the
 // implicit resource rules (R10-R12: "settings ... restricted by the usage of
-// register and shared memory ... only non-spilled parameter settings are explored").
+// register and shared memory ... only non-spilled parameter settings are explored") and
+// R14, the structural requirements of the temporally blocked path (field 20, bt).
 //
-// Canonical order: lexicographic over the 19 fields in Table I row order, values
+// Canonical order: lexicographic over the 20 fields (Table I row order, then bt), values
 // ascending.  count / rank / unrank are exact (bit-exact with oracle/space.py).
 #include <algorithm>
 #include <cstring>
@@ -15,12 +16,12 @@ namespace cst {
 const char* const kFieldNames[F_COUNT] = {
     "tb_x", "tb_y", "tb_z", "staging", "use_constant", "use_streaming", "sd", "sb",
     "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z", "bm_x", "bm_y", "bm_z",
-    "use_retiming", "prefetch"};
+    "use_retiming", "prefetch", "bt"};
 
 Tuple to_tuple(const cst_setting& s) {
   return Tuple{s.tb[0], s.tb[1], s.tb[2], s.staging, s.use_constant, s.use_streaming,
                s.sd, s.sb, s.uf[0], s.uf[1], s.uf[2], s.cm[0], s.cm[1], s.cm[2],
-               s.bm[0], s.bm[1], s.bm[2], s.use_retiming, s.prefetch};
+               s.bm[0], s.bm[1], s.bm[2], s.use_retiming, s.prefetch, s.bt};
 }
 
 cst_setting from_tuple(const Tuple& t) {
@@ -33,7 +34,7 @@ cst_setting from_tuple(const Tuple& t) {
     s.cm[d] = t[F_CMX + d];
     s.bm[d] = t[F_BMX + d];
   }
-  s.use_retiming = t[F_RET]; s.prefetch = t[F_PF];
+  s.use_retiming = t[F_RET]; s.prefetch = t[F_PF]; s.bt = t[F_BT];
   return s;
 }
 
@@ -64,6 +65,40 @@ static void tiles(const Tuple& t, int64_t T[3]) {
     T[d] = (int64_t)t[F_TBX + d] * t[F_BMX + d] * t[F_CMX + d];
 }
 
+static int64_t xr_of(int r) { return r + (r & 1); }
+static int64_t rnd128(int64_t bytes) { return (bytes + 127) / 128 * 128; }
+
+// temporally blocked CTA (bt > 1): level lv extents, level 0 = TMA input box, lv = bt the
+// output tile (mirrors tb_wa / tb_wb in csrc/kernels/cst_kernels.cuh)
+static void tb_extent(int r, const Tuple& t, int lv, int64_t* ex, int64_t* ey) {
+  int64_t T[3];
+  tiles(t, T);
+  const int64_t k = t[F_BT] - lv;
+  *ex = T[0] + 2 * xr_of(r) * k;
+  *ey = T[1] + 2 * (int64_t)r * k;
+}
+
+static int64_t tb_blocks_per_thread(int r, const Tuple& t, int lv) {
+  int64_t ex, ey;
+  tb_extent(r, t, lv, &ex, &ey);
+  const int64_t nthr = (int64_t)t[F_TBX] * t[F_TBY] * t[F_TBZ];
+  return ((ex / t[F_BMX]) * (ey / t[F_BMY]) + nthr - 1) / nthr;
+}
+
+static int64_t tb_smem_bytes(int r, const Tuple& t) {
+  int64_t e0x, e0y, e1x, e1y;
+  tb_extent(r, t, 0, &e0x, &e0y);
+  tb_extent(r, t, 1, &e1x, &e1y);
+  return t[F_PF] * rnd128(e0x * e0y * 8) + (t[F_BT] - 1) * 2 * rnd128(e1x * e1y * 8);
+}
+
+static bool tb_path_ok(int kind, const Tuple& t) {
+  return (kind == CST_STAR || kind == CST_BOX) && t[F_STREAM] == 2 && t[F_SD] == 3 &&
+         t[F_STAGING] == 3 && t[F_RET] == 2 && t[F_TBZ] == 1 && t[F_BMZ] == 1 &&
+         t[F_CMX] == 1 && t[F_CMY] == 1 && t[F_CMZ] == 1 && t[F_BMX] <= 2 && t[F_BMY] <= 2 &&
+         t[F_UFX] == 1 && t[F_UFY] == 1 && t[F_UFZ] == 1;
+}
+
 // (P, NP): in-plane (or 3-D box) elements and ring planes of the modelled staging
 static void plane_geometry(int kind, int r, const Tuple& t, int64_t* P, int64_t* NP) {
   int64_t T[3];
@@ -87,6 +122,7 @@ static void plane_geometry(int kind, int r, const Tuple& t, int64_t* P, int64_t*
 
 int64_t model_smem_bytes(int kind, int r, const Tuple& t) {
   if (t[F_STAGING] == 1) return 0;
+  if (t[F_BT] > 1) return tb_smem_bytes(r, t);
   int64_t P, NP;
   plane_geometry(kind, r, t, &P, &NP);
   const int64_t plane = (P * 8 + 127) / 128 * 128;
@@ -96,6 +132,7 @@ int64_t model_smem_bytes(int kind, int r, const Tuple& t) {
 int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
   // mirrors csrc/kernels/cst_kernels.cuh: x halo XR = r rounded up to even
   if (t[F_STAGING] == 1) return 0;
+  if (t[F_BT] > 1) return tb_smem_bytes(r, t) + 2 * (int64_t)t[F_PF] * 8;  // + mbarriers
   const int64_t XR = r + (r & 1);
   int64_t T[3];
   tiles(t, T);
@@ -119,6 +156,13 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
 }
 
 int64_t model_regs(int kind, int r, const Tuple& t) {
+  if (t[F_BT] > 1) {
+    int64_t pts = 0;
+    for (int lv = 1; lv <= t[F_BT]; ++lv) pts += tb_blocks_per_thread(r, t, lv);
+    pts *= (int64_t)t[F_BMX] * t[F_BMY];
+    const int64_t win = (t[F_BMY] + 2 * (int64_t)r) * (t[F_BMX] + 2 * xr_of(r));
+    return 32 + 2 * ((2 * r + 1) * pts + win);
+  }
   int64_t ppt = 1;
   for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
   const int64_t nthr = (int64_t)t[F_TBX] * t[F_TBY] * t[F_TBZ];
@@ -138,6 +182,11 @@ static bool tma_ok(int r, const Tuple& t) {
   int64_t T[3];
   tiles(t, T);
   if (T[0] % 2) return false;
+  if (t[F_BT] > 1) {
+    int64_t ex, ey;
+    tb_extent(r, t, 0, &ex, &ey);
+    return ex <= 256 && ey <= 256;
+  }
   for (int d = 0; d < 3; ++d) {
     const bool streamed = t[F_STREAM] == 2 && d == t[F_SD] - 1;
     const int64_t e = streamed ? T[d] : T[d] + 2 * r;
@@ -166,6 +215,7 @@ const char* check_rules(const StencilInfo& st, const Tuple& t) {
   }
   if (t[F_RET] < 1 || t[F_RET] > 2) return "range: use_retiming";
   if (t[F_PF] < 1 || t[F_PF] > 4) return "range: prefetch";
+  if (t[F_BT] != 1 && t[F_BT] != 2 && t[F_BT] != 4) return "range: bt";
 
   const int64_t tb = (int64_t)t[F_TBX] * t[F_TBY] * t[F_TBZ];
   if (tb > 1024) return "R1";
@@ -190,6 +240,7 @@ const char* check_rules(const StencilInfo& st, const Tuple& t) {
   for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
   if (ppt > 16) return "R7";
   if (t[F_PF] > 1 && !stream) return "R9";
+  if (t[F_BT] > 1 && !tb_path_ok(st.kind, t)) return "R14";
   if (model_smem_bytes(st.kind, st.r, t) > SMEM_LIMIT) return "R10";
   if (model_regs(st.kind, st.r, t) > REG_LIMIT) return "R11";
   if (t[F_STAGING] == 3 && !tma_ok(st.r, t)) return "R12";
@@ -231,13 +282,17 @@ void Space::cores_for(const int32_t* pre, std::vector<Core>* cores) const {
                 if ((int64_t)pre[F_TBX + d] * cm[d] * bm[d] > st_.M[d]) cover = false;
               if (!cover) continue;
               for (int32_t ret = 1; ret <= 2; ++ret)
-                for (int32_t pf = 1; pf <= 4; ++pf) {
+                for (int32_t pf = 1; pf <= 4; ++pf)
+                  for (int32_t bt = 1; bt <= 4; bt *= 2) {
                   for (int d = 0; d < 3; ++d) {
                     t[F_CMX + d] = cm[d];
                     t[F_BMX + d] = bm[d];
                   }
                   t[F_RET] = ret;
                   t[F_PF] = pf;
+                  t[F_BT] = bt;
+                  // UF is not part of the core: R14 needs UF = 1, which the UF counts
+                  // below encode (a bt > 1 core admits only the first UF value per dim)
                   if (check_rules(st_, t) != nullptr) continue;
                   Core c;
                   for (int d = 0; d < 3; ++d) {
@@ -246,19 +301,20 @@ void Space::cores_for(const int32_t* pre, std::vector<Core>* cores) const {
                     const int64_t Td = (int64_t)pre[F_TBX + d] * cm[d] * bm[d];
                     const int64_t trip = (stream && d == sd) ? pre[F_SB] / Td
                                                              : (int64_t)cm[d] * bm[d];
-                    c.nuf[d] = count_le(p2_[d], trip);
+                    c.nuf[d] = bt > 1 ? 1 : count_le(p2_[d], trip);
                   }
                   c.ret = ret;
                   c.pf = pf;
+                  c.bt = bt;
                   cores->push_back(c);
                 }
             }
       }
-  // canonical core order: CMx, CMy, CMz, BMx, BMy, BMz, ret, pf
+  // canonical core order: CMx, CMy, CMz, BMx, BMy, BMz, ret, pf, bt
   std::stable_sort(cores->begin(), cores->end(), [](const Core& a, const Core& b) {
-    const int32_t ka[8] = {a.cm[0], a.cm[1], a.cm[2], a.bm[0], a.bm[1], a.bm[2], a.ret, a.pf};
-    const int32_t kb[8] = {b.cm[0], b.cm[1], b.cm[2], b.bm[0], b.bm[1], b.bm[2], b.ret, b.pf};
-    return std::lexicographical_compare(ka, ka + 8, kb, kb + 8);
+    const int32_t ka[9] = {a.cm[0], a.cm[1], a.cm[2], a.bm[0], a.bm[1], a.bm[2], a.ret, a.pf, a.bt};
+    const int32_t kb[9] = {b.cm[0], b.cm[1], b.cm[2], b.bm[0], b.bm[1], b.bm[2], b.ret, b.pf, b.bt};
+    return std::lexicographical_compare(ka, ka + 9, kb, kb + 9);
   });
 }
 
@@ -351,6 +407,7 @@ bool Space::at(uint64_t rank, Tuple* out) const {
       }
       t[F_RET] = c.ret;
       t[F_PF] = c.pf;
+      t[F_BT] = c.bt;
       *out = t;
       return true;
     }
@@ -402,7 +459,7 @@ bool Space::rank(const Tuple& t, uint64_t* out) const {
   }
   for (const Core& c : cores) {
     if (uidx[0] >= c.nuf[0] || uidx[1] >= c.nuf[1] || uidx[2] >= c.nuf[2]) continue;
-    bool same = c.ret == t[F_RET] && c.pf == t[F_PF];
+    bool same = c.ret == t[F_RET] && c.pf == t[F_PF] && c.bt == t[F_BT];
     for (int d = 0; d < 3; ++d)
       same = same && c.cm[d] == t[F_CMX + d] && c.bm[d] == t[F_BMX + d];
     if (same) {

@@ -393,6 +393,7 @@ extern "C" void cst_tune_opts_default(cst_tune_opts* o) {
   o->quantile_sample = 65536;
   o->warm_start = 1;
   o->metrics_mode = 0;
+  o->nsteps = 1;
 }
 
 namespace {
@@ -423,8 +424,20 @@ struct Evaluator {
     return metrics_source == "cupti" ? kHwMetrics : kModelMetrics;
   }
 
+  // device copies for multi-step timing (ping-pong overwrites its input)
+  double* tin = nullptr;
+  double* tout = nullptr;
+
+  // the setting that actually runs for the workload: one step never fuses sweeps
+  Tuple effective(Tuple t) const {
+    if (o->nsteps <= 1 && check_rules(h->info, t) == nullptr) t[F_BT] = 1;
+    return t;
+  }
+
   // evaluate (memoised) a batch; invalid settings (rules) get ms = inf without timing
-  cst_status run(const std::vector<Tuple>& cands, std::vector<EvalResult>* res) {
+  cst_status run(const std::vector<Tuple>& cands_in, std::vector<EvalResult>* res) {
+    std::vector<Tuple> cands;
+    for (const Tuple& t : cands_in) cands.push_back(effective(t));
     std::vector<Tuple> todo;
     std::set<Tuple> seen;
     for (const Tuple& t : cands)
@@ -458,10 +471,30 @@ struct Evaluator {
           });
         for (auto& th : pool) th.join();
         jit_s += std::chrono::duration<double>(std::chrono::steady_clock::now() - j0).count();
+        const int nsteps = std::max(1, o->nsteps);
+        const int64_t numel = (h->grid.nz + 2 * (int64_t)h->grid.halo) * h->grid.pitch_y *
+                              h->grid.pitch_x;
+        if (nsteps > 1 && !tin) {
+          if (cudaMalloc(&tin, numel * 8) != cudaSuccess ||
+              cudaMalloc(&tout, numel * 8) != cudaSuccess) {
+            cudaGetLastError();
+            return fail(CST_E_OOM, "tuner: multi-step timing buffers");
+          }
+        }
         for (size_t i = 0; i < ss.size(); ++i) {
           double m = INFINITY;
-          const cst_status st = cst_time_setting(h, &ss[i], in, out, o->warmup,
-                                                 std::max(1, o->reps), stream, &m);
+          cst_status st;
+          if (nsteps > 1) {
+            // fresh copy of the input for every candidate (values stay bounded)
+            CST_CUDA(cudaMemcpyAsync(tin, in[0], numel * 8, cudaMemcpyDeviceToDevice, stream));
+            const double* ti[1] = {tin};
+            double* to[1] = {tout};
+            st = cst_time_setting(h, &ss[i], ti, to, nsteps, o->warmup, std::max(1, o->reps),
+                                  stream, &m);
+          } else {
+            st = cst_time_setting(h, &ss[i], in, out, 1, o->warmup, std::max(1, o->reps),
+                                  stream, &m);
+          }
           if (st == CST_E_CUDA) return st;  // sticky device error: stop
           ms[i] = st == CST_OK ? m : INFINITY;
         }
@@ -542,6 +575,15 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
       if (s) cudaStreamDestroy(s);
     }
   } guard{ev.stream};
+  struct BufGuard {
+    Evaluator& e;
+    ~BufGuard() {
+      if (e.tin) cudaFree(e.tin);
+      if (e.tout) cudaFree(e.tout);
+    }
+  } bguard{ev};
+  if (o->nsteps > 1 && h->desc.n_inputs != h->desc.n_outputs)
+    return fail(CST_E_INVALID, "cst_tune: nsteps > 1 needs n_inputs == n_outputs");
 
   Json js;
   js.o << "{";
@@ -924,7 +966,7 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
     if (o->time_budget_s > 0 && elapsed() > o->time_budget_s) break;
   }
   js.o << "]";
-  *best_out = from_tuple(cur);
+  *best_out = from_tuple(ev.effective(cur));
   rep->best_ms = cur_ms;
   rep->best_gstencils = std::isfinite(cur_ms)
                             ? (double)h->grid.nx * h->grid.ny * h->grid.nz / (cur_ms * 1e-3) / 1e9

@@ -30,7 +30,7 @@ N_OUT = {CST_STAR: 1, CST_BOX: 1, CST_HYPTERM: 5, CST_RHS4: 3}
 
 FIELDS = ("tb_x", "tb_y", "tb_z", "staging", "use_constant", "use_streaming", "sd", "sb",
           "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z", "bm_x", "bm_y", "bm_z",
-          "use_retiming", "prefetch")
+          "use_retiming", "prefetch", "bt")
 
 
 class CstError(RuntimeError):
@@ -63,7 +63,8 @@ class cst_setting(ctypes.Structure):
                 ("use_constant", ctypes.c_int32), ("use_streaming", ctypes.c_int32),
                 ("sd", ctypes.c_int32), ("sb", ctypes.c_int32), ("uf", ctypes.c_int32 * 3),
                 ("cm", ctypes.c_int32 * 3), ("bm", ctypes.c_int32 * 3),
-                ("use_retiming", ctypes.c_int32), ("prefetch", ctypes.c_int32)]
+                ("use_retiming", ctypes.c_int32), ("prefetch", ctypes.c_int32),
+                ("bt", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         d = {}
@@ -73,7 +74,7 @@ class cst_setting(ctypes.Structure):
             d["cm_" + ax] = self.cm[i]
             d["bm_" + ax] = self.bm[i]
         for f in ("staging", "use_constant", "use_streaming", "sd", "sb", "use_retiming",
-                  "prefetch"):
+                  "prefetch", "bt"):
             d[f] = getattr(self, f)
         return {k: d[k] for k in FIELDS}
 
@@ -92,6 +93,7 @@ class cst_setting(ctypes.Structure):
         for f in ("staging", "use_constant", "use_streaming", "sd", "sb", "use_retiming",
                   "prefetch"):
             setattr(s, f, d[f])
+        s.bt = d.get("bt", 1)   # field 20 (temporal blocking); older records predate it
         return s
 
     def __repr__(self):
@@ -114,7 +116,8 @@ class cst_tune_opts(ctypes.Structure):
                 ("num_collections", ctypes.c_int32), ("time_budget_s", ctypes.c_double),
                 ("reps", ctypes.c_int32), ("warmup", ctypes.c_int32), ("log_path", ctypes.c_char_p),
                 ("n_user_metrics", ctypes.c_int32), ("quantile_sample", ctypes.c_int32),
-                ("warm_start", ctypes.c_int32), ("metrics_mode", ctypes.c_int32)]
+                ("warm_start", ctypes.c_int32), ("metrics_mode", ctypes.c_int32),
+                ("nsteps", ctypes.c_int32)]
 
 
 class cst_tune_report(ctypes.Structure):
@@ -167,7 +170,7 @@ _decl("cst_last_launch_count", ctypes.c_int64, _P)
 _decl("cst_fill_uniform", _S, ctypes.POINTER(cst_grid), _P, ctypes.c_uint64, ctypes.c_uint64,
       ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_double, _P)
 _decl("cst_time_setting", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP, ctypes.c_int32,
-      ctypes.c_int32, _P, ctypes.POINTER(ctypes.c_double))
+      ctypes.c_int32, ctypes.c_int32, _P, ctypes.POINTER(ctypes.c_double))
 _decl("cst_collect_metrics", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP,
       ctypes.POINTER(ctypes.c_char_p), ctypes.c_int32, ctypes.POINTER(ctypes.c_double))
 _decl("cst_fp64_peak", _S, ctypes.c_int, ctypes.POINTER(ctypes.c_double),
@@ -296,12 +299,14 @@ def cst_fill_uniform(grid: cst_grid, dev_ptr: int, seed: int, array_id: int, nx_
                                 ctypes.c_void_p(stream)))
 
 
-def cst_time_setting(h, s: cst_setting, in_ptrs, out_ptrs, warmup=2, reps=5, stream=0) -> float:
+def cst_time_setting(h, s: cst_setting, in_ptrs, out_ptrs, warmup=2, reps=5, stream=0,
+                     nsteps=1) -> float:
+    """Median ms PER STEP of `reps` timed cst_sweep calls of `nsteps` steps."""
     pi, _a = _ptrs(in_ptrs)
     po, _b = _ptrs(out_ptrs)
     ms = ctypes.c_double()
-    check(_lib.cst_time_setting(h, ctypes.byref(s), pi, po, warmup, reps, ctypes.c_void_p(stream),
-                                ctypes.byref(ms)))
+    check(_lib.cst_time_setting(h, ctypes.byref(s), pi, po, nsteps, warmup, reps,
+                                ctypes.c_void_p(stream), ctypes.byref(ms)))
     return ms.value
 
 

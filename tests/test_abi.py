@@ -131,6 +131,14 @@ def test_rules_agree_with_oracle_on_random_tuples():
                 d["uf_" + ax] = rng.choice(p2(M[i])[:4])
                 d["cm_" + ax] = rng.choice(p2(M[i])[:3])
                 d["bm_" + ax] = rng.choice(p2(M[i])[:4])
+            d["bt"] = rng.choice([1, 1, 2, 4])
+            if rng.random() < 0.3:              # the temporally blocked path's shape (R14)
+                d.update(use_streaming=2, sd=3, staging=3, use_retiming=2, tb_z=1, bm_z=1,
+                         bt=rng.choice([2, 4]), sb=rng.choice(p2(M[2])))
+                for ax in "xyz":
+                    d["cm_" + ax] = d["uf_" + ax] = 1
+                d["bm_x"], d["bm_y"] = rng.choice([1, 2]), rng.choice([1, 2])
+                d["tb_x"], d["tb_y"] = rng.choice([8, 16, 32, 64]), rng.choice([1, 2, 4, 8])
             want = S.check(kind, r, M, d)
             s = C.cst_setting.from_dict(d)
             try:

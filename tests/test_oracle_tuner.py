@@ -145,7 +145,7 @@ def test_literal_table1_counts():
 def test_space_rules_spot_checks():
     base = dict(tb_x=32, tb_y=4, tb_z=1, staging=3, use_constant=1, use_streaming=2, sd=3,
                 sb=64, uf_x=1, uf_y=1, uf_z=1, cm_x=1, cm_y=1, cm_z=1, bm_x=1, bm_y=1, bm_z=1,
-                use_retiming=2, prefetch=2)
+                use_retiming=2, prefetch=2, bt=1)
     M = (512, 512, 512)
     assert S.check(1, 4, M, base) is None
     assert S.check(1, 4, M, dict(base, tb_x=64, tb_y=32)) == "R1"
@@ -162,6 +162,24 @@ def test_space_rules_spot_checks():
     assert S.check(1, 4, M, dict(base, tb_x=128, tb_y=1)) is None
     assert S.check(1, 4, M, dict(base, tb_x=256, tb_y=1)) == "R12"
     assert S.check(1, 4, M, dict(base, tb_x=32, tb_y=1, bm_x=8)) == "R12"
+    # temporal blocking (field 20): R14 structure, models by hand
+    tb = dict(base, bm_x=2, bm_y=2, bt=2)
+    assert S.check(2, 1, M, tb) is None
+    assert S.check(3, 4, M, tb) == "R14"                       # hypterm: no fused path
+    assert S.check(2, 1, M, dict(tb, staging=2)) == "R14"
+    assert S.check(2, 1, M, dict(tb, use_retiming=1)) == "R14"
+    assert S.check(2, 1, M, dict(tb, sd=2, sb=64)) == "R14"
+    assert S.check(2, 1, M, dict(tb, uf_z=2)) == "R14"
+    assert S.check(2, 1, M, dict(tb, bm_x=4, tb_x=16)) == "R14"
+    assert S.check(2, 1, M, dict(tb, cm_x=2, tb_x=16)) == "R14"
+    # box r=1, tile 64x8, bt=2, 2 stages: input box (64+2*2*2)x(8+2*2) = 72x12 doubles
+    # = 6912 B per ring slot; level 1 (64+4)x(8+2) = 680 doubles = 5440 B -> 5504 B slots
+    assert S.smem_bytes(2, 1, tb) == 2 * 6912 + 2 * 5504
+    # registers: level 1 has 34x5 = 170 blocks -> 2 per thread, level 2 128 -> 1; 3 blocks
+    # x 4 points x 3 accumulators + a (2+2)x(2+4) window = 36 + 24 doubles
+    assert S.est_regs(2, 1, tb) == 32 + 2 * (36 + 24)
+    assert S.check(1, 4, M, dict(tb, bt=4)) == "R11"
+    assert S.check(2, 1, M, dict(tb, tb_x=128, tb_y=1, bm_y=1)) == "R12"  # 256 + 8 > 256
 
 
 def test_space_enumeration_small_is_sorted_and_valid():

@@ -117,7 +117,7 @@ def test_groups_collections_selection_bit_exact(tuned, space_list):
     _, _, log, _ = tuned
     o = _oracle_preprocess(log, space_list)
     assert log["groups"] == o["groups"]
-    assert sorted(p for g in o["groups"] for p in g) == list(range(19))
+    assert sorted(p for g in o["groups"] for p in g) == list(range(len(S.FIELDS)))
     assert log["collections"] == o["cols"]
     assert log["selected"] == o["sel"]
 
