@@ -218,6 +218,41 @@ def other_configs(C, torch, peak, steps=10, fp64_peak=None):
     return res
 
 
+TBLOCK_SETTING = dict(tb_x=32, tb_y=8, tb_z=1, staging=3, use_constant=1, use_streaming=2, sd=3,
+                      sb=128, uf_x=1, uf_y=1, uf_z=1, cm_x=1, cm_y=1, cm_z=1, bm_x=2, bm_y=2,
+                      bm_z=1, use_retiming=2, prefetch=2)
+
+
+def tblock_config(C, torch, peak, nsteps=8, steps=5):
+    """temporal blocking.  8 ping-pong steps of the order-1 (7-point) star at
+    512^3 per cst_sweep call, ms per step, with the fused bt = 2 setting (measured best,
+    profiles/r01_tblock_explore.json) against the same tile unfused (bt = 1).  Algorithmic
+    HBM bytes per step = 16 B / bt per point."""
+    n, r = (512, 512, 512), 1
+    g = C.make_grid(*n, r)
+    w = [1.0, -2.0, 1.0]
+    h = C.cst_stencil_create(1, r, [3 * w[1]] + [w[0], w[2]] * 3, g)
+    ins = [torch.empty(g.numel, dtype=torch.float64, device="cuda")]
+    outs = [torch.empty(g.numel, dtype=torch.float64, device="cuda")]
+    pts = n[0] * n[1] * n[2]
+    res = {"workload": "SURVEY NEXT-2: 7-point star (order 1), 512^3, 8 steps per call, "
+                       "temporal blocking bt=2 vs bt=1 (ms per step)", "nsteps": nsteps}
+    for bt in (1, 2):
+        s = C.cst_setting.from_dict(dict(TBLOCK_SETTING, bt=bt))
+        C.cst_fill_uniform(g, ins[0].data_ptr(), 7, 0)
+        ms = C.cst_time_setting(h, s, [ins[0].data_ptr()], [outs[0].data_ptr()], 2, steps,
+                                torch.cuda.current_stream().cuda_stream, nsteps=nsteps)
+        gbs = pts * 16.0 / bt / (ms * 1e-3) / 1e9
+        res[f"bt{bt}"] = {"gstencils_per_step": pts / (ms * 1e-3) / 1e9, "ms_per_step": ms,
+                          "alg_hbm_bytes_per_point_step": 16.0 / bt, "achieved_GBs": gbs,
+                          "hbm_frac_measured": gbs / peak, "setting": s.as_dict()}
+    res["speedup_bt2_over_bt1"] = res["bt2"]["gstencils_per_step"] / res["bt1"]["gstencils_per_step"]
+    del ins, outs
+    C.cst_stencil_destroy(h)
+    torch.cuda.empty_cache()
+    return res
+
+
 def cpu_baseline(target_s: float = 10.0):
     """The oracle, as it stands, on a bounded sample of the same workload: a 512 x 512 x 16
     slab of the 512^3 star25 grid swept repeatedly until >= target_s seconds."""
@@ -405,6 +440,7 @@ def main():
             fp64_peak = None
         others = other_configs(C, torch, peak, fp64_peak=fp64_peak)
         others["fp64_peak_TFLOPs_measured"] = fp64_peak
+        others["next2_tblock_star7_512_T8"] = tblock_config(C, torch, peak)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
