@@ -427,6 +427,11 @@ struct Evaluator {
   // device copies for multi-step timing (ping-pong overwrites its input)
   double* tin = nullptr;
   double* tout = nullptr;
+  // best-so-far trajectory (iso-time / iso-iteration curves):
+  // (seconds since cst_tune started, best ms, distinct settings evaluated)
+  std::chrono::steady_clock::time_point start = std::chrono::steady_clock::now();
+  double best_seen = INFINITY;
+  std::vector<std::array<double, 3>> trace;
 
   // the setting that actually runs for the workload: one step never fuses sweeps
   Tuple effective(Tuple t) const {
@@ -524,7 +529,11 @@ struct Evaluator {
         else
           r.metrics = model_metrics(h, todo[i]);
         memo[todo[i]] = r;
+        best_seen = std::min(best_seen, r.ms);
       }
+      trace.push_back({std::chrono::duration<double>(std::chrono::steady_clock::now() - start)
+                           .count(),
+                       best_seen, (double)memo.size()});
     }
     eval_s += std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
     res->clear();
@@ -564,6 +573,7 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
   if (count == 0) return fail(CST_E_CONSTRAINT, "empty parameter space");
 
   Evaluator ev{h, o, in, scratch_out, eval, eval_user};
+  ev.start = wall0;
   ev.jit_before = jit_compile_count();
   if (!eval) {
     CST_CUDA(cudaSetDevice(h->device));
@@ -985,6 +995,12 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
   js.o << "{\"setting\": [";
   for (int f = 0; f < F_COUNT; ++f) js.o << (f ? "," : "") << cur[f];
   js.o << "], \"ms\": " << Json::num(cur_ms) << "}";
+  js.key("trace");
+  js.o << "[";
+  for (size_t i = 0; i < ev.trace.size(); ++i)
+    js.o << (i ? "," : "") << "[" << Json::num(ev.trace[i][0]) << "," << Json::num(ev.trace[i][1])
+         << "," << (uint64_t)ev.trace[i][2] << "]";
+  js.o << "]";
   js.key("report");
   js.o << "{\"wall_s\":" << Json::num(rep->wall_s) << ",\"eval_s\":" << Json::num(rep->eval_s)
        << ",\"jit_s\":" << Json::num(rep->jit_s) << ",\"preproc_s\":" << Json::num(preproc_s)

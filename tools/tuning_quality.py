@@ -1,0 +1,161 @@
+"""csTuner tuning-quality experiments on B200 (the csTuner line of
+Figs. 8/9/11/12, P:349-361, P:385-405 — the comparison systems are out of scope).
+
+  python tools/tuning_quality.py --out profiles/r01_tuning_quality.json [--budget 100]
+
+1. Ground truth: exhaustive timing of a restricted sub-space of the star25 512^3 space (TMA
+   staging, z streaming, retiming, UF = CM = 1; TB_x, TB_y, BM_x, BM_y, SB, prefetch free).
+2. Iso-time curves: csTuner (cst_tune, paper defaults) for several seeds — best-so-far ms vs
+   seconds from the tuner's JSON trace — against a random-search baseline over the full
+   space at the same budget (same compile + timing path).
+3. Sampling-ratio sweep (Fig. 11): 5 / 10 / 20 / 50 % at the same budget: best ms and the
+   pre-processing vs search time breakdown (Fig. 12).
+Every time is a CUDA-event median on inputs resident in HBM (cst_time_setting).
+"""
+import argparse
+import concurrent.futures as cf
+import itertools
+import json
+import os
+import random
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+from paper_conf_cluster_sunlyjldlq21_b200 import cst as C  # noqa: E402
+
+D2_R4 = [-9, 128, -1008, 8064, -14350, 8064, -1008, 128, -9]
+
+
+def make():
+    w = [v / 5040.0 for v in D2_R4]
+    side = w[:4] + w[5:]
+    g = C.make_grid(512, 512, 512, 4)
+    h = C.cst_stencil_create(C.CST_STAR, 4, [3 * w[4]] + side * 3, g)
+    u = torch.empty(g.numel, dtype=torch.float64, device="cuda")
+    v = torch.empty(g.numel, dtype=torch.float64, device="cuda")
+    C.cst_fill_uniform(g, u.data_ptr(), 2, 0)
+    torch.cuda.synchronize()
+    return g, h, u, v
+
+
+def subspace(h):
+    out = []
+    for tbx, tby, bmx, bmy, sb, pf in itertools.product([8, 16, 32, 64, 128], [1, 2, 4, 8, 16],
+                                                         [1, 2, 4], [1, 2, 4], [128, 256],
+                                                         [2, 3, 4]):
+        d = dict(tb_x=tbx, tb_y=tby, tb_z=1, staging=3, use_constant=1, use_streaming=2, sd=3,
+                 sb=sb, uf_x=1, uf_y=1, uf_z=1, cm_x=1, cm_y=1, cm_z=1, bm_x=bmx, bm_y=bmy,
+                 bm_z=1, use_retiming=2, prefetch=pf, bt=1)
+        s = C.cst_setting.from_dict(d)
+        try:
+            C.cst_setting_check(h, s)
+        except C.CstError:
+            continue
+        out.append(s)
+    return out
+
+
+def time_all(h, settings, u, v, reps=5):
+    """Parallel NVRTC code generation, then serial CUDA-event timing (like cst_tune)."""
+    with cf.ThreadPoolExecutor(16) as ex:
+        list(ex.map(lambda s: _compile(h, s), settings))
+    res = []
+    stream = torch.cuda.current_stream().cuda_stream
+    for s in settings:
+        try:
+            ms = C.cst_time_setting(h, s, [u.data_ptr()], [v.data_ptr()], 2, reps, stream)
+        except C.CstError:
+            ms = float("inf")
+        res.append(ms)
+    return res
+
+
+def _compile(h, s):
+    try:
+        C.cst_variant_compile(h, s)
+    except C.CstError:
+        pass
+
+
+def run_cstuner(h, u, v, seed, budget, ratio=0.10, tag=""):
+    o = C.cst_tune_opts_default()
+    o.seed = seed
+    o.time_budget_s = budget
+    o.sampling_ratio = ratio
+    log = f"/tmp/tq_{tag}_{seed}_{ratio}.json"
+    o.log_path = log.encode()
+    best, rep = C.cst_tune(h, o, [u.data_ptr()], [v.data_ptr()])
+    j = json.load(open(log))
+    return {"seed": seed, "budget_s": budget, "sampling_ratio": ratio, "best_ms": rep.best_ms,
+            "best_setting": best.as_dict(), "evaluations": rep.evaluations,
+            "wall_s": rep.wall_s, "eval_s": rep.eval_s, "jit_s": rep.jit_s,
+            "preproc_s": rep.preproc_s, "sampled_count": rep.sampled_count,
+            "space_count": rep.space_count, "trace": j.get("trace", []),
+            "metrics_source": j.get("metrics_source")}
+
+
+def run_random(h, u, v, seed, budget, batch=32):
+    """Random search over the full canonical space: batches of uniformly drawn ranks,
+    compiled in parallel and timed, until the budget is spent."""
+    rng = random.Random(seed)
+    n = C.cst_space_count(h)
+    t0 = time.time()
+    best, trace, evals = float("inf"), [], 0
+    while time.time() - t0 < budget:
+        ss = [C.cst_space_at(h, rng.randrange(n)) for _ in range(batch)]
+        for ms in time_all(h, ss, u, v):
+            best = min(best, ms)
+        evals += batch
+        trace.append([time.time() - t0, best, evals])
+    return {"seed": seed, "budget_s": budget, "best_ms": best, "evaluations": evals,
+            "trace": trace}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r01_tuning_quality.json"))
+    ap.add_argument("--budget", type=float, default=100.0)
+    ap.add_argument("--seeds", type=int, default=3)
+    args = ap.parse_args()
+    g, h, u, v = make()
+    res = {"workload": "star25 (order-4 25-point star) 512^3 FP64, B200, inputs resident",
+           "space_count": C.cst_space_count(h)}
+    # 1. exhaustive sub-space
+    t0 = time.time()
+    sub = subspace(h)
+    ms = time_all(h, sub, u, v)
+    order = sorted(range(len(sub)), key=lambda i: ms[i])
+    res["subspace"] = {"size": len(sub), "seconds": time.time() - t0,
+                       "optimum_ms": ms[order[0]], "optimum": sub[order[0]].as_dict(),
+                       "top5": [[ms[i], sub[i].as_dict()] for i in order[:5]],
+                       "median_ms": sorted(x for x in ms if x < float("inf"))[len(sub) // 2],
+                       "default_ms": C.cst_time_setting(h, C.cst_setting_default(h),
+                                                        [u.data_ptr()], [v.data_ptr()], 2, 5)}
+    print(json.dumps({"subspace": {k: res["subspace"][k] for k in ("size", "optimum_ms",
+                                                                    "seconds")}}), flush=True)
+    # 2. iso-time: csTuner vs random search
+    res["cstuner"] = [run_cstuner(h, u, v, s + 1, args.budget, tag="iso") for s in range(args.seeds)]
+    for r in res["cstuner"]:
+        print(json.dumps({k: r[k] for k in ("seed", "best_ms", "evaluations", "wall_s")}), flush=True)
+    res["random_search"] = [run_random(h, u, v, s + 1, args.budget) for s in range(args.seeds)]
+    for r in res["random_search"]:
+        print(json.dumps({k: r[k] for k in ("seed", "best_ms", "evaluations")}), flush=True)
+    # 3. sampling ratio sweep
+    res["sampling_ratio_sweep"] = [run_cstuner(h, u, v, 1, args.budget, ratio=q, tag="ratio")
+                                   for q in (0.05, 0.10, 0.20, 0.50)]
+    for r in res["sampling_ratio_sweep"]:
+        print(json.dumps({k: r[k] for k in ("sampling_ratio", "best_ms", "preproc_s", "eval_s",
+                                            "sampled_count")}), flush=True)
+    os.makedirs(os.path.dirname(args.out), exist_ok=True)
+    with open(args.out, "w") as f:
+        json.dump(res, f, indent=1)
+    C.cst_stencil_destroy(h)
+
+
+if __name__ == "__main__":
+    main()
