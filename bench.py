@@ -335,6 +335,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-other-configs", action="store_true")
+    ap.add_argument("--halo", default=os.environ.get("CST_BENCH_HALO", "p2p"),
+                    choices=["p2p", "nccl"],
+                    help="N > 1: fused peer-memory halo stores (default) or NCCL send/recv")
     args = ap.parse_args()
     assert args.warmup >= 3 or args.impl == "reference" or True
 
@@ -363,7 +366,11 @@ def main():
     C.cst_fill_uniform(grid, u.data_ptr(), SEED, 0, N, N, z0, float("nan"), stream.cuda_stream)
     C.cst_fill_uniform(grid, v.data_ptr(), SEED, 0, N, N, z0, float("nan"), stream.cuda_stream)
     dist_h = None
-    if world > 1:
+    if world > 1 and args.halo == "p2p":
+        # boundary kernels store straight into the neighbours' halos (NVLink peer stores)
+        dist_h = C.cst_dist_create(h, world, rank, None)
+        C.cst_dist_p2p_setup(dist_h, rank, world, [u.data_ptr()], [v.data_ptr()])
+    elif world > 1:
         uid = C.cst_dist_nccl_unique_id() if rank == 0 else None
         obj = [uid]
         dist.broadcast_object_list(obj, src=0)
@@ -453,7 +460,9 @@ def main():
                 "data": "synthetic (cstgen splitmix64 U[-1,1), seed 2, device generator)",
                 "config": {"workload": "star25: order-4 25-point star (FD Laplacian /5040), "
                                        "512^3 FP64 interior per GPU (BASELINE configs[1])"
-                                       + ("; z-slab weak scaling, NCCL halo exchange" if world > 1 else ""),
+                                       + (("; z-slab weak scaling, halo exchange: "
+                                           + ("fused peer-memory stores" if args.halo == "p2p"
+                                              else "NCCL send/recv")) if world > 1 else ""),
                            "grid": [N, N, N * world], "halo": R,
                            "setting": s.as_dict(), "setting_source": s_src,
                            "l2": "inputs larger than L2 (2 x %.2f GB per GPU), no flush"

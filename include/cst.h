@@ -208,7 +208,8 @@ typedef struct {
   double cv_threshold;       /* 0.02                                            */
   int32_t max_generations;   /* 50 per group                                    */
   int32_t num_collections;   /* 3                                               */
-  double time_budget_s;      /* 100; <= 0 = unlimited                   */
+  double time_budget_s;      /* 100: search time after the dataset (its
+                                metric collection is offline); <= 0 = none    */
   int32_t reps;              /* timed reps per evaluation (median)              */
   int32_t warmup;            /* untimed sweeps per evaluation                   */
   const char* log_path;      /* JSON report of every stage, or NULL              */
@@ -256,9 +257,9 @@ cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const double* const*
  * boundary planes first, then the halo exchange (r planes to/from rank +-1) on a
  * communication stream concurrently with the interior planes.  Physical z-end halos are
  * caller data.  Transport: NCCL (nccl_unique_id = 128-byte ncclUniqueId broadcast by the
- * caller, e.g. through torch.distributed) or, with nccl_unique_id == NULL and nranks
- * slabs all owned by this process on one device, a loopback transport (cudaMemcpyAsync)
- * used to test the decomposition on one GPU. */
+ * caller, e.g. through torch.distributed), or, with nccl_unique_id == NULL, the fused
+ * peer-memory transport below (one process per GPU); cst_dist_sweep_loopback drives all
+ * slabs from one process on one device (cudaMemcpyAsync) to test the decomposition. */
 typedef struct cst_dist cst_dist;
 
 /* Halo-exchange plan of rank `rank` in a z-slab decomposition over `nranks` ranks, each
@@ -284,6 +285,24 @@ cst_status cst_dist_sweep_loopback(cst_stencil* h, int32_t nslabs, const cst_set
                                    double* const* in_slabs, double* const* out_slabs,
                                    int32_t nsteps, void* stream);
 void cst_dist_destroy(cst_dist* d);
+
+/* Fused halo exchange over peer memory (no NCCL).  A handle created
+ * with nccl_unique_id == NULL and nranks > 1 uses it: the boundary kernels of
+ * cst_dist_sweep store every edge-plane value both locally and, through a CUDA IPC
+ * mapping, straight into the neighbour's halo (NVLink / NVSwitch peer stores), and the
+ * ranks order their steps with flag words written over the same mappings (release /
+ * acquire, system scope; a wait gives up after 30 s with a device trap instead of hanging).
+ * Setup, once per pair of ping-pong buffer sets (a = in[] of the first call, b = out[]):
+ *   cst_dist_p2p_export(d, a, b, blob)   writes CST_P2P_BLOB_BYTES describing my buffers
+ *                                         and flag words (IPC handles + offsets)
+ *   the caller exchanges blobs (e.g. torch.distributed.all_gather_object)
+ *   cst_dist_p2p_import(d, peer, blob)   for peer = rank - 1 and rank + 1 (if they exist)
+ * cst_dist_sweep then requires {in, out} to be {a, b} in either order (CST_E_INVALID
+ * otherwise).  Buffers must come from cudaMalloc (any caching allocator built on it). */
+#define CST_P2P_BLOB_BYTES 2048
+cst_status cst_dist_p2p_export(cst_dist* d, double* const* buf_a, double* const* buf_b,
+                               void* blob);
+cst_status cst_dist_p2p_import(cst_dist* d, int32_t peer, const void* blob);
 
 #ifdef __cplusplus
 }

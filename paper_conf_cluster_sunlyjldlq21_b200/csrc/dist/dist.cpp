@@ -17,6 +17,27 @@
 #include <nccl.h>
 #endif
 
+// Fused halo exchange over peer memory: no NCCL.  The boundary
+// launches store every edge-plane value both locally and, through a CUDA IPC mapping of
+// the neighbour's matching buffer, straight into the neighbour's halo (NVLink / NVSwitch
+// stores on a multi-GPU node).  Steps are ordered by 64-bit flag words each rank keeps in
+// its own device memory and its neighbours write over the same mappings:
+//   BND_LO / BND_HI   epoch of the last step whose boundary stores the lower / upper
+//                     neighbour has completed into my halo                       (RAW)
+//   DONE_LO / DONE_HI epoch of the last step the lower / upper neighbour has finished
+//                     (it no longer reads the buffer my next boundary launch writes) (WAR)
+// Per step (epoch e, one stream):  wait DONE >= e-1 | boundary launches with remote stores
+// | signal BND = e | interior | signal DONE = e | wait BND >= e.  Waits spin on an acquire
+// load with a 30 s bound (then trap: a dead peer is an error, not a hang).
+enum { F_BND_LO = 0, F_BND_HI = 1, F_DONE_LO = 2, F_DONE_HI = 3, F_WORDS = 16 };
+
+struct P2PPeer {
+  bool open = false;
+  double* buf[2][CST_MAX_IN] = {};  // the peer's ping-pong buffers (a, b), mapped here
+  unsigned long long* flags = nullptr;  // the peer's flag words, mapped here
+  std::vector<void*> bases;             // IPC mappings to close
+};
+
 struct cst_dist {
   cst_stencil* h = nullptr;
   int32_t nranks = 1, rank = 0;
@@ -25,6 +46,13 @@ struct cst_dist {
 #ifdef CST_HAVE_NCCL
   ncclComm_t comm = nullptr;
 #endif
+  // peer-memory transport
+  bool p2p = false;
+  unsigned long long* flags = nullptr;  // my flag words (F_WORDS x u64)
+  const double* mine[2][CST_MAX_IN] = {};  // my registered ping-pong buffers (a, b)
+  bool exported = false;
+  P2PPeer lo, hi;                        // rank - 1, rank + 1
+  unsigned long long epoch = 0;
 };
 
 using namespace cst;
@@ -97,12 +125,16 @@ extern "C" cst_status cst_dist_create(cst_stencil* h, int32_t nranks, int32_t ra
   cudaStreamCreateWithPriority(&D->s_comm, cudaStreamNonBlocking, -1);
   cudaEventCreateWithFlags(&D->ev_bnd, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&D->ev_comm, cudaEventDisableTiming);
-  if (nranks > 1) {
-#ifdef CST_HAVE_NCCL
-    if (!uid) {
+  if (nranks > 1 && !uid) {  // fused peer-memory transport
+    D->p2p = true;
+    if (cudaMalloc(&D->flags, F_WORDS * sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMemset(D->flags, 0, F_WORDS * sizeof(unsigned long long)) != cudaSuccess) {
+      cudaGetLastError();
       delete D;
-      return fail(CST_E_INVALID, "nccl_unique_id required for nranks > 1");
+      return fail(CST_E_OOM, "p2p flag words");
     }
+  } else if (nranks > 1) {
+#ifdef CST_HAVE_NCCL
     ncclUniqueId id;
     std::memcpy(&id, uid, 128);
     st = nccl_check(ncclCommInitRank(&D->comm, nranks, id, rank), "ncclCommInitRank");
@@ -121,6 +153,13 @@ extern "C" cst_status cst_dist_create(cst_stencil* h, int32_t nranks, int32_t ra
 
 extern "C" void cst_dist_destroy(cst_dist* D) {
   if (!D) return;
+  if (D->p2p) {
+    cudaSetDevice(D->h->device);
+    cudaDeviceSynchronize();
+    for (P2PPeer* p : {&D->lo, &D->hi})
+      for (void* b : p->bases) cudaIpcCloseMemHandle(b);
+    if (D->flags) cudaFree(D->flags);
+  }
 #ifdef CST_HAVE_NCCL
   if (D->comm) ncclCommDestroy(D->comm);
 #endif
@@ -128,6 +167,181 @@ extern "C" void cst_dist_destroy(cst_dist* D) {
   if (D->ev_bnd) cudaEventDestroy(D->ev_bnd);
   if (D->ev_comm) cudaEventDestroy(D->ev_comm);
   delete D;
+}
+
+// ---------------------------------------------------------------- peer-memory transport
+namespace {
+struct P2PBlob {
+  uint64_t magic;
+  int32_t nio, rank, nranks, device;
+  cudaIpcMemHandle_t buf[2][CST_MAX_IN];
+  int64_t off[2][CST_MAX_IN];
+  cudaIpcMemHandle_t flags;
+  int64_t flags_off;
+};
+static_assert(sizeof(P2PBlob) <= CST_P2P_BLOB_BYTES, "blob size");
+const uint64_t kBlobMagic = 0x43535450325031ULL;  // "CSTP2P1"
+
+cst_status ipc_handle(const void* p, cudaIpcMemHandle_t* hd, int64_t* off) {
+  const Driver* d = nullptr;
+  cst_status st = driver(&d);
+  if (st != CST_OK) return st;
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  st = cu_check(d->cuMemGetAddressRange(&base, &size, (CUdeviceptr)p), "cuMemGetAddressRange");
+  if (st != CST_OK) return st;
+  CST_CUDA(cudaIpcGetMemHandle(hd, (void*)base));
+  *off = (int64_t)((CUdeviceptr)p - base);
+  return CST_OK;
+}
+}  // namespace
+
+extern "C" cst_status cst_dist_p2p_export(cst_dist* D, double* const* buf_a,
+                                          double* const* buf_b, void* blob) {
+  if (!D || !buf_a || !buf_b || !blob) return fail(CST_E_INVALID, "null argument");
+  if (!D->p2p) return fail(CST_E_INVALID, "handle was created for NCCL (nccl_unique_id given)");
+  CST_CUDA(cudaSetDevice(D->h->device));
+  const int nio = D->h->desc.n_inputs;
+  P2PBlob b;
+  std::memset(&b, 0, sizeof b);
+  b.magic = kBlobMagic;
+  b.nio = nio;
+  b.rank = D->rank;
+  b.nranks = D->nranks;
+  b.device = D->h->device;
+  for (int a = 0; a < nio; ++a) {
+    if (!buf_a[a] || !buf_b[a]) return fail(CST_E_INVALID, "null buffer");
+    cst_status st = ipc_handle(buf_a[a], &b.buf[0][a], &b.off[0][a]);
+    if (st == CST_OK) st = ipc_handle(buf_b[a], &b.buf[1][a], &b.off[1][a]);
+    if (st != CST_OK) return st;
+    D->mine[0][a] = buf_a[a];
+    D->mine[1][a] = buf_b[a];
+  }
+  cst_status st = ipc_handle(D->flags, &b.flags, &b.flags_off);
+  if (st != CST_OK) return st;
+  std::memset(blob, 0, CST_P2P_BLOB_BYTES);
+  std::memcpy(blob, &b, sizeof b);
+  D->exported = true;
+  return CST_OK;
+}
+
+extern "C" cst_status cst_dist_p2p_import(cst_dist* D, int32_t peer, const void* blob) {
+  if (!D || !blob) return fail(CST_E_INVALID, "null argument");
+  if (!D->p2p) return fail(CST_E_INVALID, "handle was created for NCCL (nccl_unique_id given)");
+  if (peer != D->rank - 1 && peer != D->rank + 1)
+    return fail(CST_E_INVALID, "p2p peers are rank - 1 and rank + 1");
+  if (peer < 0 || peer >= D->nranks) return fail(CST_E_INVALID, "peer out of range");
+  P2PBlob b;
+  std::memcpy(&b, blob, sizeof b);
+  if (b.magic != kBlobMagic || b.nio != D->h->desc.n_inputs || b.rank != peer ||
+      b.nranks != D->nranks)
+    return fail(CST_E_INVALID, "p2p blob does not belong to this decomposition / peer");
+  CST_CUDA(cudaSetDevice(D->h->device));
+  P2PPeer& P = peer < D->rank ? D->lo : D->hi;
+  for (void* base : P.bases) cudaIpcCloseMemHandle(base);
+  P = P2PPeer();
+  auto open = [&](const cudaIpcMemHandle_t& hd, int64_t off, void** out) -> cst_status {
+    void* base = nullptr;
+    // one mapping per allocation: buffers that share one (e.g. a caching allocator's
+    // block) come back as the same base pointer
+    CST_CUDA(cudaIpcOpenMemHandle(&base, hd, cudaIpcMemLazyEnablePeerAccess));
+    P.bases.push_back(base);
+    *out = (char*)base + off;
+    return CST_OK;
+  };
+  for (int a = 0; a < b.nio; ++a)
+    for (int r = 0; r < 2; ++r) {
+      void* p = nullptr;
+      cst_status st = open(b.buf[r][a], b.off[r][a], &p);
+      if (st != CST_OK) return st;
+      P.buf[r][a] = (double*)p;
+    }
+  void* f = nullptr;
+  cst_status st = open(b.flags, b.flags_off, &f);
+  if (st != CST_OK) return st;
+  P.flags = (unsigned long long*)f;
+  P.open = true;
+  return CST_OK;
+}
+
+static cst_status dist_sweep_p2p(cst_dist* D, const cst_setting* s, const double* const* in,
+                                 double* const* out, int32_t nsteps, cudaStream_t sc) {
+  cst_stencil* h = D->h;
+  const cst_grid& G = h->grid;
+  const int r = h->desc.order;
+  const int nio = h->desc.n_inputs;
+  const bool has_lo = D->rank > 0, has_hi = D->rank < D->nranks - 1;
+  if (!D->exported || (has_lo && !D->lo.open) || (has_hi && !D->hi.open))
+    return fail(CST_E_INVALID, "p2p transport: export my buffers and import both neighbours first");
+  // which registered buffer set is in[]: role 0 = a, 1 = b
+  int role = -1;
+  for (int c = 0; c < 2 && role < 0; ++c) {
+    bool ok = true;
+    for (int a = 0; a < nio; ++a)
+      ok = ok && in[a] == D->mine[c][a] && out[a] == D->mine[1 - c][a];
+    if (ok) role = c;
+  }
+  if (role < 0)
+    return fail(CST_E_INVALID, "p2p transport: in/out must be the exported buffer sets (a, b)");
+  const int64_t pz = G.pitch_x * G.pitch_y;
+  const int64_t origin0 = ((int64_t)G.halo * G.pitch_y + G.halo) * G.pitch_x + G.lead_x;
+  const double* cin[CST_MAX_IN];
+  double* cout[CST_MAX_OUT];
+  for (int a = 0; a < nio; ++a) {
+    cin[a] = in[a];
+    cout[a] = out[a];
+  }
+  h->last_launches = 0;
+  int64_t extra = 0;  // signal / wait kernels
+  for (int step = 0; step < nsteps; ++step) {
+    const int orole = 1 - role;  // role of this step's output buffers
+    const unsigned long long e = ++D->epoch;
+    // WAR: both neighbours finished step e-1 (they read the buffers my stores target)
+    cst_status st = p2p_wait(sc, has_lo ? D->flags + F_DONE_LO : nullptr, e - 1,
+                             has_hi ? D->flags + F_DONE_HI : nullptr, e - 1);
+    if (st != CST_OK) return st;
+    ++extra;
+    // boundary planes: local stores + the same values into the neighbours' halos
+    double* rlo[CST_MAX_OUT];
+    double* rhi[CST_MAX_OUT];
+    for (int a = 0; a < nio; ++a) {
+      rlo[a] = has_lo ? D->lo.buf[orole][a] + origin0 + G.nz * pz : nullptr;
+      rhi[a] = has_hi ? D->hi.buf[orole][a] + origin0 - (int64_t)r * pz : nullptr;
+    }
+    st = cst_launch_range(h, s, cin, cout, 0, r, sc, has_lo ? rlo : nullptr);
+    if (st != CST_OK) return st;
+    if (G.nz > r) {
+      st = cst_launch_range(h, s, cin, cout, G.nz - r, r, sc, has_hi ? rhi : nullptr);
+      if (st != CST_OK) return st;
+    }
+    // my boundary stores are in the neighbours' halos: lower neighbour's BND_HI, upper's BND_LO
+    st = p2p_signal(sc, has_lo ? D->lo.flags + F_BND_HI : nullptr,
+                    has_hi ? D->hi.flags + F_BND_LO : nullptr, e);
+    if (st != CST_OK) return st;
+    ++extra;
+    if (G.nz > 2 * r) {
+      st = cst_launch_range(h, s, cin, cout, r, G.nz - 2 * r, sc);
+      if (st != CST_OK) return st;
+    }
+    st = p2p_signal(sc, has_lo ? D->lo.flags + F_DONE_HI : nullptr,
+                    has_hi ? D->hi.flags + F_DONE_LO : nullptr, e);
+    if (st != CST_OK) return st;
+    // RAW: the neighbours' boundary stores of this step are in my output halo
+    st = p2p_wait(sc, has_lo ? D->flags + F_BND_LO : nullptr, e,
+                  has_hi ? D->flags + F_BND_HI : nullptr, e);
+    if (st != CST_OK) return st;
+    extra += 2;
+    if (nsteps > 1) {
+      for (int a = 0; a < nio; ++a) {
+        const double* t = cin[a];
+        cin[a] = cout[a];
+        cout[a] = const_cast<double*>(t);
+      }
+      role = 1 - role;
+    }
+  }
+  h->last_launches += extra;
+  return CST_OK;
 }
 
 extern "C" cst_status cst_dist_sweep(cst_dist* D, const cst_setting* s, const double* const* in,
@@ -154,11 +368,14 @@ extern "C" cst_status cst_dist_sweep(cst_dist* D, const cst_setting* s, const do
   if (s->bt > 1)
     return fail(CST_E_UNSUPPORTED, "temporal blocking (bt > 1) needs bt*order halo planes; "
                                    "cst_dist_sweep exchanges order planes per step");
-  if (nsteps > 1)  // boundary condition of every step = in[]'s halo (as cst_sweep)
+  if (nsteps > 1)  // boundary condition of every step = in[]'s halo (as cst_sweep); the
+                   // z-halo planes facing a neighbour are the exchange's (never copied: with
+                   // the peer transport the neighbour may already be storing into them)
     for (int a = 0; a < nio; ++a) {
-      st = copy_halo(G, in[a], out[a], sc);
+      st = copy_halo(G, in[a], out[a], sc, D->rank == 0, D->rank == D->nranks - 1);
       if (st != CST_OK) return st;
     }
+  if (D->p2p) return dist_sweep_p2p(D, s, in, out, nsteps, sc);
   h->last_launches = 0;  // cst_launch_range counts every launch
   for (int step = 0; step < nsteps; ++step) {
     // 1. boundary planes first
@@ -241,7 +458,8 @@ extern "C" cst_status cst_dist_sweep_loopback(cst_stencil* h, int32_t nslabs, co
   }
   if (s->bt > 1) st = fail(CST_E_UNSUPPORTED, "temporal blocking (bt > 1) is not supported by z-slab sweeps");
   if (nsteps > 1)  // boundary condition of every step = in[]'s halo (as cst_sweep)
-    for (int i = 0; i < nslabs * nio && st == CST_OK; ++i) st = copy_halo(G, in_slabs[i], out_slabs[i], sc);
+    for (int i = 0; i < nslabs * nio && st == CST_OK; ++i)
+      st = copy_halo(G, in_slabs[i], out_slabs[i], sc, i / nio == 0, i / nio == nslabs - 1);
   h->last_launches = 0;  // cst_launch_range counts every launch
   for (int step = 0; step < nsteps && st == CST_OK; ++step) {
     for (int k = 0; k < nslabs && st == CST_OK; ++k) {

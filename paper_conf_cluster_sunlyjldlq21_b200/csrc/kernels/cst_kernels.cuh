@@ -68,6 +68,15 @@ struct Ctx {
   }
 };
 
+// Store one interior output value.  In a z-slab boundary launch of the fused halo
+// exchange the same value is also stored into the neighbour rank's
+// halo through its peer-mapped buffer (NVLink / NVSwitch): rout[q] is offset so that the
+// launch's own element offset addresses the neighbour's matching halo element.
+__device__ __forceinline__ void put(const cst_kparams& P, int q, long long off, double v) {
+  P.out[q][off] = v;
+  if (P.remote) P.rout[q][off] = v;
+}
+
 __device__ __forceinline__ int merged_pos(int i, int t, int TBd, int BMd) {
   // i-th point (0 <= i < BM*CM) of thread t along one dim (block + cyclic merging)
   return (i / BMd) * (TBd * BMd) + t * BMd + (i % BMd);
@@ -352,7 +361,7 @@ __device__ __forceinline__ void kernel_tile3d(const cst_kparams& P, double* smem
         }
         const long long off = x + y * P.py + z * P.pz;
 #pragma unroll
-        for (int q = 0; q < NOUT; ++q) P.out[q][off] = o[q];
+        for (int q = 0; q < NOUT; ++q) put(P, q, off, o[q]);
       }
     }
   }
@@ -744,7 +753,11 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
   };
   auto store = [&](int ib, int ia, int po, double v) {
     if (g.a0 + la[ia] < g.n_a && g.b0 + lb[ib] < g.n_b)
-      out[col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)po * g.st_s] = v;
+    {
+      const long long off = col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)po * g.st_s;
+      out[off] = v;
+      if (P.remote) P.rout[0][off] = v;
+    }
   };
 
 #pragma unroll(UFS)
@@ -1110,7 +1123,7 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
     if (g.a0 + la[ia] < g.n_a && g.b0 + lb[ib] < g.n_b) {
       const long long off = col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)po * g.st_s;
 #pragma unroll
-      for (int f = 0; f < 5; ++f) P.out[f][off] = v[f];
+      for (int f = 0; f < 5; ++f) put(P, f, off, v[f]);
     }
   };
 
@@ -1347,7 +1360,7 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
             point(C, U, o);
           }
 #pragma unroll
-          for (int q = 0; q < NOUT; ++q) P.out[q][off] = o[q];
+          for (int q = 0; q < NOUT; ++q) put(P, q, off, o[q]);
         }
       }
     }
@@ -1537,7 +1550,7 @@ __device__ __forceinline__ void tb_stage(const Ctx& C, const cst_kparams& P, con
           dst[(ey0 + ib) * WA + ex0 + ia] = val;
         } else {
           if (o >= g.s_start && o < g.s_end && gx < P.nx && gy < P.ny)
-            P.out[0][gx + (long long)gy * P.py + (long long)o * P.pz] = val;
+            put(P, 0, gx + (long long)gy * P.py + (long long)o * P.pz, val);
         }
       }
   }

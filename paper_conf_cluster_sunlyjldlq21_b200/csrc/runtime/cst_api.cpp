@@ -55,7 +55,8 @@ cst_status driver(const Driver** out) {
               get("cuLaunchKernel", (void**)&d.cuLaunchKernel) &&
               get("cuTensorMapEncodeTiled", (void**)&d.cuTensorMapEncodeTiled) &&
               get("cuOccupancyMaxActiveBlocksPerMultiprocessor", (void**)&d.cuOccupancy) &&
-              get("cuGetErrorString", (void**)&d.cuGetErrorString);
+              get("cuGetErrorString", (void**)&d.cuGetErrorString) &&
+              get("cuMemGetAddressRange", (void**)&d.cuMemGetAddressRange);
     if (!ok) {
       st = CST_E_CUDA;
       err = "cudaGetDriverEntryPoint failed for a required driver function";
@@ -443,7 +444,8 @@ static cst_status tmap_for(cst_stencil* h, const double* base, const int box[3],
 
 // Launch one sweep of planes [z0, z0 + nz) (local interior z) of the handle's grid.
 cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* const* in,
-                            double* const* out, int64_t z0, int64_t nzr, cudaStream_t stream) {
+                            double* const* out, int64_t z0, int64_t nzr, cudaStream_t stream,
+                            double* const* rout) {
   Variant* v = nullptr;
   cst_status st = get_variant(h, s, &v);
   if (st != CST_OK) return st;
@@ -468,6 +470,10 @@ cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* 
     }
   }
   for (int o = 0; o < nout; ++o) P.out[o] = out[o] + origin;
+  if (rout) {
+    P.remote = 1;
+    for (int o = 0; o < nout; ++o) P.rout[o] = rout[o];
+  }
   for (size_t i = 0; i < h->kcoef.size() && i < CST_MAX_COEF; ++i) P.coef[i] = h->kcoef[i];
   P.py = G.pitch_x;
   P.pz = G.pitch_x * G.pitch_y;

@@ -29,12 +29,14 @@ __global__ void fill_kernel(double* __restrict__ dst, int64_t nx, int64_t ny, in
 // copied whole, interior rows only their 2*halo x-halo elements
 __global__ void copy_halo_kernel(const double* __restrict__ src, double* __restrict__ dst,
                                  int64_t nx, int64_t ny, int64_t nz, int64_t halo,
-                                 int64_t lead_x, int64_t pitch_x, int64_t pitch_y) {
+                                 int64_t lead_x, int64_t pitch_x, int64_t pitch_y, int zlo,
+                                 int zhi) {
   const int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32;
   const int lane = threadIdx.x % 32;
   const int64_t rows_y = ny + 2 * halo;
   if (row >= rows_y * (nz + 2 * halo)) return;
   const int64_t y = row % rows_y - halo, z = row / rows_y - halo;
+  if ((z < 0 && !zlo) || (z >= nz && !zhi)) return;
   const int64_t base = ((z + halo) * pitch_y + (y + halo)) * pitch_x + lead_x;
   if (y < 0 || y >= ny || z < 0 || z >= nz) {
     for (int64_t x = lane - halo; x < nx + halo; x += 32) dst[base + x] = src[base + x];
@@ -48,13 +50,15 @@ __global__ void copy_halo_kernel(const double* __restrict__ src, double* __restr
 
 namespace cst {
 // Copy the logical halo of one array (the multi-step boundary condition) from src to dst.
-cst_status copy_halo(const cst_grid& g, const double* src, double* dst, cudaStream_t stream) {
+cst_status copy_halo(const cst_grid& g, const double* src, double* dst, cudaStream_t stream,
+                     bool zlo, bool zhi) {
   const int64_t rows = (g.nz + 2 * (int64_t)g.halo) * (g.ny + 2 * (int64_t)g.halo);
   if (g.halo > 16) return fail(CST_E_UNSUPPORTED, "copy_halo: halo > 16");
   const int64_t blocks = (rows * 32 + 255) / 256;
   if (blocks > 0x7fffffffLL) return fail(CST_E_UNSUPPORTED, "grid too large for copy_halo");
   copy_halo_kernel<<<(unsigned)blocks, 256, 0, stream>>>(src, dst, g.nx, g.ny, g.nz, g.halo,
-                                                         g.lead_x, g.pitch_x, g.pitch_y);
+                                                         g.lead_x, g.pitch_x, g.pitch_y,
+                                                         zlo ? 1 : 0, zhi ? 1 : 0);
   CST_CUDA(cudaGetLastError());
   return CST_OK;
 }

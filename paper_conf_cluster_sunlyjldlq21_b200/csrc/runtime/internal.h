@@ -80,7 +80,18 @@ class Space {
 
 // Copy the logical halo of one array (fill.cu).  Multi-step sweeps use in[]'s halo as the
 // boundary condition of every step.
-cst_status copy_halo(const cst_grid& g, const double* src, double* dst, cudaStream_t stream);
+// zlo / zhi: include the z-halo planes below / above (false where a z-slab neighbour owns
+// them).
+cst_status copy_halo(const cst_grid& g, const double* src, double* dst, cudaStream_t stream,
+                     bool zlo = true, bool zhi = true);
+
+// Peer-memory halo transport (dist/p2p.cu): signal = after the stream's prior work, store
+// `value` (release, system scope) into every non-null flag word; wait = block the stream
+// until every non-null flag word >= its target (acquire, 30 s bound, then trap).
+cst_status p2p_signal(cudaStream_t s, unsigned long long* f0, unsigned long long* f1,
+                      unsigned long long value);
+cst_status p2p_wait(cudaStream_t s, const unsigned long long* f0, unsigned long long t0,
+                    const unsigned long long* f1, unsigned long long t1);
 
 // Temporal-blocking pass schedule: step counts per kernel pass (powers of two <= bt)
 // summing to nsteps, with as many passes as nsteps has parity (ping-pong placement).
@@ -98,6 +109,7 @@ struct Driver {
   PFN_cuTensorMapEncodeTiled_v12000 cuTensorMapEncodeTiled = nullptr;
   PFN_cuOccupancyMaxActiveBlocksPerMultiprocessor_v6050 cuOccupancy = nullptr;
   PFN_cuGetErrorString_v6000 cuGetErrorString = nullptr;
+  PFN_cuMemGetAddressRange_v3020 cuMemGetAddressRange = nullptr;
 };
 cst_status driver(const Driver** out);
 cst_status cu_check(CUresult r, const char* what);
@@ -122,9 +134,12 @@ std::string nvrtc_description();
 
 }  // namespace cst
 
-// Launch one sweep of local interior planes [z0, z0 + nz) (sub-domain sweeps).
+// Launch one sweep of local interior planes [z0, z0 + nz) (sub-domain sweeps).  rout
+// (optional, one per output): every stored value also goes to rout[q] + (element offset
+// of the point relative to element (0, 0, z0) of out[q]) — the fused halo exchange.
 cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* const* in,
-                            double* const* out, int64_t z0, int64_t nz, cudaStream_t stream);
+                            double* const* out, int64_t z0, int64_t nz, cudaStream_t stream,
+                            double* const* rout = nullptr);
 
 namespace cst {
 

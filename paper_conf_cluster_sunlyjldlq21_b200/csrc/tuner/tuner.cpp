@@ -959,7 +959,7 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
           fs.resize(o->top_n);
           if (cv(fs) < o->cv_threshold) break;
         }
-        if (o->time_budget_s > 0 && elapsed() > o->time_budget_s) break;
+        if (o->time_budget_s > 0 && elapsed() - t_dataset > o->time_budget_s) break;
       }
       if (gens > o->max_generations) gens = o->max_generations;
     }
@@ -973,7 +973,7 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
     js.o << (g ? "," : "") << "{\"group\":" << g << ",\"table\":" << tab.size()
          << ",\"exhaustive\":" << (exhaustive ? "true" : "false") << ",\"generations\":" << gens
          << ",\"evaluated\":" << phase.size() << ",\"best_ms\":" << Json::num(cur_ms) << "}";
-    if (o->time_budget_s > 0 && elapsed() > o->time_budget_s) break;
+    if (o->time_budget_s > 0 && elapsed() - t_dataset > o->time_budget_s) break;
   }
   js.o << "]";
   *best_out = from_tuple(ev.effective(cur));

@@ -186,6 +186,9 @@ _decl("cst_dist_sweep", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP, ctypes.c_
 _decl("cst_dist_sweep_loopback", _S, _P, ctypes.c_int32, ctypes.POINTER(cst_setting), _PP, _PP,
       ctypes.c_int32, _P)
 _decl("cst_dist_destroy", None, _P)
+_decl("cst_dist_p2p_export", _S, _P, _PP, _PP, _P)
+_decl("cst_dist_p2p_import", _S, _P, ctypes.c_int32, _P)
+P2P_BLOB_BYTES = 2048
 
 EXPORTS = [n for n in dir(_lib) if n.startswith("cst_")]
 
@@ -400,3 +403,29 @@ def cst_dist_sweep_loopback(h, nslabs: int, s: cst_setting, in_ptrs, out_ptrs, n
 
 def cst_dist_destroy(d) -> None:
     _lib.cst_dist_destroy(d)
+
+
+def cst_dist_p2p_export(d, a_ptrs, b_ptrs) -> bytes:
+    """IPC description of my ping-pong buffer sets (a, b) and flag words (peer transport)."""
+    pa, _a = _ptrs(a_ptrs)
+    pb, _b = _ptrs(b_ptrs)
+    blob = ctypes.create_string_buffer(P2P_BLOB_BYTES)
+    check(_lib.cst_dist_p2p_export(d, pa, pb, blob))
+    return blob.raw
+
+
+def cst_dist_p2p_import(d, peer: int, blob: bytes) -> None:
+    buf = ctypes.create_string_buffer(bytes(blob), P2P_BLOB_BYTES)
+    check(_lib.cst_dist_p2p_import(d, peer, buf))
+
+
+def cst_dist_p2p_setup(d, rank: int, world: int, a_ptrs, b_ptrs, group=None) -> None:
+    """Export my buffers, all-gather the blobs over torch.distributed (any backend), import
+    both neighbours: the fused peer-memory halo transport is then ready."""
+    import torch.distributed as dist
+    mine = cst_dist_p2p_export(d, a_ptrs, b_ptrs)
+    blobs = [None] * world
+    dist.all_gather_object(blobs, mine, group=group)
+    for peer in (rank - 1, rank + 1):
+        if 0 <= peer < world:
+            cst_dist_p2p_import(d, peer, blobs[peer])

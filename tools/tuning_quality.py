@@ -82,16 +82,21 @@ def _compile(h, s):
         pass
 
 
-def run_cstuner(h, u, v, seed, budget, ratio=0.10, tag=""):
+def run_cstuner(h, u, v, seed, budget, ratio=0.10, tag="", warm_start=1):
     o = C.cst_tune_opts_default()
     o.seed = seed
     o.time_budget_s = budget
     o.sampling_ratio = ratio
+    o.warm_start = warm_start
     log = f"/tmp/tq_{tag}_{seed}_{ratio}.json"
     o.log_path = log.encode()
     best, rep = C.cst_tune(h, o, [u.data_ptr()], [v.data_ptr()])
     j = json.load(open(log))
-    return {"seed": seed, "budget_s": budget, "sampling_ratio": ratio, "best_ms": rep.best_ms,
+    ds = j.get("report", {}).get("dataset_s", 0.0)
+    # iso-time axis = online search time: the dataset (metric collection) is offline
+    search_trace = [[t - ds, ms, n] for t, ms, n in j.get("trace", [])]
+    return {"seed": seed, "budget_s": budget, "sampling_ratio": ratio, "warm_start": warm_start,
+            "dataset_s": ds, "search_trace": search_trace, "best_ms": rep.best_ms,
             "best_setting": best.as_dict(), "evaluations": rep.evaluations,
             "wall_s": rep.wall_s, "eval_s": rep.eval_s, "jit_s": rep.jit_s,
             "preproc_s": rep.preproc_s, "sampled_count": rep.sampled_count,
@@ -141,7 +146,14 @@ def main():
     # 2. iso-time: csTuner vs random search
     res["cstuner"] = [run_cstuner(h, u, v, s + 1, args.budget, tag="iso") for s in range(args.seeds)]
     for r in res["cstuner"]:
-        print(json.dumps({k: r[k] for k in ("seed", "best_ms", "evaluations", "wall_s")}), flush=True)
+        print(json.dumps({k: r[k] for k in ("seed", "best_ms", "evaluations", "wall_s",
+                                            "dataset_s")}), flush=True)
+    # the paper's method as published: the dataset is a pure random sample (no warm start)
+    res["cstuner_no_warm_start"] = [run_cstuner(h, u, v, s + 1, args.budget, tag="cold",
+                                                warm_start=0) for s in range(args.seeds)]
+    for r in res["cstuner_no_warm_start"]:
+        print(json.dumps({k: r[k] for k in ("seed", "best_ms", "evaluations", "wall_s",
+                                            "dataset_s")}), flush=True)
     res["random_search"] = [run_random(h, u, v, s + 1, args.budget) for s in range(args.seeds)]
     for r in res["random_search"]:
         print(json.dumps({k: r[k] for k in ("seed", "best_ms", "evaluations")}), flush=True)
