@@ -25,6 +25,9 @@
 #ifndef CST_HYP_SCALAR
 #define CST_HYP_SCALAR 0
 #endif
+#ifndef CST_REMOTE
+#define CST_REMOTE 0  // 1: fused-halo twin (z-slab boundary launches, NEXT-3)
+#endif
 
 // ------------------------------------------------------------------ configuration
 constexpr int KIND = CST_KIND;  // 1 star, 2 box, 3 hypterm, 4 rhs4center-like
@@ -71,10 +74,11 @@ struct Ctx {
 // Store one interior output value.  In a z-slab boundary launch of the fused halo
 // exchange the same value is also stored into the neighbour rank's
 // halo through its peer-mapped buffer (NVLink / NVSwitch): rout[q] is offset so that the
-// launch's own element offset addresses the neighbour's matching halo element.
+// launch's own element offset addresses the neighbour's matching halo element.  A
+// compile-time twin (CST_REMOTE): the plain variant carries no trace of it.
 __device__ __forceinline__ void put(const cst_kparams& P, int q, long long off, double v) {
   P.out[q][off] = v;
-  if (P.remote) P.rout[q][off] = v;
+  if constexpr (CST_REMOTE) P.rout[q][off] = v;
 }
 
 __device__ __forceinline__ int merged_pos(int i, int t, int TBd, int BMd) {
@@ -756,7 +760,7 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
     {
       const long long off = col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)po * g.st_s;
       out[off] = v;
-      if (P.remote) P.rout[0][off] = v;
+      if constexpr (CST_REMOTE) P.rout[0][off] = v;
     }
   };
 

@@ -312,10 +312,11 @@ extern "C" cst_status cst_space_rank(cst_stencil* h, const cst_setting* s, uint6
 }
 
 // ====================================================================== variants
-static cst_status get_variant(cst_stencil* h, const cst_setting* s, Variant** out) {
+static cst_status get_variant(cst_stencil* h, const cst_setting* s, Variant** out,
+                              bool remote = false) {
   const char* rule = check_rules(h->info, to_tuple(*s));
   if (rule) return fail(CST_E_CONSTRAINT, std::string("setting violates ") + rule);
-  const std::string key = setting_key(*s);
+  const std::string key = setting_key(*s) + (remote ? ",remote" : "");
   auto it = h->variants.find(key);
   if (it != h->variants.end()) {
     if (!it->second.fn)
@@ -337,7 +338,7 @@ static cst_status get_variant(cst_stencil* h, const cst_setting* s, Variant** ou
                                       " B exceeds 227 KiB");
   }
   std::string cubin;
-  st = jit_cubin(h->info, t, &cubin, &v.compile_s);
+  st = jit_cubin(h->info, t, &cubin, &v.compile_s, remote);
   if (st != CST_OK) return st;
   st = cu_check(d->cuModuleLoadData(&v.mod, cubin.data()), "cuModuleLoadData");
   if (st != CST_OK) return st;
@@ -447,7 +448,7 @@ cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* 
                             double* const* out, int64_t z0, int64_t nzr, cudaStream_t stream,
                             double* const* rout) {
   Variant* v = nullptr;
-  cst_status st = get_variant(h, s, &v);
+  cst_status st = get_variant(h, s, &v, rout != nullptr);
   if (st != CST_OK) return st;
   const Driver* d = nullptr;
   st = driver(&d);
@@ -470,7 +471,7 @@ cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* 
     }
   }
   for (int o = 0; o < nout; ++o) P.out[o] = out[o] + origin;
-  if (rout) {
+  if (rout) {  // the CST_REMOTE twin of the variant reads these
     P.remote = 1;
     for (int o = 0; o < nout; ++o) P.rout[o] = rout[o];
   }

@@ -126,9 +126,11 @@ struct Variant {
   double compile_s = 0;
   bool coef_uploaded = false;
 };
-// Compile (or fetch from the memory/disk cache) the cubin of a variant.
+// Compile (or fetch from the memory/disk cache) the cubin of a variant; remote = the
+// fused-halo twin whose stores also go to the neighbour's halo (CST_REMOTE).
 cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
-                     double* compile_s);
+                     double* compile_s,
+                     bool remote = false);
 uint64_t jit_compile_count();
 std::string nvrtc_description();
 

@@ -117,9 +117,10 @@ std::string nvrtc_description() {
   return "nvrtc " + std::to_string(N->major) + "." + std::to_string(N->minor) + " (" + N->path + ")";
 }
 
-static std::string prefix_for(const StencilInfo& st, const Tuple& t) {
+static std::string prefix_for(const StencilInfo& st, const Tuple& t, bool remote) {
   std::ostringstream o;
   o << "#define CST_KIND " << st.kind << "\n#define CST_R " << st.r << "\n";
+  if (remote) o << "#define CST_REMOTE 1\n";
   static const char* names[F_COUNT] = {"TBX", "TBY", "TBZ", "STAGING", "CONST", "STREAM",
                                        "SD",  "SB",  "UFX", "UFY",     "UFZ",   "CMX",
                                        "CMY", "CMZ", "BMX", "BMY",     "BMZ",   "RET",
@@ -130,8 +131,8 @@ static std::string prefix_for(const StencilInfo& st, const Tuple& t) {
 }
 
 cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
-                     double* compile_s) {
-  const std::string src = prefix_for(st, t);
+                     double* compile_s, bool remote) {
+  const std::string src = prefix_for(st, t, remote);
   std::vector<std::string> optv = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo",
                                    "--fmad=true", "-default-device", "-DCST_NVRTC=1"};
   // experiment hook: extra -D options (e.g. "-DCST_EMPTY_BARRIERS=1"), part of the cache key
