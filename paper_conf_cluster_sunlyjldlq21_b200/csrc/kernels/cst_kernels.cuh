@@ -205,8 +205,24 @@ __device__ __forceinline__ void hypterm_point(const Ctx& C, const Acc& U, double
 // with the constant factors folded (host-precomputed in the coefficient bank):
 // kcoef[3 + d] = s_d^2 / 6 scales the unscaled V sum, kcoef[6 + pair(d, i)] = s_d s_i / 144
 // scales the unscaled outer(inner) difference of each mixed term.
-template <class Acc>
-__device__ __forceinline__ void rhs4_point(const Ctx& C, const Acc& U, double* r) {
+// Two x-adjacent points evaluated in lockstep (the paired rhs4 path): the same operations
+// in the same order per lane as the scalar code.
+struct dpair {
+  double x, y;
+};
+__device__ __forceinline__ dpair operator+(dpair a, dpair b) { return {a.x + b.x, a.y + b.y}; }
+__device__ __forceinline__ dpair operator-(dpair a, dpair b) { return {a.x - b.x, a.y - b.y}; }
+__device__ __forceinline__ dpair operator*(dpair a, dpair b) { return {a.x * b.x, a.y * b.y}; }
+__device__ __forceinline__ dpair operator*(double a, dpair b) { return {a * b.x, a * b.y}; }
+__device__ __forceinline__ dpair fma(double a, dpair b, dpair c) {
+  return {fma(a, b.x, c.x), fma(a, b.y, c.y)};
+}
+__device__ __forceinline__ dpair fma(dpair a, dpair b, dpair c) {
+  return {fma(a.x, b.x, c.x), fma(a.y, b.y, c.y)};
+}
+
+template <class T, class Acc>
+__device__ __forceinline__ void rhs4_point_t(const Ctx& C, const Acc& U, T* r) {
   auto at = [&](int arr, int d, int k, int d2, int k2) {
     int o[3] = {0, 0, 0};
     o[d] += k;
@@ -215,21 +231,21 @@ __device__ __forceinline__ void rhs4_point(const Ctx& C, const Acc& U, double* r
   };
 #pragma unroll
   for (int i = 0; i < 3; ++i) {
-    double acc = 0.0;
+    T acc{};
 #pragma unroll
     for (int d = 0; d < 3; ++d) {
       auto a = [&](int k) {
-        const double m = at(3, d, k, d, 0);
+        const T m = at(3, d, k, d, 0);
         return d == i ? fma(2.0, m, at(4, d, k, d, 0)) : m;
       };
       auto f = [&](int k) { return at(i, d, k, d, 0); };
-      const double am2 = a(-2), am1 = a(-1), a0 = a(0), ap1 = a(1), ap2 = a(2);
-      const double m1 = fma(-0.75, a0 + am2, am1);
-      const double m2 = fma(3.0, a0 + am1, am2 + ap1);
-      const double m3 = fma(3.0, ap1 + a0, am1 + ap2);
-      const double m4 = fma(-0.75, a0 + ap2, ap1);
-      const double f0 = f(0);
-      double v = m1 * (f(-2) - f0);
+      const T am2 = a(-2), am1 = a(-1), a0 = a(0), ap1 = a(1), ap2 = a(2);
+      const T m1 = fma(-0.75, a0 + am2, am1);
+      const T m2 = fma(3.0, a0 + am1, am2 + ap1);
+      const T m3 = fma(3.0, ap1 + a0, am1 + ap2);
+      const T m4 = fma(-0.75, a0 + ap2, ap1);
+      const T f0 = f(0);
+      T v = m1 * (f(-2) - f0);
       v = fma(m2, f(-1) - f0, v);
       v = fma(m3, f(1) - f0, v);
       v = fma(m4, f(2) - f0, v);
@@ -240,7 +256,7 @@ __device__ __forceinline__ void rhs4_point(const Ctx& C, const Acc& U, double* r
       if (d == i) continue;
       auto mixed = [&](int outer, int inner, int coef, int comp) {
         auto inner_d = [&](int ko) {
-          const double g = fma(8.0, at(comp, outer, ko, inner, 1) - at(comp, outer, ko, inner, -1),
+          const T g = fma(8.0, at(comp, outer, ko, inner, 1) - at(comp, outer, ko, inner, -1),
                                at(comp, outer, ko, inner, -2) - at(comp, outer, ko, inner, 2));
           return at(coef, outer, ko, outer, 0) * g;
         };
@@ -252,6 +268,11 @@ __device__ __forceinline__ void rhs4_point(const Ctx& C, const Acc& U, double* r
     }
     r[i] = acc;
   }
+}
+
+template <class Acc>
+__device__ __forceinline__ void rhs4_point(const Ctx& C, const Acc& U, double* r) {
+  rhs4_point_t<double>(C, U, r);
 }
 
 template <class Acc>
@@ -447,6 +468,8 @@ struct GlobPlane {
 };
 
 constexpr int NCA = BMA * CMA, NCB = BMB * CMB;
+// rhs4 in the generic streaming path with BM_x = 2: two points per thread in lockstep
+constexpr bool PAIRED = KIND == 4 && BMA == 2 && CMA == 1 && STAGING >= 2;
 constexpr int W = 2 * R + 1;
 
 // load the x-window [la0 - XR, la0 + BMA + XR) of row lb (only [la0-R, la0+BMA+R) used)
@@ -1342,6 +1365,36 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
 #pragma unroll(UFB)
       for (int ib = 0; ib < BMB * CMB; ++ib) {
         const int lbp = merged_pos(ib, tb, TBB, BMB);
+        if constexpr (PAIRED) {
+          // rhs4, BM_x = 2: the thread's two x-adjacent points in lockstep; every smem
+          // operand is one 16-B load for both (odd x-offsets combine the two aligned
+          // neighbours, which the even offsets load anyway)
+          const int lap = merged_pos(0, ta, TBA, BMA);
+          const int a = g.a0 + lap, b = g.b0 + lbp;
+          if (a >= g.n_a || b >= g.n_b || s >= g.s_end) continue;
+          const long long off = a + b * g.st_b + (long long)s * g.st_s;
+          const int jp = s - g.s_start + R;
+          auto U2 = [&](int arr, int dx, int dy, int dz) {
+            const int db = SZ ? dy : dz, ds = SZ ? dz : dy;
+            const double* row = smem + ((jp + ds) % NP) * NIN * SLOT + arr * SLOT +
+                                (lbp + R + db) * PA + lap + XR;
+            if ((dx & 1) == 0) {
+              const double2 v = *reinterpret_cast<const double2*>(row + dx);
+              return dpair{v.x, v.y};
+            }
+            const double2 lo = *reinterpret_cast<const double2*>(row + dx - 1);
+            const double2 hi = *reinterpret_cast<const double2*>(row + dx + 1);
+            return dpair{lo.y, hi.x};
+          };
+          dpair o2[3];
+          rhs4_point_t<dpair>(C, U2, o2);
+#pragma unroll
+          for (int q = 0; q < NOUT; ++q) {
+            put(P, q, off, o2[q].x);
+            if (a + 1 < g.n_a) put(P, q, off + 1, o2[q].y);
+          }
+          continue;
+        }
 #pragma unroll(UFA)
         for (int ia = 0; ia < BMA * CMA; ++ia) {
           const int lap = merged_pos(ia, ta, TBA, BMA);

@@ -136,6 +136,28 @@ def test_config_coefficients_default_setting(kind, r):
         H.assert_parity(L, got[o], want[o], f"out{o}")
 
 
+RHS4_PAIRED = [("paired-tma", dict(tb_x=8, tb_y=8, bm_x=2)),
+               ("paired-ldst", dict(tb_x=8, tb_y=8, bm_x=2, staging=2)),
+               ("paired-bmy2", dict(tb_x=8, tb_y=4, bm_x=2, bm_y=2)),
+               ("paired-sd-y", dict(tb_x=8, tb_y=1, tb_z=8, sd=2, bm_x=2)),
+               ("scalar-bmx1", dict(tb_x=16, tb_y=8, bm_x=1))]
+
+
+@pytest.mark.parametrize("name,kw", RHS4_PAIRED, ids=[p[0] for p in RHS4_PAIRED])
+def test_rhs4_paired_points_ragged(name, kw):
+    """rhs4 with BM_x = 2: the paired (two points per 16-B operand) evaluation, odd nx so
+    the last pair of a row is half outside, poisoned far halo."""
+    kind, r = 4, 2
+    L = H.layout((37, 22, 19), r + 1)
+    c = H.coeffs(kind, r, "random", seed=9)
+    ins = H.inputs(kind, L, seed=13, poison_beyond=r)
+    _, want = H.oracle_outputs(kind, r, c, L, ins)
+    _, got = run_gpu(kind, r, c, L, ins, S(sb=8, uf_z=1, **kw))
+    for o in range(ost.N_OUT[kind]):
+        H.assert_parity(L, got[o], want[o], f"{name} out{o}")
+        H.assert_halo_untouched(L, got[o], np.full(L.numel, np.nan))
+
+
 def test_integer_polynomial_bit_exact():
     """Integer weights and integer data: FMA is exact, so GPU == oracle bit-for-bit."""
     r = 4

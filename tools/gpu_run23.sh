@@ -1,0 +1,7 @@
+#!/bin/bash
+cd "$GRAFT_REPO_ROOT" 2>/dev/null || cd /root/repo
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout -k 10 900 python -m pytest tests/test_gpu_sweep.py -m gpu -q -k "rhs4 or 4-2" --timeout 600 -p no:cacheprovider > gpurun_out/pytest_rhs4.log 2>&1
+timeout -k 10 900 python tools/explore.py --kind 4 --order 2 --n 320 320 320 --settings tools/rhs4_explore3.json --reps 5 > gpurun_out/explore_rhs4c.log 2>&1
+echo done
