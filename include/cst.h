@@ -102,6 +102,13 @@ typedef struct {
                            * optimization parameters").  Rule R14: bt > 1 needs star/box,
                            * z streaming with T_z = 1, TMA staging, retiming, CM = UF = 1,
                            * BM_x, BM_y <= 2.  Only matters for nsteps > 1 (cst_sweep). */
+  int32_t qstore;         /* where the streamed-direction state lives {1 registers, 2 tensor
+                           * memory (TMEM)}: B200 extension of retiming — a ring of R
+                           * (value, partial output) pairs per point in TMEM frees the
+                           * registers for larger register blocks.  Rule
+                           * R15: qstore = 2 needs the star, streaming with T_SD = 1, TMA
+                           * staging, retiming, bt = 1, and ceil(threads/128) * points per
+                           * thread * 4r <= 512 TMEM columns. */
 } cst_setting;
 
 typedef struct cst_stencil cst_stencil;     /* opaque: JIT modules, TMA descriptors, space */
@@ -112,13 +119,14 @@ cst_status cst_stencil_create(const cst_stencil_desc* desc, const cst_grid* grid
                               cst_stencil** out);
 void cst_stencil_destroy(cst_stencil* h);
 
-/* Rules R1-R12 (explicit, and implicit analytic resource rules).
+/* Rules R1-R12, R14, R15 (explicit, implicit analytic resource rules, P:149-151,
+ * and the structural rules of the B200 extensions).
  * CST_OK if valid, else CST_E_CONSTRAINT with the rule in cst_last_error(). */
 cst_status cst_setting_check(const cst_stencil* h, const cst_setting* s);
 /* A good default setting for the handle's stencil (valid by construction). */
 cst_status cst_setting_default(const cst_stencil* h, cst_setting* s);
 
-/* Canonical valid space: lexicographic order of the 20 fields (Table I row order, then bt;
+/* Canonical valid space: lexicographic order of the 21 fields (Table I row order, bt, qstore;
  * values ascending) restricted to valid tuples; rank = position (bit-exact with
  * oracle/space.py). */
 cst_status cst_space_count(cst_stencil* h, uint64_t* n);

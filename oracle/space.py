@@ -23,6 +23,9 @@ Space (readings Q14/Q15 of SURVEY.md §8(c)):
                                                     per pass (B200 extension, SURVEY §8(f)
                                                     NEXT-2; "more optimization parameters",
                                                     P:127 / P:419)
+  21  qstore         {1 registers, 2 TMEM}          where the streamed-direction state of the
+                                                    retimed sweep lives (B200
+                                                    extension: tensor memory)
 
 Rules: paper R1 prod TB <= 1024; R2 SD=SB=1 when streaming off; R3 UF_SD <= SB when
 streaming on.  Ours (Q15): R4 prod TB >= 32; R5 T_d = TB_d*BM_d*CM_d <= E_d (E_d = M_d,
@@ -31,7 +34,9 @@ streaming); R7 prod(BM*CM) <= 16; R8 streaming => SD != 1; R9 prefetch > 1 => st
 R10 modelled smem <= SMEM_LIMIT; R11 modelled registers <= 255; R12 TMA box: T_x even and
 every box extent <= 256; R14 bt > 1 only for the temporally blocked path: star / box,
 streaming along z with T_SD = 1, TMA staging, retimed accumulators, no cyclic merging,
-BM_x, BM_y <= 2, every UF = 1 (reading Q23).
+BM_x, BM_y <= 2, every UF = 1 (reading Q23); R15 qstore = 2 only for the
+TMEM path: star, streaming with T_SD = 1, TMA staging, retimed, bt = 1, and
+ceil(threads/128) * points per thread * 4r <= 512 TMEM columns.
 """
 from __future__ import annotations
 
@@ -39,7 +44,7 @@ import math
 
 FIELDS = ("tb_x", "tb_y", "tb_z", "staging", "use_constant", "use_streaming", "sd", "sb",
           "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z", "bm_x", "bm_y", "bm_z",
-          "use_retiming", "prefetch", "bt")
+          "use_retiming", "prefetch", "bt", "qstore")
 
 STAR, BOX, HYPTERM, RHS4 = 1, 2, 3, 4
 SMEM_LIMIT = 227 * 1024 - 1024      # data bytes; 1 KiB kept for mbarriers / alignment
@@ -123,7 +128,34 @@ def smem_bytes(kind: int, r: int, s: dict) -> int:
     return n_arrays(kind) * NP * plane
 
 
+def points_per_thread(s: dict) -> int:
+    ppt = 1
+    for d in "xyz":
+        ppt *= s["bm_" + d] * s["cm_" + d]
+    return ppt
+
+
+def tmem_columns(r: int, s: dict) -> int:
+    """TMEM columns of one CTA of the qstore = 2 path: warps are spread over the 4 lane
+    quarters (ceil(threads/128) share one), each thread keeps 4r columns per point."""
+    nthr = s["tb_x"] * s["tb_y"] * s["tb_z"]
+    return (nthr // 32 + 3) // 4 * points_per_thread(s) * 4 * r
+
+
+def qs_path_ok(kind: int, r: int, s: dict) -> bool:
+    """R15: the TMEM streamed-state path's structural and capacity requirements."""
+    if not (kind == STAR and s["use_streaming"] == 2 and s["staging"] == 3
+            and s["use_retiming"] == 2 and s["bt"] == 1):
+        return False
+    if tiles(s)[s["sd"] - 1] != 1:
+        return False
+    return tmem_columns(r, s) <= 512
+
+
 def est_regs(kind: int, r: int, s: dict) -> int:
+    if s["qstore"] == 2:
+        # in-plane part + centre per point, one point's ring, the block's column windows
+        return 32 + 2 * (2 * points_per_thread(s) + (r + 1) + 2 * r)
     if s["bt"] > 1:
         # 2r+1 rotating accumulators per point of every level + one operand window
         pts = sum(tb_blocks_per_thread(r, s, lv) for lv in range(1, s["bt"] + 1))
@@ -190,6 +222,8 @@ def check(kind: int, r: int, M, s: dict):
         return "R9"
     if s["bt"] > 1 and not tb_path_ok(kind, s):
         return "R14"
+    if s["qstore"] == 2 and not qs_path_ok(kind, r, s):
+        return "R15"
     if smem_bytes(kind, r, s) > SMEM_LIMIT:
         return "R10"
     if est_regs(kind, r, s) > REG_LIMIT:
@@ -267,13 +301,14 @@ def _inner(kind, r, M, s):
                                         for ret in (1, 2):
                                             for pf in (1, 2, 3, 4):
                                                 for bt in (1, 2, 4):
-                                                    t = dict(s, uf_x=ufx, uf_y=ufy, uf_z=ufz,
-                                                             cm_x=cmx, cm_y=cmy, cm_z=cmz,
-                                                             bm_x=bmx, bm_y=bmy, bm_z=bmz,
-                                                             use_retiming=ret, prefetch=pf,
-                                                             bt=bt)
-                                                    if check(kind, r, M, t) is None:
-                                                        found.append(t)
+                                                    for qs in (1, 2):
+                                                        t = dict(s, uf_x=ufx, uf_y=ufy, uf_z=ufz,
+                                                                 cm_x=cmx, cm_y=cmy, cm_z=cmz,
+                                                                 bm_x=bmx, bm_y=bmy, bm_z=bmz,
+                                                                 use_retiming=ret, prefetch=pf,
+                                                                 bt=bt, qstore=qs)
+                                                        if check(kind, r, M, t) is None:
+                                                            found.append(t)
     found.sort(key=as_tuple)
     yield from found
 

@@ -28,6 +28,9 @@
 #ifndef CST_REMOTE
 #define CST_REMOTE 0  // 1: fused-halo twin (z-slab boundary launches, NEXT-3)
 #endif
+#ifndef CST_QSTORE
+#define CST_QSTORE 1  // streamed-direction state: 1 registers, 2 tensor memory (TMEM)
+#endif
 
 // ------------------------------------------------------------------ configuration
 constexpr int KIND = CST_KIND;  // 1 star, 2 box, 3 hypterm, 4 rhs4center-like
@@ -43,6 +46,7 @@ constexpr int CMX = CST_CMX, CMY = CST_CMY, CMZ = CST_CMZ;
 constexpr int BMX = CST_BMX, BMY = CST_BMY, BMZ = CST_BMZ;
 constexpr bool RETIME = CST_RET == 2;
 constexpr int PF = CST_PF;  // pipeline stages (1 = no prefetch)
+constexpr bool QTM = CST_QSTORE == 2;
 
 constexpr int NIN = KIND == 3 ? 8 : (KIND == 4 ? 5 : 1);
 constexpr int NOUT = KIND == 3 ? 5 : (KIND == 4 ? 3 : 1);
@@ -405,6 +409,32 @@ struct SGeo {
   int a0, b0, s_start, s_end;
 };
 
+// Work unit = (tile, chunk), tiles fastest.  The fast streaming kernels loop over units
+// (unit = first + k * stride): launched with one CTA per unit (grid = tiles x chunks) each
+// runs one; launched persistent (P.units > grid, host: cst_launch_range) every CTA walks
+// units in the hardware's own order, so neighbouring tiles stream the same planes at the
+// same time and their shared halo rows are read from L2 instead of HBM.
+__device__ __forceinline__ SGeo stream_geo_unit(const cst_kparams& P, int unit) {
+  SGeo g;
+  g.n_a = P.nx;
+  g.n_b = SZ ? P.ny : P.nz;
+  g.n_s = SZ ? P.nz : P.ny;
+  g.st_b = SZ ? P.py : P.pz;
+  g.st_s = SZ ? P.pz : P.py;
+  const int ntiles = P.tiles_a * P.tiles_b;
+  const int tile = unit % ntiles;
+  g.a0 = (tile % P.tiles_a) * TA;
+  g.b0 = (tile / P.tiles_a) * TB;
+  g.s_start = (unit / ntiles) * SB;
+  g.s_end = min(g.n_s, g.s_start + SB);
+  return g;
+}
+__device__ __forceinline__ int unit_first() { return blockIdx.x + blockIdx.y * gridDim.x; }
+__device__ __forceinline__ int unit_stride() { return gridDim.x * gridDim.y; }
+__device__ __forceinline__ int n_units(const cst_kparams& P) {
+  return P.units > 0 ? P.units : P.tiles_a * P.tiles_b * P.chunks;
+}
+
 __device__ __forceinline__ SGeo stream_geo(const cst_kparams& P) {
   SGeo g;
   g.n_a = P.nx;
@@ -712,11 +742,9 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
   Ctx C{P};
   constexpr int D = PF;
   constexpr int NP = STAGING == 1 ? 1 : NP1;
-  const SGeo g = stream_geo(P);
   const int ta = thread_x();
   const int tb = SZ ? thread_y() : thread_z();
   const int tid = threadIdx.x;
-  const int n_planes = (g.s_end - g.s_start) + 2 * R;
   const double* __restrict__ in = P.in[0];
   double* __restrict__ out = P.out[0];
   u64* bars = (u64*)(smem + NP * NIN * SLOT);
@@ -726,6 +754,28 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
   for (int i = 0; i < NCA; ++i) la[i] = merged_pos(i, ta, TBA, BMA);
 #pragma unroll
   for (int i = 0; i < NCB; ++i) lb[i] = merged_pos(i, tb, TBB, BMB);
+
+  if constexpr (STAGING == 3) {
+    if (tid == 0) {
+      for (int s = 0; s < NP; ++s) {
+        mbar_init(&bars[s], 1);  // full: producer arrive + TMA bytes
+#if CST_EMPTY_BARRIERS
+        mbar_init(&bars[NP + s], NTHR / 32);  // empty: one arrive per warp
+#endif
+      }
+      fence_mbar_init();
+    }
+    __syncthreads();
+  }
+  // ring slot / mbarrier phase of the unit's plane x: planes of all units of this CTA go
+  // through the ring in sequence (J0 = planes of the earlier units)
+  int J0 = 0;
+  auto SL = [&](int x) { return (J0 + x) % NP; };
+  auto PH = [&](int x) { return (u32)(((J0 + x) / NP) & 1); };
+  const int nu = n_units(P);
+  for (int unit = unit_first(); unit < nu; unit += unit_stride()) {
+  const SGeo g = stream_geo_unit(P, unit);
+  const int n_planes = (g.s_end - g.s_start) + 2 * R;
   const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
 
   // retimed: acc = pending outputs (2R+1 per point); gather: queue of centre values
@@ -742,23 +792,14 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
   // ---- prologue: first D planes in flight
   if constexpr (STAGING == 3) {
     if (tid == 0) {
-      for (int s = 0; s < NP; ++s) {
-        mbar_init(&bars[s], 1);  // full: producer arrive + TMA bytes
-#if CST_EMPTY_BARRIERS
-        mbar_init(&bars[NP + s], NTHR / 32);  // empty: one arrive per warp
-#endif
-      }
-      fence_mbar_init();
-    }
-    __syncthreads();
-    if (tid == 0) {
+      fence_proxy_async();  // slots last read by the previous unit's generic loads
       for (int j = 0; j < D && j < n_planes; ++j) {
-        mbar_arrive_expect_tx(&bars[j % NP], NIN * PL * 8);
-        tma_plane(P, g, smem + (j % NP) * NIN * SLOT, &bars[j % NP], g.s_start - R + j);
+        mbar_arrive_expect_tx(&bars[SL(j)], NIN * PL * 8);
+        tma_plane(P, g, smem + SL(j) * NIN * SLOT, &bars[SL(j)], g.s_start - R + j);
       }
     }
   } else if constexpr (STAGING == 2) {
-    ldst_plane(P, g, smem, g.s_start - R);
+    ldst_plane(P, g, smem + SL(0) * NIN * SLOT, g.s_start - R);
     if constexpr (D > 1) {
 #pragma unroll
       for (int f = 0; f < D - 1; ++f)
@@ -794,8 +835,8 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
       const int j = j0 + u;
       if (j >= n_planes) return;  // CTA-uniform
       const int p = g.s_start - R + j;
-      const int slot = j % NP;
-      if constexpr (STAGING == 3) mbar_wait(&bars[slot], (u32)((j / NP) & 1));
+      const int slot = SL(j);
+      if constexpr (STAGING == 3) mbar_wait(&bars[slot], PH(j));
 
       if constexpr (KIND == 1 && RETIME) {
         // retiming: plane p adds ws[p-o]*u to outputs o = p-R..p+R, its in-plane
@@ -825,7 +866,7 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
         if (j >= 2 * R) {
           const int po = p - R;
           double ip[NCB][NCA], cen[NCB][NCA];
-          star_inplane(C, plane_ld((j - R) % NP, po), la, lb, ip, cen);
+          star_inplane(C, plane_ld(SL(j - R), po), la, lb, ip, cen);
 #pragma unroll
           for (int ib = 0; ib < NCB; ++ib)
 #pragma unroll
@@ -874,7 +915,7 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
             for (int ia = 0; ia < NCA; ++ia) S[0][ib][ia] = 0.0;
           static_for<0, W>([&](auto QQ) {
             constexpr int ds = decltype(QQ)::value - R;
-            box_slices<1, ds, 0>(C, plane_ld((j - R + ds) % NP, po + ds), la, lb, S);
+            box_slices<1, ds, 0>(C, plane_ld(SL(j - R + ds), po + ds), la, lb, S);
           });
 #pragma unroll
           for (int ib = 0; ib < NCB; ++ib)
@@ -889,17 +930,17 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
         // per-warp release on an "empty" mbarrier; only the producer waits (experimental)
         if (j >= RETAIN) {
           __syncwarp();
-          if ((tid & 31) == 0) mbar_arrive(&bars[NP + (j - RETAIN) % NP]);
+          if ((tid & 31) == 0) mbar_arrive(&bars[NP + SL(j - RETAIN)]);
         }
         if (tid == 0 && j + D < n_planes) {
-          const int jn = j + D, sl = jn % NP;
-          if (jn >= NP) mbar_wait(&bars[NP + sl], (u32)((jn / NP - 1) & 1));
+          const int jn = j + D, sl = SL(jn);
+          if (J0 + jn >= NP) mbar_wait(&bars[NP + sl], (u32)(((J0 + jn) / NP - 1) & 1));
 #else
         // CTA barrier: every warp is done with the slot of plane j - RETAIN, which is then
         // refilled with plane j + D
         __syncthreads();
         if (tid == 0 && j + D < n_planes) {
-          const int sl = (j + D) % NP;
+          const int sl = SL(j + D);
 #endif
           fence_proxy_async();
           mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
@@ -908,7 +949,7 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
       } else if constexpr (STAGING == 2) {
         __syncthreads();
         if (j + 1 < n_planes) {
-          double* dst = smem + ((j + 1) % NP) * NIN * SLOT;
+          double* dst = smem + SL(j + 1) * NIN * SLOT;
           if constexpr (D == 1) {
             ldst_plane(P, g, dst, p + 1);
           } else {
@@ -933,6 +974,8 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
       }
     });
   }
+  J0 += n_planes;
+  }  // units
 }
 
 
@@ -1074,11 +1117,9 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   Ctx C{P};
   constexpr int D = PF;
   constexpr int NP = STAGING == 1 ? 1 : NP1;
-  const SGeo g = stream_geo(P);
   const int ta = thread_x();
   const int tb = SZ ? thread_y() : thread_z();
   const int tid = threadIdx.x;
-  const int n_planes = (g.s_end - g.s_start) + 2 * R;
   u64* bars = (u64*)(smem + NP * NIN * SLOT);
 
   int la[NCA], lb[NCB];
@@ -1086,12 +1127,32 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   for (int i = 0; i < NCA; ++i) la[i] = merged_pos(i, ta, TBA, BMA);
 #pragma unroll
   for (int i = 0; i < NCB; ++i) lb[i] = merged_pos(i, tb, TBB, BMB);
-  const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
 
   // streamed-direction weights ws[k] = -sign(k) dxinv_s a_|k| (host-precomputed, in the
   // constant bank after the 7 user coefficients: 8 for s = z, then 8 for s = y):
   // plane p contributes ws[p-o] * E_f(p) to flux_f(o)
   auto ws = [&](int k) { return C.coef(7 + (DS == 1 ? 8 : 0) + (k < 0 ? k + R : k + R - 1)); };
+
+  if constexpr (STAGING == 3) {
+    if (tid == 0) {
+      for (int s = 0; s < NP; ++s) {
+        mbar_init(&bars[s], 1);  // full: producer arrive + TMA bytes
+#if CST_EMPTY_BARRIERS
+        mbar_init(&bars[NP + s], NTHR / 32);  // empty: one arrive per warp
+#endif
+      }
+      fence_mbar_init();
+    }
+    __syncthreads();
+  }
+  int J0 = 0;  // planes of this CTA's earlier units (ring slot / phase continuity)
+  auto SL = [&](int x) { return (J0 + x) % NP; };
+  auto PH = [&](int x) { return (u32)(((J0 + x) / NP) & 1); };
+  const int nu = n_units(P);
+  for (int unit = unit_first(); unit < nu; unit += unit_stride()) {
+  const SGeo g = stream_geo_unit(P, unit);
+  const int n_planes = (g.s_end - g.s_start) + 2 * R;
+  const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
 
   double acc[5][NCB][NCA][W];  // retimed: pending fluxes ; gather: queue of E_f
 #pragma unroll
@@ -1106,23 +1167,14 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   double frag[D > 1 && STAGING == 2 ? (D - 1) * FR : 1];
   if constexpr (STAGING == 3) {
     if (tid == 0) {
-      for (int s = 0; s < NP; ++s) {
-        mbar_init(&bars[s], 1);  // full: producer arrive + TMA bytes
-#if CST_EMPTY_BARRIERS
-        mbar_init(&bars[NP + s], NTHR / 32);  // empty: one arrive per warp
-#endif
-      }
-      fence_mbar_init();
-    }
-    __syncthreads();
-    if (tid == 0) {
+      fence_proxy_async();  // slots last read by the previous unit's generic loads
       for (int j = 0; j < D && j < n_planes; ++j) {
-        mbar_arrive_expect_tx(&bars[j % NP], NIN * PL * 8);
-        tma_plane(P, g, smem + (j % NP) * NIN * SLOT, &bars[j % NP], g.s_start - R + j);
+        mbar_arrive_expect_tx(&bars[SL(j)], NIN * PL * 8);
+        tma_plane(P, g, smem + SL(j) * NIN * SLOT, &bars[SL(j)], g.s_start - R + j);
       }
     }
   } else if constexpr (STAGING == 2) {
-    ldst_plane(P, g, smem, g.s_start - R);
+    ldst_plane(P, g, smem + SL(0) * NIN * SLOT, g.s_start - R);
     if constexpr (D > 1) {
 #pragma unroll
       for (int f = 0; f < D - 1; ++f)
@@ -1161,8 +1213,8 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
       const int j = j0 + u;
       if (j >= n_planes) return;
       const int p = g.s_start - R + j;
-      const int slot = j % NP;
-      if constexpr (STAGING == 3) mbar_wait(&bars[slot], (u32)((j / NP) & 1));
+      const int slot = SL(j);
+      if constexpr (STAGING == 3) mbar_wait(&bars[slot], PH(j));
       LDT ld[NIN];
       loaders(slot, p, ld);
       if constexpr (RETIME) {
@@ -1233,7 +1285,7 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
         if (j >= 2 * R) {
           const int po = p - R;
           LDT ldo[NIN];
-          loaders((j - R) % NP, po, ldo);
+          loaders(SL(j - R), po, ldo);
           double ta_[5][NCB][NCA], tb_[5][NCB][NCA];
           hyp_inplane<0>(C, ldo, la, lb, ta_);
           hyp_inplane<1>(C, ldo, la, lb, tb_);
@@ -1264,17 +1316,17 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
         // per-warp release on an "empty" mbarrier; only the producer waits (experimental)
         if (j >= RETAIN) {
           __syncwarp();
-          if ((tid & 31) == 0) mbar_arrive(&bars[NP + (j - RETAIN) % NP]);
+          if ((tid & 31) == 0) mbar_arrive(&bars[NP + SL(j - RETAIN)]);
         }
         if (tid == 0 && j + D < n_planes) {
-          const int jn = j + D, sl = jn % NP;
-          if (jn >= NP) mbar_wait(&bars[NP + sl], (u32)((jn / NP - 1) & 1));
+          const int jn = j + D, sl = SL(jn);
+          if (J0 + jn >= NP) mbar_wait(&bars[NP + sl], (u32)(((J0 + jn) / NP - 1) & 1));
 #else
         // CTA barrier: every warp is done with the slot of plane j - RETAIN, which is then
         // refilled with plane j + D
         __syncthreads();
         if (tid == 0 && j + D < n_planes) {
-          const int sl = (j + D) % NP;
+          const int sl = SL(j + D);
 #endif
           fence_proxy_async();
           mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
@@ -1283,7 +1335,7 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
       } else if constexpr (STAGING == 2) {
         __syncthreads();
         if (j + 1 < n_planes) {
-          double* dst = smem + ((j + 1) % NP) * NIN * SLOT;
+          double* dst = smem + SL(j + 1) * NIN * SLOT;
           if constexpr (D == 1) {
             ldst_plane(P, g, dst, p + 1);
           } else {
@@ -1308,6 +1360,8 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
       }
     });
   }
+  J0 += n_planes;
+  }  // units
 }
 
 // =============================================================================
@@ -1680,15 +1734,242 @@ __device__ __forceinline__ void kernel_tblock(const cst_kparams& P, double* smem
   }
 }
 
+
+// In-plane part of the star in row-scatter form: the block's window rows are visited
+// once, top to bottom, and each row's values are added into the in-plane sums of the block
+// rows within R (y-terms) — plus, for the block's own rows, the x-terms and the centre.
+// Only the block's sums, centres and one row window are live: the register budget of the
+// TMEM path, whose streamed state is not in registers.
+template <class LD>
+__device__ __forceinline__ void star_inplane_rows(const Ctx& C, const LD& ld, const int* la,
+                                                  const int* lb, double (&ip)[NCB][NCA],
+                                                  double (&cen)[NCB][NCA]) {
+#pragma unroll
+  for (int cb = 0; cb < CMB; ++cb) {
+    const int lb0 = lb[cb * BMB];
+#pragma unroll
+    for (int ca = 0; ca < CMA; ++ca) {
+      const int la0 = la[ca * BMA];
+#pragma unroll
+      for (int wr = -R; wr < BMB + R; ++wr) {
+        if (wr >= 0 && wr < BMB) {
+          double w[BMA + 2 * XR];
+          load_xwin(ld, la0, lb0 + wr, w);
+#pragma unroll
+          for (int b = 0; b < BMA; ++b) {
+            const double c = w[XR + b];
+            double x = C.coef(0) * c;
+#pragma unroll
+            for (int k = -R; k <= R; ++k)
+              if (k != 0) x = fma(C.coef(star_ci(AX_A, k)), w[XR + b + k], x);
+            // every sum was started by its k = -R row (visited first), so add here
+            ip[cb * BMB + wr][ca * BMA + b] += x;
+            cen[cb * BMB + wr][ca * BMA + b] = c;
+#pragma unroll
+            for (int rb = 0; rb < BMB; ++rb) {
+              const int k = wr - rb;
+              if (k == 0 || k < -R || k > R) continue;
+              double& B = ip[cb * BMB + rb][ca * BMA + b];
+              B = (k == -R) ? C.coef(star_ci(AX_B, k)) * c : fma(C.coef(star_ci(AX_B, k)), c, B);
+            }
+          }
+        } else {
+          double v[BMA];
+          if constexpr (LD::VEC && (BMA % 2 == 0)) {
+#pragma unroll
+            for (int b = 0; b < BMA; b += 2) {
+              const double2 t = ld.at2(la0 + b, lb0 + wr);
+              v[b] = t.x;
+              v[b + 1] = t.y;
+            }
+          } else {
+#pragma unroll
+            for (int b = 0; b < BMA; ++b) v[b] = ld.at(la0 + b, lb0 + wr);
+          }
+#pragma unroll
+          for (int b = 0; b < BMA; ++b)
+#pragma unroll
+            for (int rb = 0; rb < BMB; ++rb) {
+              const int k = wr - rb;
+              if (k < -R || k > R) continue;
+              double& B = ip[cb * BMB + rb][ca * BMA + b];
+              B = (k == -R) ? C.coef(star_ci(AX_B, k)) * v[b] : fma(C.coef(star_ci(AX_B, k)), v[b], B);
+            }
+        }
+      }
+    }
+  }
+}
+
+// =============================================================================
+// star, streamed-direction state in tensor memory (qstore = 2)
+//
+// The retimed star keeps 2R+1 pending outputs per point in registers, which caps the
+// register blocking (merging) and so the shared-memory reuse of the in-plane
+// windows: at BM 2x2 the x/y windows cost ~10 smem loads per point and the kernel is
+// bound by the shared-memory pipe (profiles/).  Here the per-point streamed state lives in
+// TMEM instead — a ring of R (u, A) pairs per point, where at plane q
+//   A(q)     = ip(q) + sum_{k=-R..-1} ws[k] u(q+k)          (in-plane part + lower half)
+//   out(q-R) = A(q-R) + sum_{k=1..R-1} ws[k] u(q-R+k) + ws[R] u(q)
+// (the retimed split of P:69: each plane's contributions are added once, in plane order)
+// — so the registers hold only the current plane and the block can grow to 4x4 points.
+// TMEM reads run beside the shared-memory pipe (tools/tmem_bench.cu).
+// Layout: warp w -> lanes 32*(w%4) + lane, column block (w/4) * NPT*4R; point i of the
+// thread at +i*4R: u slots [0, 2R), A slots [2R, 4R), slot s = plane index mod R.
+// =============================================================================
+constexpr int NPT = NCA * NCB;
+constexpr int TM_WPQ = (NTHR / 32 + 3) / 4;  // warps sharing one TMEM lane quarter
+constexpr int TM_PCOLS = 4 * R;              // columns per point
+constexpr int TM_USED = TM_WPQ * NPT * TM_PCOLS;
+constexpr int TM_COLS = TM_USED <= 32 ? 32 : TM_USED <= 64 ? 64 : TM_USED <= 128 ? 128
+                      : TM_USED <= 256 ? 256 : 512;
+
+template <int DUMMY>
+__device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* smem) {
+  static_assert(KIND == 1 && STAGING == 3 && TS == 1, "TMEM queue: star, TMA, T_SD = 1");
+  static_assert(TM_USED <= 512, "TMEM queue exceeds 512 columns");
+  Ctx C{P};
+  constexpr int D = PF, NP = PF;
+  const int ta = thread_x();
+  const int tb = SZ ? thread_y() : thread_z();
+  const int tid = threadIdx.x, warp = tid / 32;
+  double* __restrict__ out = P.out[0];
+  u64* bars = (u64*)(smem + NP * SLOT);
+  u32* tslot = (u32*)(bars + NP);  // spare mbarrier words (kernel_smem_bytes reserves 2 NP)
+
+  int la[NCA], lb[NCB];
+#pragma unroll
+  for (int i = 0; i < NCA; ++i) la[i] = merged_pos(i, ta, TBA, BMA);
+#pragma unroll
+  for (int i = 0; i < NCB; ++i) lb[i] = merged_pos(i, tb, TBB, BMB);
+
+  if (warp == 0) tmem_alloc(tslot, TM_COLS);
+  if (tid == 0) {
+    for (int s = 0; s < NP; ++s) mbar_init(&bars[s], 1);
+    fence_mbar_init();
+  }
+  tmem_fence_before_sync();
+  __syncthreads();
+  tmem_fence_after_sync();
+  const u32 tq = *tslot + ((u32)((warp & 3) * 32) << 16) + (u32)((warp >> 2) * NPT * TM_PCOLS);
+  auto ws = [&](int k) { return C.coef(star_ci(AX_S, k)); };
+  int J0 = 0;  // planes of this CTA's earlier units (ring slot / phase continuity)
+  const int nu = n_units(P);
+  for (int unit = unit_first(); unit < nu; unit += unit_stride()) {
+  const SGeo g = stream_geo_unit(P, unit);
+  const int n_planes = (g.s_end - g.s_start) + 2 * R;
+  const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
+  if (tid == 0) {
+    fence_proxy_async();
+    for (int j = 0; j < D && j < n_planes; ++j) {
+      const int sl = (J0 + j) % NP;
+      mbar_arrive_expect_tx(&bars[sl], PL * 8);
+      tma_plane(P, g, smem + sl * SLOT, &bars[sl], g.s_start - R + j);
+    }
+  }
+
+  // one plane per iteration, ring slots rotated at run time (slot of plane j = j mod R):
+  // a compile-time rotation would need R unrolled copies of the plane, whose hoisted
+  // invariants cost more registers than the TMEM ring saves
+#pragma unroll 1
+  for (int j = 0; j < n_planes; ++j) {
+    const int p = g.s_start - R + j;
+    const int slot = (J0 + j) % NP;
+    const int u = j % R;
+    mbar_wait(&bars[slot], (u32)(((J0 + j) / NP) & 1));
+    const SmemPlane ld{smem + slot * SLOT};
+    const bool need_a = j >= R && j < n_planes - R;  // A(p) feeds an interior output
+    u32 cu[R];  // column of u(p - R + m), m = 0..R-1: slot (j + m) mod R
+#pragma unroll
+    for (int m = 0; m < R; ++m) cu[m] = (u32)(2 * ((u + m) % R));
+    const u32 cs = (u32)(2 * u);  // this plane's slot (holds plane j - R until rewritten)
+    auto issue = [&](int pt, TmQ<R>& q) {
+      const u32 tp = tq + (u32)(pt * TM_PCOLS);
+      u32 ta[R];
+#pragma unroll
+      for (int m = 0; m < R; ++m) ta[m] = tp + cu[m];
+      tmem_ld_issue<R>(ta, tp + 2 * R + cs, q);
+    };
+    // the ring of point 0 is in flight while the in-plane part is computed; the ring of
+    // point pt + 1 while point pt is finished (one-deep TMEM load pipeline)
+    TmQ<R> q0, q1;
+    if (j >= R) issue(0, q0);
+    double ip[NCB][NCA], cen[NCB][NCA];
+    if (need_a) star_inplane_rows(C, ld, la, lb, ip, cen);
+    else load_centres(ld, la, lb, cen);
+    auto finish = [&](auto PP, TmQ<R>& q, TmQ<R>& qn) {
+      constexpr int pt = decltype(PP)::value, ib = pt / NCA, ia = pt % NCA;
+      const u32 tp = tq + (u32)(pt * TM_PCOLS);
+      if (j >= R) {
+        tmem_ld_wait<R>(q);
+        if constexpr (pt + 1 < NPT) issue(pt + 1, qn);
+        if (need_a) {  // A(p) = ip(p) + sum_{k=-R..-1} ws[k] u(p+k)
+          double a = ip[ib][ia];
+#pragma unroll
+          for (int m = 0; m < R; ++m) a = fma(ws(m - R), tmq_u<R>(q, m), a);
+          tmem_st_d(tp + 2 * R + cs, a);
+        }
+        if (j >= 2 * R) {  // out(p-R) = A(p-R) + sum_{k=1..R-1} ws[k] u(p-R+k) + ws[R] u(p)
+          double o = tmq_a<R>(q);
+#pragma unroll
+          for (int k = 1; k < R; ++k) o = fma(ws(k), tmq_u<R>(q, k), o);
+          o = fma(ws(R), cen[ib][ia], o);
+          if (g.a0 + la[ia] < g.n_a && g.b0 + lb[ib] < g.n_b) {
+            const long long off =
+                col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)(p - R) * g.st_s;
+            out[off] = o;
+            if constexpr (CST_REMOTE) P.rout[0][off] = o;
+          }
+        }
+      }
+      tmem_st_d(tp + cs, cen[ib][ia]);
+    };
+    static_for<0, NPT>([&](auto PP) {
+      if constexpr (decltype(PP)::value % 2 == 0) finish(PP, q0, q1);
+      else finish(PP, q1, q0);
+    });
+    tmem_wait_st();  // the next plane reads these slots
+    __syncthreads();
+    if (tid == 0 && j + D < n_planes) {
+      const int sl = (J0 + j + D) % NP;
+      fence_proxy_async();
+      mbar_arrive_expect_tx(&bars[sl], PL * 8);
+      tma_plane(P, g, smem + sl * SLOT, &bars[sl], p + D);
+    }
+  }
+  J0 += n_planes;
+  }  // units
+  tmem_fence_before_sync();
+  __syncthreads();
+  tmem_fence_after_sync();
+  if (warp == 0) tmem_dealloc(*tslot, TM_COLS);
+}
+
 // =============================================================================
 // entry point
 // =============================================================================
-extern "C" __global__ void __launch_bounds__(NTHR) cst_kernel(const __grid_constant__ cst_kparams P) {
+// TMEM path: cap the registers at ~96 + 4 per point of the block (minimum resident CTAs
+// for ptxas) — with the ring in TMEM the registers only hold the current plane, and the
+// unconstrained schedule hoists every shared-memory load of the block (up to 255 registers)
+#define CST_TM_NPT (CST_BMX * CST_CMX * CST_BMY * CST_CMY * CST_BMZ * CST_CMZ)
+#define CST_TM_NTHR (CST_TBX * CST_TBY * CST_TBZ)
+#ifndef CST_TM_MINB
+#define CST_TM_MINB (65536 / (CST_TM_NTHR * (96 + 4 * CST_TM_NPT)) > 0 \
+                         ? 65536 / (CST_TM_NTHR * (96 + 4 * CST_TM_NPT)) : 1)
+#endif
+#if CST_QSTORE == 2
+#define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ, CST_TM_MINB)
+#else
+#define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ)
+#endif
+extern "C" __global__ void CST_LB cst_kernel(const __grid_constant__ cst_kparams P) {
   extern __shared__ __align__(128) double cst_smem[];
   if constexpr (BT > 1) {
     kernel_tblock<0>(P, cst_smem);
   } else if constexpr (!STREAM) {
     kernel_tile3d(P, cst_smem);
+  } else if constexpr (QTM) {
+    kernel_star_tmem<0>(P, cst_smem);
   } else if constexpr ((KIND == 1 || KIND == 2) && TS == 1) {
     kernel_stream1(P, cst_smem);
   } else if constexpr (KIND == 3 && TS == 1) {

@@ -29,11 +29,11 @@ cst_status fail(cst_status s, const std::string& msg);
   } while (0)
 
 // ------------------------------------------------------------------ settings
-// The 20 fields in canonical order: Table I row order, then the temporal
-// blocking degree (B200 extension, NEXT-2).
+// The 21 fields in canonical order: Table I row order, then the temporal
+// blocking degree (B200 extension, NEXT-2) and the streamed-state store (qstore, TMEM).
 enum Field {
   F_TBX, F_TBY, F_TBZ, F_STAGING, F_CONST, F_STREAM, F_SD, F_SB, F_UFX, F_UFY, F_UFZ,
-  F_CMX, F_CMY, F_CMZ, F_BMX, F_BMY, F_BMZ, F_RET, F_PF, F_BT, F_COUNT
+  F_CMX, F_CMY, F_CMZ, F_BMX, F_BMY, F_BMZ, F_RET, F_PF, F_BT, F_QS, F_COUNT
 };
 using Tuple = std::array<int32_t, F_COUNT>;
 Tuple to_tuple(const cst_setting& s);
@@ -46,10 +46,12 @@ struct StencilInfo {
   int64_t M[3];  // nx, ny, nz
 };
 
-// Rule check (R1..R12, R14).  Returns nullptr if valid else the rule id.
+// Rule check (R1..R12, R14, R15).  Returns nullptr if valid else the rule id.
 const char* check_rules(const StencilInfo& st, const Tuple& t);
 int64_t model_smem_bytes(int kind, int r, const Tuple& t);
 int64_t model_regs(int kind, int r, const Tuple& t);
+// TMEM columns one CTA of the qstore = 2 path allocates (power of two >= 32)
+int tmem_cols_alloc(int r, const Tuple& t);
 // Dynamic shared memory the kernel variant actually uses (<= model for fast paths).
 int64_t kernel_smem_bytes(int kind, int r, const Tuple& t);
 
@@ -62,8 +64,8 @@ class Space {
   bool rank(const Tuple& t, uint64_t* out) const;
 
  private:
-  struct Core {  // (CM x3, BM x3, ret, pf, bt) and its per-dim UF bounds (counts)
-    int32_t cm[3], bm[3], ret, pf, bt;
+  struct Core {  // (CM x3, BM x3, ret, pf, bt, qs) and its per-dim UF bounds (counts)
+    int32_t cm[3], bm[3], ret, pf, bt, qs;
     int32_t nuf[3];
   };
   struct Prefix {
@@ -153,6 +155,7 @@ struct cst_stencil {
   std::vector<double> kcoef;    // kernel coefficient bank (coeffs + derived weights)
   cst_grid grid{};
   int device = 0;
+  int num_sms = 0;              // SMs of the device (persistent launches); 0 = unknown
   cst::StencilInfo info{};
   std::unique_ptr<cst::Space> space;
   std::map<std::string, cst::Variant> variants;

@@ -124,7 +124,7 @@ static std::string prefix_for(const StencilInfo& st, const Tuple& t, bool remote
   static const char* names[F_COUNT] = {"TBX", "TBY", "TBZ", "STAGING", "CONST", "STREAM",
                                        "SD",  "SB",  "UFX", "UFY",     "UFZ",   "CMX",
                                        "CMY", "CMZ", "BMX", "BMY",     "BMZ",   "RET",
-                                       "PF",  "BT"};
+                                       "PF",  "BT",      "QSTORE"};
   for (int i = 0; i < F_COUNT; ++i) o << "#define CST_" << names[i] << " " << t[i] << "\n";
   o << "#include \"cst_kernels.cuh\"\n";
   return o.str();

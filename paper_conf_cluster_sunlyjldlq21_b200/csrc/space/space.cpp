@@ -2,9 +2,10 @@
 // explicit rules of P:149 (R1-R3), our semantics rules (R4-R9) and the
 // implicit resource rules (R10-R12: "settings ... restricted by the usage of
 // register and shared memory ... only non-spilled parameter settings are explored") and
-// R14, the structural requirements of the temporally blocked path (field 20, bt).
+// R14, the structural requirements of the temporally blocked path (field 20, bt), and
+// R15, those of the TMEM streamed-state path (field 21, qstore).
 //
-// Canonical order: lexicographic over the 20 fields (Table I row order, then bt), values
+// Canonical order: lexicographic over the 21 fields (Table I row order, bt, qstore), values
 // ascending.  count / rank / unrank are exact (bit-exact with oracle/space.py).
 #include <algorithm>
 #include <cstring>
@@ -16,12 +17,12 @@ namespace cst {
 const char* const kFieldNames[F_COUNT] = {
     "tb_x", "tb_y", "tb_z", "staging", "use_constant", "use_streaming", "sd", "sb",
     "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z", "bm_x", "bm_y", "bm_z",
-    "use_retiming", "prefetch", "bt"};
+    "use_retiming", "prefetch", "bt", "qstore"};
 
 Tuple to_tuple(const cst_setting& s) {
   return Tuple{s.tb[0], s.tb[1], s.tb[2], s.staging, s.use_constant, s.use_streaming,
                s.sd, s.sb, s.uf[0], s.uf[1], s.uf[2], s.cm[0], s.cm[1], s.cm[2],
-               s.bm[0], s.bm[1], s.bm[2], s.use_retiming, s.prefetch, s.bt};
+               s.bm[0], s.bm[1], s.bm[2], s.use_retiming, s.prefetch, s.bt, s.qstore};
 }
 
 cst_setting from_tuple(const Tuple& t) {
@@ -34,7 +35,7 @@ cst_setting from_tuple(const Tuple& t) {
     s.cm[d] = t[F_CMX + d];
     s.bm[d] = t[F_BMX + d];
   }
-  s.use_retiming = t[F_RET]; s.prefetch = t[F_PF]; s.bt = t[F_BT];
+  s.use_retiming = t[F_RET]; s.prefetch = t[F_PF]; s.bt = t[F_BT]; s.qstore = t[F_QS];
   return s;
 }
 
@@ -90,6 +91,32 @@ static int64_t tb_smem_bytes(int r, const Tuple& t) {
   tb_extent(r, t, 0, &e0x, &e0y);
   tb_extent(r, t, 1, &e1x, &e1y);
   return t[F_PF] * rnd128(e0x * e0y * 8) + (t[F_BT] - 1) * 2 * rnd128(e1x * e1y * 8);
+}
+
+// R15: the TMEM streamed-state path (qstore = 2): star, streaming with T_SD = 1, TMA,
+// retimed, bt = 1; ceil(threads / 128) warps share a TMEM lane quarter, each thread keeps
+// 4r columns per point, 512 columns per SM (mirrors TM_* in csrc/kernels/cst_kernels.cuh)
+static int64_t tmem_cols(int r, const Tuple& t) {
+  int64_t ppt = 1;
+  for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
+  const int64_t nthr = (int64_t)t[F_TBX] * t[F_TBY] * t[F_TBZ];
+  return (nthr / 32 + 3) / 4 * ppt * 4 * r;
+}
+
+int tmem_cols_alloc(int r, const Tuple& t) {
+  const int64_t used = tmem_cols(r, t);
+  int c = 32;
+  while (c < used && c < 512) c *= 2;
+  return c;
+}
+
+static bool qs_path_ok(int kind, int r, const Tuple& t) {
+  if (kind != CST_STAR || t[F_STREAM] != 2 || t[F_STAGING] != 3 || t[F_RET] != 2 ||
+      t[F_BT] != 1)
+    return false;
+  const int sd = t[F_SD] - 1;
+  if ((int64_t)t[F_TBX + sd] * t[F_BMX + sd] * t[F_CMX + sd] != 1) return false;
+  return tmem_cols(r, t) <= 512;
 }
 
 static bool tb_path_ok(int kind, const Tuple& t) {
@@ -156,6 +183,13 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
 }
 
 int64_t model_regs(int kind, int r, const Tuple& t) {
+  if (t[F_QS] == 2) {
+    // TMEM path: in-plane part + centre per point, one point's ring (r + 1 doubles) and
+    // the column windows of the block in flight
+    int64_t ppt = 1;
+    for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
+    return 32 + 2 * (2 * ppt + (r + 1) + 2 * r);
+  }
   if (t[F_BT] > 1) {
     int64_t pts = 0;
     for (int lv = 1; lv <= t[F_BT]; ++lv) pts += tb_blocks_per_thread(r, t, lv);
@@ -216,6 +250,7 @@ const char* check_rules(const StencilInfo& st, const Tuple& t) {
   if (t[F_RET] < 1 || t[F_RET] > 2) return "range: use_retiming";
   if (t[F_PF] < 1 || t[F_PF] > 4) return "range: prefetch";
   if (t[F_BT] != 1 && t[F_BT] != 2 && t[F_BT] != 4) return "range: bt";
+  if (t[F_QS] < 1 || t[F_QS] > 2) return "range: qstore";
 
   const int64_t tb = (int64_t)t[F_TBX] * t[F_TBY] * t[F_TBZ];
   if (tb > 1024) return "R1";
@@ -241,6 +276,7 @@ const char* check_rules(const StencilInfo& st, const Tuple& t) {
   if (ppt > 16) return "R7";
   if (t[F_PF] > 1 && !stream) return "R9";
   if (t[F_BT] > 1 && !tb_path_ok(st.kind, t)) return "R14";
+  if (t[F_QS] == 2 && !qs_path_ok(st.kind, st.r, t)) return "R15";
   if (model_smem_bytes(st.kind, st.r, t) > SMEM_LIMIT) return "R10";
   if (model_regs(st.kind, st.r, t) > REG_LIMIT) return "R11";
   if (t[F_STAGING] == 3 && !tma_ok(st.r, t)) return "R12";
@@ -283,7 +319,8 @@ void Space::cores_for(const int32_t* pre, std::vector<Core>* cores) const {
               if (!cover) continue;
               for (int32_t ret = 1; ret <= 2; ++ret)
                 for (int32_t pf = 1; pf <= 4; ++pf)
-                  for (int32_t bt = 1; bt <= 4; bt *= 2) {
+                  for (int32_t bt = 1; bt <= 4; bt *= 2)
+                  for (int32_t qs = 1; qs <= 2; ++qs) {
                   for (int d = 0; d < 3; ++d) {
                     t[F_CMX + d] = cm[d];
                     t[F_BMX + d] = bm[d];
@@ -291,6 +328,7 @@ void Space::cores_for(const int32_t* pre, std::vector<Core>* cores) const {
                   t[F_RET] = ret;
                   t[F_PF] = pf;
                   t[F_BT] = bt;
+                  t[F_QS] = qs;
                   // UF is not part of the core: R14 needs UF = 1, which the UF counts
                   // below encode (a bt > 1 core admits only the first UF value per dim)
                   if (check_rules(st_, t) != nullptr) continue;
@@ -306,15 +344,16 @@ void Space::cores_for(const int32_t* pre, std::vector<Core>* cores) const {
                   c.ret = ret;
                   c.pf = pf;
                   c.bt = bt;
+                  c.qs = qs;
                   cores->push_back(c);
                 }
             }
       }
-  // canonical core order: CMx, CMy, CMz, BMx, BMy, BMz, ret, pf, bt
+  // canonical core order: CMx, CMy, CMz, BMx, BMy, BMz, ret, pf, bt, qs
   std::stable_sort(cores->begin(), cores->end(), [](const Core& a, const Core& b) {
-    const int32_t ka[9] = {a.cm[0], a.cm[1], a.cm[2], a.bm[0], a.bm[1], a.bm[2], a.ret, a.pf, a.bt};
-    const int32_t kb[9] = {b.cm[0], b.cm[1], b.cm[2], b.bm[0], b.bm[1], b.bm[2], b.ret, b.pf, b.bt};
-    return std::lexicographical_compare(ka, ka + 9, kb, kb + 9);
+    const int32_t ka[10] = {a.cm[0], a.cm[1], a.cm[2], a.bm[0], a.bm[1], a.bm[2], a.ret, a.pf, a.bt, a.qs};
+    const int32_t kb[10] = {b.cm[0], b.cm[1], b.cm[2], b.bm[0], b.bm[1], b.bm[2], b.ret, b.pf, b.bt, b.qs};
+    return std::lexicographical_compare(ka, ka + 10, kb, kb + 10);
   });
 }
 
@@ -408,6 +447,7 @@ bool Space::at(uint64_t rank, Tuple* out) const {
       t[F_RET] = c.ret;
       t[F_PF] = c.pf;
       t[F_BT] = c.bt;
+      t[F_QS] = c.qs;
       *out = t;
       return true;
     }
@@ -459,7 +499,7 @@ bool Space::rank(const Tuple& t, uint64_t* out) const {
   }
   for (const Core& c : cores) {
     if (uidx[0] >= c.nuf[0] || uidx[1] >= c.nuf[1] || uidx[2] >= c.nuf[2]) continue;
-    bool same = c.ret == t[F_RET] && c.pf == t[F_PF] && c.bt == t[F_BT];
+    bool same = c.ret == t[F_RET] && c.pf == t[F_PF] && c.bt == t[F_BT] && c.qs == t[F_QS];
     for (int d = 0; d < 3; ++d)
       same = same && c.cm[d] == t[F_CMX + d] && c.bm[d] == t[F_BMX + d];
     if (same) {

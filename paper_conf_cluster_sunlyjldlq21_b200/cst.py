@@ -30,7 +30,7 @@ N_OUT = {CST_STAR: 1, CST_BOX: 1, CST_HYPTERM: 5, CST_RHS4: 3}
 
 FIELDS = ("tb_x", "tb_y", "tb_z", "staging", "use_constant", "use_streaming", "sd", "sb",
           "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z", "bm_x", "bm_y", "bm_z",
-          "use_retiming", "prefetch", "bt")
+          "use_retiming", "prefetch", "bt", "qstore")
 
 
 class CstError(RuntimeError):
@@ -64,7 +64,7 @@ class cst_setting(ctypes.Structure):
                 ("sd", ctypes.c_int32), ("sb", ctypes.c_int32), ("uf", ctypes.c_int32 * 3),
                 ("cm", ctypes.c_int32 * 3), ("bm", ctypes.c_int32 * 3),
                 ("use_retiming", ctypes.c_int32), ("prefetch", ctypes.c_int32),
-                ("bt", ctypes.c_int32)]
+                ("bt", ctypes.c_int32), ("qstore", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         d = {}
@@ -74,7 +74,7 @@ class cst_setting(ctypes.Structure):
             d["cm_" + ax] = self.cm[i]
             d["bm_" + ax] = self.bm[i]
         for f in ("staging", "use_constant", "use_streaming", "sd", "sb", "use_retiming",
-                  "prefetch", "bt"):
+                  "prefetch", "bt", "qstore"):
             d[f] = getattr(self, f)
         return {k: d[k] for k in FIELDS}
 
@@ -94,6 +94,7 @@ class cst_setting(ctypes.Structure):
                   "prefetch"):
             setattr(s, f, d[f])
         s.bt = d.get("bt", 1)   # field 20 (temporal blocking); older records predate it
+        s.qstore = d.get("qstore", 1)  # field 21 (streamed state in TMEM); likewise
         return s
 
     def __repr__(self):

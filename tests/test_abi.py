@@ -139,6 +139,15 @@ def test_rules_agree_with_oracle_on_random_tuples():
                     d["cm_" + ax] = d["uf_" + ax] = 1
                 d["bm_x"], d["bm_y"] = rng.choice([1, 2]), rng.choice([1, 2])
                 d["tb_x"], d["tb_y"] = rng.choice([8, 16, 32, 64]), rng.choice([1, 2, 4, 8])
+            d["qstore"] = rng.choice([1, 1, 2])
+            if rng.random() < 0.3:              # the TMEM streamed-state path's shape (R15)
+                d.update(use_streaming=2, sd=rng.choice([2, 3]), staging=3, use_retiming=2,
+                         bt=1, qstore=2)
+                d["sb"] = rng.choice(p2(M[d["sd"] - 1]))
+                sa = "xyz"[d["sd"] - 1]
+                d["tb_" + sa] = d["bm_" + sa] = d["cm_" + sa] = 1
+                d["bm_x"] = rng.choice([1, 2, 4])
+                d["tb_x"], d["tb_y" if sa == "z" else "tb_z"] = rng.choice([16, 32, 64]), rng.choice([1, 2, 4, 8])
             want = S.check(kind, r, M, d)
             s = C.cst_setting.from_dict(d)
             try:

@@ -145,7 +145,7 @@ def test_literal_table1_counts():
 def test_space_rules_spot_checks():
     base = dict(tb_x=32, tb_y=4, tb_z=1, staging=3, use_constant=1, use_streaming=2, sd=3,
                 sb=64, uf_x=1, uf_y=1, uf_z=1, cm_x=1, cm_y=1, cm_z=1, bm_x=1, bm_y=1, bm_z=1,
-                use_retiming=2, prefetch=2, bt=1)
+                use_retiming=2, prefetch=2, bt=1, qstore=1)
     M = (512, 512, 512)
     assert S.check(1, 4, M, base) is None
     assert S.check(1, 4, M, dict(base, tb_x=64, tb_y=32)) == "R1"
@@ -180,6 +180,22 @@ def test_space_rules_spot_checks():
     assert S.est_regs(2, 1, tb) == 32 + 2 * (36 + 24)
     assert S.check(1, 4, M, dict(tb, bt=4)) == "R11"
     assert S.check(2, 1, M, dict(tb, tb_x=128, tb_y=1, bm_y=1)) == "R12"  # 256 + 8 > 256
+    # TMEM streamed state (field 21): R15 structure + capacity, by hand
+    q = dict(base, tb_x=32, tb_y=4, bm_x=4, bm_y=4, qstore=2)
+    # 128 threads = 4 warps, one per lane quarter; 16 points x 4r = 16 columns -> 256
+    assert S.tmem_columns(4, q) == 256 and S.check(1, 4, M, q) is None
+    # registers: 2 doubles per point (in-plane part, centre) + ring (r + 1) + 2r
+    assert S.est_regs(1, 4, q) == 32 + 2 * (32 + 5 + 8)
+    assert S.check(1, 4, M, dict(base, bm_x=4, bm_y=4)) == "R11"  # same block in registers
+    assert S.check(1, 4, M, dict(q, tb_y=8)) is None    # 8 warps: 2 per quarter -> 512
+    assert S.tmem_columns(4, dict(q, tb_y=8)) == 512
+    assert S.check(1, 4, M, dict(q, tb_y=16, bm_y=2)) is None   # 4 warps/quarter x 8 x 16
+    assert S.check(1, 4, M, dict(q, tb_y=16, bm_y=4)) == "R15"  # 1024 columns
+    assert S.check(3, 4, M, dict(base, qstore=2)) == "R15"    # hypterm: no TMEM path
+    assert S.check(1, 4, M, dict(q, staging=2)) == "R15"
+    assert S.check(1, 4, M, dict(q, use_retiming=1)) == "R15"
+    assert S.check(1, 4, M, dict(q, tb_z=2, tb_y=2)) == "R15"  # T_SD = 2
+    assert S.check(1, 4, M, dict(q, sd=2, tb_y=1, tb_z=4, bm_y=1, bm_z=4)) is None
 
 
 def test_space_enumeration_small_is_sorted_and_valid():

@@ -37,7 +37,8 @@ __device__ __forceinline__ void tm_dealloc(u32 taddr, u32 ncols) {
       "r"(r[15])                                                                               \
       : "memory")
 
-// mode 0: ld only (wait every NB loads), 1: st only, 2: ld+st, 3: LDS.64 reference
+// mode 0: ld only (wait every NB loads), 1: st only, 2: ld+st, 3: LDS.64 reference,
+// 4: LDTM and LDS.64 interleaved (do the two pipes add up?)
 template <int MODE, int NB>
 __global__ void bench(int iters, unsigned long long* out, u32* sink) {
   __shared__ u32 slot;
@@ -70,17 +71,17 @@ __global__ void bench(int iters, unsigned long long* out, u32* sink) {
     for (int b = 0; b < NB; ++b) {
       const u32 col = col0 + ((it * NB + b) * 16) % colspan;
       const u32 ta = base + lane_off + col;
-      if (MODE == 0 || MODE == 2) LD16(ta, r);
+      if (MODE == 0 || MODE == 2 || MODE == 4) LD16(ta, r);
       if (MODE == 1 || MODE == 2) {
         if (MODE == 2) asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
         ST16(ta, r);
       }
-      if (MODE == 3) {
-        const double* p = sm + ((threadIdx.x + it * 7 + b * 33) & 4095);
+      if (MODE == 3 || MODE == 4) {
+        const double* p = sm + ((threadIdx.x + it * 7 + b * 33) & 3583);
         dacc += p[0] + p[64] + p[128] + p[192] + p[256] + p[320] + p[384] + p[448];
       }
     }
-    if (MODE == 0) {
+    if (MODE == 0 || MODE == 4) {
       asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 #pragma unroll
       for (int i = 0; i < 16; ++i) acc += r[i];
@@ -133,6 +134,8 @@ void run(const char* name, int threads) {
 int main() {
   for (int t : {128, 256, 512}) {
     run<0, 4>("tmem_ld", t);
+    run<0, 1>("tmem_ld_w1", t);
+    run<4, 4>("ldtm+lds", t);
     run<1, 4>("tmem_st", t);
     run<2, 4>("tmem_ldst", t);
     run<3, 4>("lds64", t);
