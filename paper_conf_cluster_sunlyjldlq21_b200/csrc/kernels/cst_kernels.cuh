@@ -409,32 +409,6 @@ struct SGeo {
   int a0, b0, s_start, s_end;
 };
 
-// Work unit = (tile, chunk), tiles fastest.  The fast streaming kernels loop over units
-// (unit = first + k * stride): launched with one CTA per unit (grid = tiles x chunks) each
-// runs one; launched persistent (P.units > grid, host: cst_launch_range) every CTA walks
-// units in the hardware's own order, so neighbouring tiles stream the same planes at the
-// same time and their shared halo rows are read from L2 instead of HBM.
-__device__ __forceinline__ SGeo stream_geo_unit(const cst_kparams& P, int unit) {
-  SGeo g;
-  g.n_a = P.nx;
-  g.n_b = SZ ? P.ny : P.nz;
-  g.n_s = SZ ? P.nz : P.ny;
-  g.st_b = SZ ? P.py : P.pz;
-  g.st_s = SZ ? P.pz : P.py;
-  const int ntiles = P.tiles_a * P.tiles_b;
-  const int tile = unit % ntiles;
-  g.a0 = (tile % P.tiles_a) * TA;
-  g.b0 = (tile / P.tiles_a) * TB;
-  g.s_start = (unit / ntiles) * SB;
-  g.s_end = min(g.n_s, g.s_start + SB);
-  return g;
-}
-__device__ __forceinline__ int unit_first() { return blockIdx.x + blockIdx.y * gridDim.x; }
-__device__ __forceinline__ int unit_stride() { return gridDim.x * gridDim.y; }
-__device__ __forceinline__ int n_units(const cst_kparams& P) {
-  return P.units > 0 ? P.units : P.tiles_a * P.tiles_b * P.chunks;
-}
-
 __device__ __forceinline__ SGeo stream_geo(const cst_kparams& P) {
   SGeo g;
   g.n_a = P.nx;
@@ -742,9 +716,11 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
   Ctx C{P};
   constexpr int D = PF;
   constexpr int NP = STAGING == 1 ? 1 : NP1;
+  const SGeo g = stream_geo(P);
   const int ta = thread_x();
   const int tb = SZ ? thread_y() : thread_z();
   const int tid = threadIdx.x;
+  const int n_planes = (g.s_end - g.s_start) + 2 * R;
   const double* __restrict__ in = P.in[0];
   double* __restrict__ out = P.out[0];
   u64* bars = (u64*)(smem + NP * NIN * SLOT);
@@ -754,28 +730,6 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
   for (int i = 0; i < NCA; ++i) la[i] = merged_pos(i, ta, TBA, BMA);
 #pragma unroll
   for (int i = 0; i < NCB; ++i) lb[i] = merged_pos(i, tb, TBB, BMB);
-
-  if constexpr (STAGING == 3) {
-    if (tid == 0) {
-      for (int s = 0; s < NP; ++s) {
-        mbar_init(&bars[s], 1);  // full: producer arrive + TMA bytes
-#if CST_EMPTY_BARRIERS
-        mbar_init(&bars[NP + s], NTHR / 32);  // empty: one arrive per warp
-#endif
-      }
-      fence_mbar_init();
-    }
-    __syncthreads();
-  }
-  // ring slot / mbarrier phase of the unit's plane x: planes of all units of this CTA go
-  // through the ring in sequence (J0 = planes of the earlier units)
-  int J0 = 0;
-  auto SL = [&](int x) { return (J0 + x) % NP; };
-  auto PH = [&](int x) { return (u32)(((J0 + x) / NP) & 1); };
-  const int nu = n_units(P);
-  for (int unit = unit_first(); unit < nu; unit += unit_stride()) {
-  const SGeo g = stream_geo_unit(P, unit);
-  const int n_planes = (g.s_end - g.s_start) + 2 * R;
   const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
 
   // retimed: acc = pending outputs (2R+1 per point); gather: queue of centre values
@@ -792,14 +746,23 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
   // ---- prologue: first D planes in flight
   if constexpr (STAGING == 3) {
     if (tid == 0) {
-      fence_proxy_async();  // slots last read by the previous unit's generic loads
+      for (int s = 0; s < NP; ++s) {
+        mbar_init(&bars[s], 1);  // full: producer arrive + TMA bytes
+#if CST_EMPTY_BARRIERS
+        mbar_init(&bars[NP + s], NTHR / 32);  // empty: one arrive per warp
+#endif
+      }
+      fence_mbar_init();
+    }
+    __syncthreads();
+    if (tid == 0) {
       for (int j = 0; j < D && j < n_planes; ++j) {
-        mbar_arrive_expect_tx(&bars[SL(j)], NIN * PL * 8);
-        tma_plane(P, g, smem + SL(j) * NIN * SLOT, &bars[SL(j)], g.s_start - R + j);
+        mbar_arrive_expect_tx(&bars[j % NP], NIN * PL * 8);
+        tma_plane(P, g, smem + (j % NP) * NIN * SLOT, &bars[j % NP], g.s_start - R + j);
       }
     }
   } else if constexpr (STAGING == 2) {
-    ldst_plane(P, g, smem + SL(0) * NIN * SLOT, g.s_start - R);
+    ldst_plane(P, g, smem, g.s_start - R);
     if constexpr (D > 1) {
 #pragma unroll
       for (int f = 0; f < D - 1; ++f)
@@ -835,8 +798,8 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
       const int j = j0 + u;
       if (j >= n_planes) return;  // CTA-uniform
       const int p = g.s_start - R + j;
-      const int slot = SL(j);
-      if constexpr (STAGING == 3) mbar_wait(&bars[slot], PH(j));
+      const int slot = j % NP;
+      if constexpr (STAGING == 3) mbar_wait(&bars[slot], (u32)((j / NP) & 1));
 
       if constexpr (KIND == 1 && RETIME) {
         // retiming: plane p adds ws[p-o]*u to outputs o = p-R..p+R, its in-plane
@@ -866,7 +829,7 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
         if (j >= 2 * R) {
           const int po = p - R;
           double ip[NCB][NCA], cen[NCB][NCA];
-          star_inplane(C, plane_ld(SL(j - R), po), la, lb, ip, cen);
+          star_inplane(C, plane_ld((j - R) % NP, po), la, lb, ip, cen);
 #pragma unroll
           for (int ib = 0; ib < NCB; ++ib)
 #pragma unroll
@@ -915,7 +878,7 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
             for (int ia = 0; ia < NCA; ++ia) S[0][ib][ia] = 0.0;
           static_for<0, W>([&](auto QQ) {
             constexpr int ds = decltype(QQ)::value - R;
-            box_slices<1, ds, 0>(C, plane_ld(SL(j - R + ds), po + ds), la, lb, S);
+            box_slices<1, ds, 0>(C, plane_ld((j - R + ds) % NP, po + ds), la, lb, S);
           });
 #pragma unroll
           for (int ib = 0; ib < NCB; ++ib)
@@ -930,17 +893,17 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
         // per-warp release on an "empty" mbarrier; only the producer waits (experimental)
         if (j >= RETAIN) {
           __syncwarp();
-          if ((tid & 31) == 0) mbar_arrive(&bars[NP + SL(j - RETAIN)]);
+          if ((tid & 31) == 0) mbar_arrive(&bars[NP + (j - RETAIN) % NP]);
         }
         if (tid == 0 && j + D < n_planes) {
-          const int jn = j + D, sl = SL(jn);
-          if (J0 + jn >= NP) mbar_wait(&bars[NP + sl], (u32)(((J0 + jn) / NP - 1) & 1));
+          const int jn = j + D, sl = jn % NP;
+          if (jn >= NP) mbar_wait(&bars[NP + sl], (u32)((jn / NP - 1) & 1));
 #else
         // CTA barrier: every warp is done with the slot of plane j - RETAIN, which is then
         // refilled with plane j + D
         __syncthreads();
         if (tid == 0 && j + D < n_planes) {
-          const int sl = SL(j + D);
+          const int sl = (j + D) % NP;
 #endif
           fence_proxy_async();
           mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
@@ -949,7 +912,7 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
       } else if constexpr (STAGING == 2) {
         __syncthreads();
         if (j + 1 < n_planes) {
-          double* dst = smem + SL(j + 1) * NIN * SLOT;
+          double* dst = smem + ((j + 1) % NP) * NIN * SLOT;
           if constexpr (D == 1) {
             ldst_plane(P, g, dst, p + 1);
           } else {
@@ -974,8 +937,6 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
       }
     });
   }
-  J0 += n_planes;
-  }  // units
 }
 
 
@@ -1117,9 +1078,11 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   Ctx C{P};
   constexpr int D = PF;
   constexpr int NP = STAGING == 1 ? 1 : NP1;
+  const SGeo g = stream_geo(P);
   const int ta = thread_x();
   const int tb = SZ ? thread_y() : thread_z();
   const int tid = threadIdx.x;
+  const int n_planes = (g.s_end - g.s_start) + 2 * R;
   u64* bars = (u64*)(smem + NP * NIN * SLOT);
 
   int la[NCA], lb[NCB];
@@ -1127,32 +1090,12 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   for (int i = 0; i < NCA; ++i) la[i] = merged_pos(i, ta, TBA, BMA);
 #pragma unroll
   for (int i = 0; i < NCB; ++i) lb[i] = merged_pos(i, tb, TBB, BMB);
+  const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
 
   // streamed-direction weights ws[k] = -sign(k) dxinv_s a_|k| (host-precomputed, in the
   // constant bank after the 7 user coefficients: 8 for s = z, then 8 for s = y):
   // plane p contributes ws[p-o] * E_f(p) to flux_f(o)
   auto ws = [&](int k) { return C.coef(7 + (DS == 1 ? 8 : 0) + (k < 0 ? k + R : k + R - 1)); };
-
-  if constexpr (STAGING == 3) {
-    if (tid == 0) {
-      for (int s = 0; s < NP; ++s) {
-        mbar_init(&bars[s], 1);  // full: producer arrive + TMA bytes
-#if CST_EMPTY_BARRIERS
-        mbar_init(&bars[NP + s], NTHR / 32);  // empty: one arrive per warp
-#endif
-      }
-      fence_mbar_init();
-    }
-    __syncthreads();
-  }
-  int J0 = 0;  // planes of this CTA's earlier units (ring slot / phase continuity)
-  auto SL = [&](int x) { return (J0 + x) % NP; };
-  auto PH = [&](int x) { return (u32)(((J0 + x) / NP) & 1); };
-  const int nu = n_units(P);
-  for (int unit = unit_first(); unit < nu; unit += unit_stride()) {
-  const SGeo g = stream_geo_unit(P, unit);
-  const int n_planes = (g.s_end - g.s_start) + 2 * R;
-  const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
 
   double acc[5][NCB][NCA][W];  // retimed: pending fluxes ; gather: queue of E_f
 #pragma unroll
@@ -1167,14 +1110,23 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   double frag[D > 1 && STAGING == 2 ? (D - 1) * FR : 1];
   if constexpr (STAGING == 3) {
     if (tid == 0) {
-      fence_proxy_async();  // slots last read by the previous unit's generic loads
+      for (int s = 0; s < NP; ++s) {
+        mbar_init(&bars[s], 1);  // full: producer arrive + TMA bytes
+#if CST_EMPTY_BARRIERS
+        mbar_init(&bars[NP + s], NTHR / 32);  // empty: one arrive per warp
+#endif
+      }
+      fence_mbar_init();
+    }
+    __syncthreads();
+    if (tid == 0) {
       for (int j = 0; j < D && j < n_planes; ++j) {
-        mbar_arrive_expect_tx(&bars[SL(j)], NIN * PL * 8);
-        tma_plane(P, g, smem + SL(j) * NIN * SLOT, &bars[SL(j)], g.s_start - R + j);
+        mbar_arrive_expect_tx(&bars[j % NP], NIN * PL * 8);
+        tma_plane(P, g, smem + (j % NP) * NIN * SLOT, &bars[j % NP], g.s_start - R + j);
       }
     }
   } else if constexpr (STAGING == 2) {
-    ldst_plane(P, g, smem + SL(0) * NIN * SLOT, g.s_start - R);
+    ldst_plane(P, g, smem, g.s_start - R);
     if constexpr (D > 1) {
 #pragma unroll
       for (int f = 0; f < D - 1; ++f)
@@ -1213,8 +1165,8 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
       const int j = j0 + u;
       if (j >= n_planes) return;
       const int p = g.s_start - R + j;
-      const int slot = SL(j);
-      if constexpr (STAGING == 3) mbar_wait(&bars[slot], PH(j));
+      const int slot = j % NP;
+      if constexpr (STAGING == 3) mbar_wait(&bars[slot], (u32)((j / NP) & 1));
       LDT ld[NIN];
       loaders(slot, p, ld);
       if constexpr (RETIME) {
@@ -1285,7 +1237,7 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
         if (j >= 2 * R) {
           const int po = p - R;
           LDT ldo[NIN];
-          loaders(SL(j - R), po, ldo);
+          loaders((j - R) % NP, po, ldo);
           double ta_[5][NCB][NCA], tb_[5][NCB][NCA];
           hyp_inplane<0>(C, ldo, la, lb, ta_);
           hyp_inplane<1>(C, ldo, la, lb, tb_);
@@ -1316,17 +1268,17 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
         // per-warp release on an "empty" mbarrier; only the producer waits (experimental)
         if (j >= RETAIN) {
           __syncwarp();
-          if ((tid & 31) == 0) mbar_arrive(&bars[NP + SL(j - RETAIN)]);
+          if ((tid & 31) == 0) mbar_arrive(&bars[NP + (j - RETAIN) % NP]);
         }
         if (tid == 0 && j + D < n_planes) {
-          const int jn = j + D, sl = SL(jn);
-          if (J0 + jn >= NP) mbar_wait(&bars[NP + sl], (u32)(((J0 + jn) / NP - 1) & 1));
+          const int jn = j + D, sl = jn % NP;
+          if (jn >= NP) mbar_wait(&bars[NP + sl], (u32)((jn / NP - 1) & 1));
 #else
         // CTA barrier: every warp is done with the slot of plane j - RETAIN, which is then
         // refilled with plane j + D
         __syncthreads();
         if (tid == 0 && j + D < n_planes) {
-          const int sl = SL(j + D);
+          const int sl = (j + D) % NP;
 #endif
           fence_proxy_async();
           mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
@@ -1335,7 +1287,7 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
       } else if constexpr (STAGING == 2) {
         __syncthreads();
         if (j + 1 < n_planes) {
-          double* dst = smem + SL(j + 1) * NIN * SLOT;
+          double* dst = smem + ((j + 1) % NP) * NIN * SLOT;
           if constexpr (D == 1) {
             ldst_plane(P, g, dst, p + 1);
           } else {
@@ -1360,8 +1312,6 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
       }
     });
   }
-  J0 += n_planes;
-  }  // units
 }
 
 // =============================================================================
@@ -1853,16 +1803,12 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
   tmem_fence_after_sync();
   const u32 tq = *tslot + ((u32)((warp & 3) * 32) << 16) + (u32)((warp >> 2) * NPT * TM_PCOLS);
   auto ws = [&](int k) { return C.coef(star_ci(AX_S, k)); };
-  int J0 = 0;  // planes of this CTA's earlier units (ring slot / phase continuity)
-  const int nu = n_units(P);
-  for (int unit = unit_first(); unit < nu; unit += unit_stride()) {
-  const SGeo g = stream_geo_unit(P, unit);
+  const SGeo g = stream_geo(P);
   const int n_planes = (g.s_end - g.s_start) + 2 * R;
   const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
   if (tid == 0) {
-    fence_proxy_async();
     for (int j = 0; j < D && j < n_planes; ++j) {
-      const int sl = (J0 + j) % NP;
+      const int sl = j % NP;
       mbar_arrive_expect_tx(&bars[sl], PL * 8);
       tma_plane(P, g, smem + sl * SLOT, &bars[sl], g.s_start - R + j);
     }
@@ -1874,9 +1820,9 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
 #pragma unroll 1
   for (int j = 0; j < n_planes; ++j) {
     const int p = g.s_start - R + j;
-    const int slot = (J0 + j) % NP;
+    const int slot = j % NP;
     const int u = j % R;
-    mbar_wait(&bars[slot], (u32)(((J0 + j) / NP) & 1));
+    mbar_wait(&bars[slot], (u32)((j / NP) & 1));
     const SmemPlane ld{smem + slot * SLOT};
     const bool need_a = j >= R && j < n_planes - R;  // A(p) feeds an interior output
     u32 cu[R];  // column of u(p - R + m), m = 0..R-1: slot (j + m) mod R
@@ -1931,14 +1877,12 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
     tmem_wait_st();  // the next plane reads these slots
     __syncthreads();
     if (tid == 0 && j + D < n_planes) {
-      const int sl = (J0 + j + D) % NP;
+      const int sl = (j + D) % NP;
       fence_proxy_async();
       mbar_arrive_expect_tx(&bars[sl], PL * 8);
       tma_plane(P, g, smem + sl * SLOT, &bars[sl], p + D);
     }
   }
-  J0 += n_planes;
-  }  // units
   tmem_fence_before_sync();
   __syncthreads();
   tmem_fence_after_sync();

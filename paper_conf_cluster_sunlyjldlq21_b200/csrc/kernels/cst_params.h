@@ -28,8 +28,6 @@ struct __attribute__((aligned(64))) cst_kparams {
   int chunks;                        // streaming chunks (SB)
   int remote;                        // 1: every store also goes to rout[q] + same offset
   double* rout[CST_MAX_OUT];         // peer-mapped neighbour halo (fused z-slab exchange)
-  int units;                         // fast streaming paths: (tile, chunk) work units; 0 =
-                                     // one unit per CTA (grid = tiles x chunks)
 };
 
 #endif

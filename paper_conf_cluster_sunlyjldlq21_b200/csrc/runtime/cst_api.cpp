@@ -497,42 +497,8 @@ cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* 
   P.tiles_b = g.tiles_b;
   P.tiles_c = g.tiles_c;
   P.chunks = g.chunks;
-  // Persistent launch of the fast streaming paths (T_SD = 1 star / box / hypterm / TMEM
-  // star): resident CTAs walk the (tile, chunk) units in hardware order, so neighbouring
-  // tiles stream the same planes together and share halo rows through L2.
-  unsigned gx = g.grid_x, gy = g.grid_y;
-  P.units = 0;
-  int64_t Tsd = 1;
-  if (t[F_STREAM] == 2) {
-    const int sd = t[F_SD] - 1;
-    Tsd = (int64_t)t[F_TBX + sd] * t[F_BMX + sd] * t[F_CMX + sd];
-  }
-  const bool fast = t[F_STREAM] == 2 && Tsd == 1 && t[F_BT] == 1 && h->info.kind != CST_RHS4;
-  static const bool persist = [] {
-    const char* e = std::getenv("CST_PERSIST");
-    return !(e && e[0] == '0');
-  }();
-  if (fast && persist) {
-    int occ = v->occ;
-    if (t[F_QS] == 2) {
-      // the occupancy API reports 1 for kernels that allocate tensor memory; the SM holds
-      // 512 / columns of them (tools/tmem_occ.cu), within the register / smem limits
-      const int cols = tmem_cols_alloc(h->info.r, t);
-      const int regs = ((v->regs + 7) / 8) * 8;
-      const int by_regs = 65536 / std::max(1, regs * (int)g.threads);
-      const int by_smem = (228 * 1024) / (v->smem + 1024);
-      occ = std::max(1, std::min({512 / cols, by_regs, by_smem, 2048 / (int)g.threads}));
-    }
-    const int64_t nu = (int64_t)g.grid_x * g.grid_y;
-    const int64_t cap = (int64_t)occ * h->num_sms;
-    if (occ > 0 && h->num_sms > 0 && nu > cap) {
-      P.units = (int)nu;
-      gx = (unsigned)cap;
-      gy = 1;
-    }
-  }
   void* args[] = {&P};
-  st = cu_check(d->cuLaunchKernel(v->fn, gx, gy, 1, g.threads, 1, 1,
+  st = cu_check(d->cuLaunchKernel(v->fn, g.grid_x, g.grid_y, 1, g.threads, 1, 1,
                                   (unsigned)v->smem, (CUstream)stream, args, nullptr),
                 "cuLaunchKernel");
   if (st != CST_OK) return st;

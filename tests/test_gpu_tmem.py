@@ -87,7 +87,7 @@ def test_tmem_space_rule_and_default_unchanged():
     h = C.cst_stencil_create(1, 4, [1.0] * 25, g)
     try:
         assert C.cst_setting_default(h).qstore == 1
-        C.cst_setting_check(h, Q(bm_x=4, bm_y=4))
+        C.cst_setting_check(h, Q(bm_x=4, bm_y=4, tb_x=16))
         with pytest.raises(C.CstError):
             C.cst_setting_check(h, Q(staging=2))          # R15
     finally:
