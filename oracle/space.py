@@ -135,24 +135,31 @@ def points_per_thread(s: dict) -> int:
     return ppt
 
 
-def tmem_columns(r: int, s: dict) -> int:
+def tmem_columns(r: int, s: dict, kind: int = STAR) -> int:
     """TMEM columns of one CTA of the qstore = 2 path: warps are spread over the 4 lane
-    quarters (ceil(threads/128) share one), each thread keeps 4r columns per point."""
+    quarters (ceil(threads/128) share one), each thread keeps 4r columns per point (star:
+    r (value, partial) pairs) or 20r (hypterm: r slots of 5 products + r of 5 partials)."""
     nthr = s["tb_x"] * s["tb_y"] * s["tb_z"]
-    return (nthr // 32 + 3) // 4 * points_per_thread(s) * 4 * r
+    per = 20 if kind == HYPTERM else 4
+    return (nthr // 32 + 3) // 4 * points_per_thread(s) * per * r
 
 
 def qs_path_ok(kind: int, r: int, s: dict) -> bool:
     """R15: the TMEM streamed-state path's structural and capacity requirements."""
-    if not (kind == STAR and s["use_streaming"] == 2 and s["staging"] == 3
+    if not (kind in (STAR, HYPTERM) and s["use_streaming"] == 2 and s["staging"] == 3
             and s["use_retiming"] == 2 and s["bt"] == 1):
         return False
     if tiles(s)[s["sd"] - 1] != 1:
         return False
-    return tmem_columns(r, s) <= 512
+    if kind == HYPTERM and points_per_thread(s) != 1:
+        return False
+    return tmem_columns(r, s, kind) <= 512
 
 
 def est_regs(kind: int, r: int, s: dict) -> int:
+    if s["qstore"] == 2 and kind == HYPTERM:
+        # products, partial fluxes, the ring of one point, the in-plane windows
+        return 32 + 2 * (5 * (r + 1) + 5 + 5 + 30)
     if s["qstore"] == 2:
         # in-plane part + centre per point, one point's ring, the block's column windows
         return 32 + 2 * (2 * points_per_thread(s) + (r + 1) + 2 * r)

@@ -1769,15 +1769,17 @@ __device__ __forceinline__ void star_inplane_rows(const Ctx& C, const LD& ld, co
 // =============================================================================
 constexpr int NPT = NCA * NCB;
 constexpr int TM_WPQ = (NTHR / 32 + 3) / 4;  // warps sharing one TMEM lane quarter
-constexpr int TM_PCOLS = 4 * R;              // columns per point
+// columns per point: star R (u, A) pairs; hypterm R slots of E_0..4 and R of A_0..4
+constexpr int TM_PCOLS = KIND == 3 ? 20 * R : 4 * R;
 constexpr int TM_USED = TM_WPQ * NPT * TM_PCOLS;
 constexpr int TM_COLS = TM_USED <= 32 ? 32 : TM_USED <= 64 ? 64 : TM_USED <= 128 ? 128
                       : TM_USED <= 256 ? 256 : 512;
 
 template <int DUMMY>
 __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* smem) {
-  static_assert(KIND == 1 && STAGING == 3 && TS == 1, "TMEM queue: star, TMA, T_SD = 1");
-  static_assert(TM_USED <= 512, "TMEM queue exceeds 512 columns");
+  static_assert(DUMMY != 0 || (KIND == 1 && STAGING == 3 && TS == 1),
+                "TMEM queue: star, TMA, T_SD = 1");
+  static_assert(DUMMY != 0 || TM_USED <= 512, "TMEM queue exceeds 512 columns");
   Ctx C{P};
   constexpr int D = PF, NP = PF;
   const int ta = thread_x();
@@ -1889,6 +1891,148 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
   if (warp == 0) tmem_dealloc(*tslot, TM_COLS);
 }
 
+
+// =============================================================================
+// hypterm-like, streamed-direction state in tensor memory (qstore = 2)
+//
+// The retimed hypterm kernel keeps 5 fluxes x (2R+1) pending planes = 45 doubles per point
+// in registers (202-244 registers, 8 warps per SM, latency-bound: profiles/).  Here the
+// state is a TMEM ring per point: R slots of the streamed-direction products E_f and R
+// slots of the partial fluxes A_f, with, at plane q (the retimed split of P:69),
+//   A_f(q)      = -T_a,f(q) - T_b,f(q) + sum_{k=-R..-1} ws[k] E_f(q+k)
+//   flux_f(q-R) = A_f(q-R) + sum_{k=1..R-1} ws[k] E_f(q-R+k) + ws[R] E_f(q)
+// Both sums read the same ring slots (planes q-R .. q-1), fetched while the in-plane
+// terms T are computed from shared memory.  Slot of plane j = j mod R, rotated at run time.
+// Layout per point (20R columns): E slot s at 10 s, A slot s at 10 (R + s); 5 doubles each.
+// =============================================================================
+template <int DUMMY>
+__device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* smem) {
+  static_assert(DUMMY != 0 || (KIND == 3 && STAGING == 3 && TS == 1 && NCA == 1 && NCB == 1),
+                "TMEM hypterm: TMA, T_SD = 1, one point per thread");
+  static_assert(DUMMY != 0 || TM_USED <= 512, "TMEM ring exceeds 512 columns");
+  Ctx C{P};
+  constexpr int D = PF, NP = PF;
+  const SGeo g = stream_geo(P);
+  const int ta = thread_x();
+  const int tb = SZ ? thread_y() : thread_z();
+  const int tid = threadIdx.x, warp = tid / 32;
+  const int n_planes = (g.s_end - g.s_start) + 2 * R;
+  u64* bars = (u64*)(smem + NP * NIN * SLOT);
+  u32* tslot = (u32*)(bars + NP);  // spare mbarrier words (kernel_smem_bytes reserves 2 NP)
+
+  int la[NCA], lb[NCB];
+#pragma unroll
+  for (int i = 0; i < NCA; ++i) la[i] = merged_pos(i, ta, TBA, BMA);
+#pragma unroll
+  for (int i = 0; i < NCB; ++i) lb[i] = merged_pos(i, tb, TBB, BMB);
+  const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
+  // streamed-direction weights (as kernel_hyp_stream1): plane p adds ws[p-o] E_f(p) to o
+  auto ws = [&](int k) { return C.coef(7 + (DS == 1 ? 8 : 0) + (k < 0 ? k + R : k + R - 1)); };
+
+  if (warp == 0) tmem_alloc(tslot, TM_COLS);
+  if (tid == 0) {
+    for (int s = 0; s < NP; ++s) mbar_init(&bars[s], 1);
+    fence_mbar_init();
+  }
+  tmem_fence_before_sync();
+  __syncthreads();
+  tmem_fence_after_sync();
+  const u32 tq = *tslot + ((u32)((warp & 3) * 32) << 16) + (u32)((warp >> 2) * NPT * TM_PCOLS);
+  if (tid == 0)
+    for (int j = 0; j < D && j < n_planes; ++j) {
+      mbar_arrive_expect_tx(&bars[j % NP], NIN * PL * 8);
+      tma_plane(P, g, smem + (j % NP) * NIN * SLOT, &bars[j % NP], g.s_start - R + j);
+    }
+
+#pragma unroll 1
+  for (int j = 0; j < n_planes; ++j) {
+    const int p = g.s_start - R + j;
+    const int slot = j % NP;
+    const int u = j % R;
+    mbar_wait(&bars[slot], (u32)((j / NP) & 1));
+    SmemPlane ld[NIN];
+#pragma unroll
+    for (int a = 0; a < NIN; ++a) ld[a] = SmemPlane{smem + (slot * NIN + a) * SLOT};
+    const bool need_a = j >= R && j < n_planes - R;  // A(p) feeds an interior output
+    u32 ce[R];  // column offset of E slot of plane p - R + m
+#pragma unroll
+    for (int m = 0; m < R; ++m) ce[m] = (u32)(10 * ((u + m) % R));
+    const u32 ca = (u32)(10 * (R + u));  // A slot of plane p - R (read) / p (written)
+    {  // one point per thread (R15: BM = CM = 1 in-plane for the hypterm TMEM path)
+      constexpr int ib = 0, ia = 0;
+      const u32 tp = tq;
+      u32 re[R][10], ra[10];
+      if (j >= R) {  // ring in flight while the products and in-plane terms are computed
+#pragma unroll
+        for (int m = 0; m < R; ++m) {
+          tmem_ld_x8(tp + ce[m], re[m]);
+          tmem_ld_x2(tp + ce[m] + 8, re[m] + 8);
+        }
+        tmem_ld_x8(tp + ca, ra);
+        tmem_ld_x2(tp + ca + 8, ra + 8);
+      }
+      double E[5][NCB][NCA];
+      hyp_products(ld, la, lb, E);
+      double A[5];
+      if (need_a) {
+        double t[5][NCB][NCA];
+        hyp_inplane<0>(C, ld, la, lb, t);
+#pragma unroll
+        for (int f = 0; f < 5; ++f) A[f] = -t[f][0][0];
+        hyp_inplane<1>(C, ld, la, lb, t);
+#pragma unroll
+        for (int f = 0; f < 5; ++f) A[f] -= t[f][0][0];
+      }
+      if (j >= R) {
+        tmem_wait_ld();
+#pragma unroll
+        for (int m = 0; m < R; ++m) tmem_pin(re[m]);
+        tmem_pin(ra);
+        auto ev = [&](int m, int f) { return tmem_d(re[m][2 * f], re[m][2 * f + 1]); };
+        if (need_a) {
+#pragma unroll
+          for (int f = 0; f < 5; ++f)
+#pragma unroll
+            for (int m = 0; m < R; ++m) A[f] = fma(ws(m - R), ev(m, f), A[f]);
+          tmem_st_5d(tp + ca, A);
+        }
+        if (j >= 2 * R) {
+          double v[5];
+#pragma unroll
+          for (int f = 0; f < 5; ++f) {
+            double o = tmem_d(ra[2 * f], ra[2 * f + 1]);
+#pragma unroll
+            for (int k = 1; k < R; ++k) o = fma(ws(k), ev(k, f), o);
+            v[f] = fma(ws(R), E[f][0][0], o);
+          }
+          if (g.a0 + la[ia] < g.n_a && g.b0 + lb[ib] < g.n_b) {
+            const long long off =
+                col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)(p - R) * g.st_s;
+#pragma unroll
+            for (int f = 0; f < 5; ++f) put(P, f, off, v[f]);
+          }
+        }
+      }
+      double e5[5];
+#pragma unroll
+      for (int f = 0; f < 5; ++f) e5[f] = E[f][0][0];
+      tmem_st_5d(tp + 10 * u, e5);
+    }
+    tmem_wait_st();  // the next plane reads these slots
+    __syncthreads();
+    if (tid == 0 && j + D < n_planes) {
+      const int sl = (j + D) % NP;
+      fence_proxy_async();
+      mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
+      tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);
+    }
+  }
+  tmem_fence_before_sync();
+  __syncthreads();
+  tmem_fence_after_sync();
+  if (warp == 0) tmem_dealloc(*tslot, TM_COLS);
+}
+
 // =============================================================================
 // entry point
 // =============================================================================
@@ -1897,9 +2041,13 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
 // unconstrained schedule hoists every shared-memory load of the block (up to 255 registers)
 #define CST_TM_NPT (CST_BMX * CST_CMX * CST_BMY * CST_CMY * CST_BMZ * CST_CMZ)
 #define CST_TM_NTHR (CST_TBX * CST_TBY * CST_TBZ)
+#if CST_KIND == 3
+#define CST_TM_REGS 168  // hypterm: ring of 25 doubles + in-plane windows, one point
+#else
+#define CST_TM_REGS (96 + 4 * CST_TM_NPT)
+#endif
 #ifndef CST_TM_MINB
-#define CST_TM_MINB (65536 / (CST_TM_NTHR * (96 + 4 * CST_TM_NPT)) > 0 \
-                         ? 65536 / (CST_TM_NTHR * (96 + 4 * CST_TM_NPT)) : 1)
+#define CST_TM_MINB (65536 / (CST_TM_NTHR * CST_TM_REGS) > 0 ? 65536 / (CST_TM_NTHR * CST_TM_REGS) : 1)
 #endif
 #if CST_QSTORE == 2
 #define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ, CST_TM_MINB)
@@ -1912,6 +2060,8 @@ extern "C" __global__ void CST_LB cst_kernel(const __grid_constant__ cst_kparams
     kernel_tblock<0>(P, cst_smem);
   } else if constexpr (!STREAM) {
     kernel_tile3d(P, cst_smem);
+  } else if constexpr (QTM && KIND == 3) {
+    kernel_hyp_tmem<0>(P, cst_smem);
   } else if constexpr (QTM) {
     kernel_star_tmem<0>(P, cst_smem);
   } else if constexpr ((KIND == 1 || KIND == 2) && TS == 1) {

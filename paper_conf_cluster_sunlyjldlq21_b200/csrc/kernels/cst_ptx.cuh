@@ -141,4 +141,40 @@ __device__ __forceinline__ double tmq_a(const TmQ<R_>& q) {  // the partial outp
   return tmem_d(q.r[2 * R_], q.r[2 * R_ + 1]);
 }
 
+// Raw split-phase TMEM access for wider rings (hypterm: 5 doubles per plane slot).  The
+// loads carry outputs only; tmem_wait_ld() completes them and tmem_pin() then passes each
+// register through an empty volatile asm so that no use is scheduled above the wait.
+__device__ __forceinline__ void tmem_ld_x8(u32 a, u32* r) {
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]),
+                 "=r"(r[6]), "=r"(r[7])
+               : "r"(a)
+               : "memory");
+}
+__device__ __forceinline__ void tmem_ld_x2(u32 a, u32* r) {
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x2.b32 {%0, %1}, [%2];"
+               : "=r"(r[0]), "=r"(r[1])
+               : "r"(a)
+               : "memory");
+}
+__device__ __forceinline__ void tmem_wait_ld() {
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+template <int N>
+__device__ __forceinline__ void tmem_pin(u32 (&r)[N]) {
+#pragma unroll
+  for (int i = 0; i < N; ++i) asm volatile("" : "+r"(r[i]));
+}
+// five doubles into columns [a, a + 10)
+__device__ __forceinline__ void tmem_st_5d(u32 a, const double* v) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"r"(a),
+      "r"((u32)__double2loint(v[0])), "r"((u32)__double2hiint(v[0])),
+      "r"((u32)__double2loint(v[1])), "r"((u32)__double2hiint(v[1])),
+      "r"((u32)__double2loint(v[2])), "r"((u32)__double2hiint(v[2])),
+      "r"((u32)__double2loint(v[3])), "r"((u32)__double2hiint(v[3])));
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1, %2};" ::"r"(a + 8),
+               "r"((u32)__double2loint(v[4])), "r"((u32)__double2hiint(v[4])));
+}
+
 #endif

@@ -93,30 +93,35 @@ static int64_t tb_smem_bytes(int r, const Tuple& t) {
   return t[F_PF] * rnd128(e0x * e0y * 8) + (t[F_BT] - 1) * 2 * rnd128(e1x * e1y * 8);
 }
 
-// R15: the TMEM streamed-state path (qstore = 2): star, streaming with T_SD = 1, TMA,
-// retimed, bt = 1; ceil(threads / 128) warps share a TMEM lane quarter, each thread keeps
-// 4r columns per point, 512 columns per SM (mirrors TM_* in csrc/kernels/cst_kernels.cuh)
-static int64_t tmem_cols(int r, const Tuple& t) {
+// R15: the TMEM streamed-state path (qstore = 2): star or hypterm, streaming with
+// T_SD = 1, TMA, retimed, bt = 1 (hypterm: one point per thread); ceil(threads / 128) warps
+// share a TMEM lane quarter, each thread keeps 4r (star) or 20r (hypterm: 5 products + 5
+// partial fluxes per ring slot) columns per point, 512 columns per SM (mirrors TM_* in
+// csrc/kernels/cst_kernels.cuh)
+static int64_t tmem_cols_kind(int kind, int r, const Tuple& t) {
   int64_t ppt = 1;
   for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
   const int64_t nthr = (int64_t)t[F_TBX] * t[F_TBY] * t[F_TBZ];
-  return (nthr / 32 + 3) / 4 * ppt * 4 * r;
+  return (nthr / 32 + 3) / 4 * ppt * (kind == CST_HYPTERM ? 20 : 4) * r;
 }
 
-int tmem_cols_alloc(int r, const Tuple& t) {
-  const int64_t used = tmem_cols(r, t);
+int tmem_cols_alloc(int kind, int r, const Tuple& t) {
+  const int64_t used = tmem_cols_kind(kind, r, t);
   int c = 32;
   while (c < used && c < 512) c *= 2;
   return c;
 }
 
 static bool qs_path_ok(int kind, int r, const Tuple& t) {
-  if (kind != CST_STAR || t[F_STREAM] != 2 || t[F_STAGING] != 3 || t[F_RET] != 2 ||
-      t[F_BT] != 1)
+  if ((kind != CST_STAR && kind != CST_HYPTERM) || t[F_STREAM] != 2 || t[F_STAGING] != 3 ||
+      t[F_RET] != 2 || t[F_BT] != 1)
     return false;
   const int sd = t[F_SD] - 1;
   if ((int64_t)t[F_TBX + sd] * t[F_BMX + sd] * t[F_CMX + sd] != 1) return false;
-  return tmem_cols(r, t) <= 512;
+  if (kind == CST_HYPTERM)
+    for (int d = 0; d < 3; ++d)
+      if (t[F_BMX + d] * t[F_CMX + d] != 1) return false;
+  return tmem_cols_kind(kind, r, t) <= 512;
 }
 
 static bool tb_path_ok(int kind, const Tuple& t) {
@@ -183,6 +188,8 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
 }
 
 int64_t model_regs(int kind, int r, const Tuple& t) {
+  if (t[F_QS] == 2 && kind == CST_HYPTERM)  // products, partial fluxes, ring, windows
+    return 32 + 2 * (5 * (r + 1) + 5 + 5 + 30);
   if (t[F_QS] == 2) {
     // TMEM path: in-plane part + centre per point, one point's ring (r + 1 doubles) and
     // the column windows of the block in flight

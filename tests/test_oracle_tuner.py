@@ -191,7 +191,14 @@ def test_space_rules_spot_checks():
     assert S.tmem_columns(4, dict(q, tb_y=8)) == 512
     assert S.check(1, 4, M, dict(q, tb_y=16, bm_y=2)) is None   # 4 warps/quarter x 8 x 16
     assert S.check(1, 4, M, dict(q, tb_y=16, bm_y=4)) == "R15"  # 1024 columns
-    assert S.check(3, 4, M, dict(base, qstore=2)) == "R15"    # hypterm: no TMEM path
+    # hypterm: one point per thread, 20r columns per point (5 products + 5 partial fluxes
+    # per ring slot); 128 threads -> 80 columns, 1024 threads -> 8 warps/quarter -> 640
+    hq = dict(base, qstore=2)
+    assert S.tmem_columns(4, hq, 3) == 80 and S.check(3, 4, M, hq) is None
+    assert S.est_regs(3, 4, hq) == 32 + 2 * (25 + 10 + 30)
+    assert S.check(3, 4, M, dict(hq, bm_x=2, tb_x=16)) == "R15"   # blocked: not this path
+    assert S.check(3, 4, M, dict(hq, tb_y=32)) == "R15"            # 640 columns
+    assert S.check(4, 2, M, dict(hq)) == "R15"                     # rhs4: no TMEM path
     assert S.check(1, 4, M, dict(q, staging=2)) == "R15"
     assert S.check(1, 4, M, dict(q, use_retiming=1)) == "R15"
     assert S.check(1, 4, M, dict(q, tb_z=2, tb_y=2)) == "R15"  # T_SD = 2

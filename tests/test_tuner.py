@@ -175,7 +175,13 @@ def test_ga_properties(tuned, space_list, tmp_path):
 
 def test_ga_finds_near_optimum_with_full_sampling(tmp_path, space_list):
     """With the whole space kept (ratio 1) the grouped GA must land within 10 % of the
-    brute-force optimum of the synthetic objective (Fig. 4: top-10 within 96.7 %)."""
-    best, rep, log, count = run_tuner(tmp_path, seed=11, ratio=1.0)
+    brute-force optimum of the synthetic objective (Fig. 4: top-10 within 96.7 %).  The GA
+    is stochastic: over four seeds at least three must be within 10 % and none beyond 15 %."""
     opt = min(synth(d)[0] for d in space_list)
-    assert rep.best_ms <= 1.10 * opt, (rep.best_ms, opt)
+    ratios = []
+    for seed in (11, 12, 13, 14):
+        d = tmp_path / f"s{seed}"
+        d.mkdir()
+        best, rep, log, count = run_tuner(d, seed=seed, ratio=1.0)
+        ratios.append(rep.best_ms / opt)
+    assert sum(q <= 1.10 for q in ratios) >= 3 and max(ratios) <= 1.15, ratios
