@@ -599,11 +599,47 @@ __device__ __forceinline__ void load_centres(const LD& ld, const int* la, const 
 // of its row and y-terms of the rows within R — so no per-point temporaries stay live.
 // Logical accumulator m of a point = output plane p - R + m (phys (m + U) % W); the
 // in-plane part belongs to m = R.
+// Paired b-rows (shared-memory traffic of the y-windows): with TB_x = 16 a warp holds two
+// b-row groups of the tile (lanes 0-15 and 16-31, g = tb & 1).  Instead of each lane
+// loading its own 2R halo rows (every lane a distinct address: 4 wavefronts per LDS.128),
+// all lanes load the union of both groups' rows, row by row with the same address in the
+// two groups (2 wavefronts), and each lane then selects its rows (shift BM_b * g).
+// 2 BM_b + 2R row loads at half cost replace 2R at full cost: -40 % of the y-window
+// wavefronts at BM_b = 2, for 2R double2 selects.  Arithmetic and its order unchanged.
+constexpr bool PAIR_ROWS = KIND == 1 && BMA == 2 && CMA == 1 && CMB == 1 && TBA == 16 &&
+                           TBB % 2 == 0 && STAGING >= 2;
+
+template <class LD>
+__device__ __forceinline__ void load_pair_halo(const LD& ld, int la0, int lb0,
+                                               double (&top)[R][2], double (&bot)[R][2],
+                                               double (&mid)[BMB][2]) {
+  const int g = (SZ ? thread_y() : thread_z()) & 1;
+  const int bw = lb0 - BMB * g;  // group 0's first block row
+  constexpr int NR = 2 * BMB + 2 * R;
+  double2 v[NR];  // rows bw - R .. bw + 2 BMB + R - 1
+#pragma unroll
+  for (int i = 0; i < NR; ++i) v[i] = ld.at2(la0, bw - R + i);
+#pragma unroll
+  for (int t = 0; t < R; ++t) {
+    const double2 a = g ? v[BMB + t] : v[t];                  // row lb0 - R + t
+    const double2 b = g ? v[2 * BMB + R + t] : v[BMB + R + t];  // row lb0 + BMB + t
+    top[t][0] = a.x; top[t][1] = a.y;
+    bot[t][0] = b.x; bot[t][1] = b.y;
+  }
+#pragma unroll
+  for (int t = 0; t < BMB; ++t) {  // the block rows' own pair (centre of their x-window)
+    const double2 c = g ? v[BMB + R + t] : v[R + t];
+    mid[t][0] = c.x; mid[t][1] = c.y;
+  }
+}
+
 template <int U, class LD>
 __device__ __forceinline__ void star_retimed_plane(const Ctx& C, const LD& ld, const int* la,
                                                    const int* lb,
                                                    double (&acc)[NCB][NCA][W]) {
   constexpr int MR = (R + U) % W;
+  double top[R][2], bot[R][2], mid[BMB][2];
+  if constexpr (PAIR_ROWS && LD::VEC) load_pair_halo(ld, la[0], lb[0], top, bot, mid);
 #pragma unroll
   for (int cb = 0; cb < CMB; ++cb) {
     const int lb0 = lb[cb * BMB];
@@ -614,7 +650,21 @@ __device__ __forceinline__ void star_retimed_plane(const Ctx& C, const LD& ld, c
       for (int wr = -R; wr < BMB + R; ++wr) {
         if (wr >= 0 && wr < BMB) {
           double w[BMA + 2 * XR];
-          load_xwin(ld, la0, lb0 + wr, w);
+          if constexpr (PAIR_ROWS && LD::VEC) {  // centre pair from the shared rows
+#pragma unroll
+            for (int q = 0; q < BMA / 2 + XR; ++q) {
+              if (q == XR / 2) {
+                w[XR] = mid[wr][0];
+                w[XR + 1] = mid[wr][1];
+                continue;
+              }
+              const double2 t = ld.at2(la0 - XR + 2 * q, lb0 + wr);
+              w[2 * q] = t.x;
+              w[2 * q + 1] = t.y;
+            }
+          } else {
+            load_xwin(ld, la0, lb0 + wr, w);
+          }
 #pragma unroll
           for (int b = 0; b < BMA; ++b) {
             double(&A)[W] = acc[cb * BMB + wr][ca * BMA + b];
@@ -637,7 +687,10 @@ __device__ __forceinline__ void star_retimed_plane(const Ctx& C, const LD& ld, c
           }
         } else {
           double v[BMA];
-          if constexpr (LD::VEC && (BMA % 2 == 0)) {
+          if constexpr (PAIR_ROWS && LD::VEC) {
+#pragma unroll
+            for (int b = 0; b < BMA; ++b) v[b] = wr < 0 ? top[wr + R][b] : bot[wr - BMB][b];
+          } else if constexpr (LD::VEC && (BMA % 2 == 0)) {
 #pragma unroll
             for (int b = 0; b < BMA; b += 2) {
               const double2 t = ld.at2(la0 + b, lb0 + wr);
@@ -951,10 +1004,25 @@ constexpr int DA = 0, DB = SZ ? 1 : 2, DS = SZ ? 2 : 1;  // direction (0 x, 1 y,
 
 // load a line of values through the point block: along a (x-window of row lb, starting
 // la - XR, length BMA + 2XR) or along b (column la, rows lb - R .., length BMB + 2R)
+// hypterm b-lines with paired b-rows (TB_a = 16: a warp = two b-row groups, g = tb & 1):
+// all lanes load rows bw - R .. bw + R + 1 (bw = group 0's row) with the same address in
+// both groups — one wavefront per load instead of two — and group 1 takes them shifted by
+// one.  2R + 2 half-cost loads replace 2R full-cost ones (-37 % of the b-line wavefronts).
+constexpr bool PAIR_B = KIND == 3 && TBA == 16 && TBB % 2 == 0 && BMA == 1 && BMB == 1 &&
+                        CMA == 1 && CMB == 1 && STAGING >= 2;
+
 template <int AXIS, class LD>
 __device__ __forceinline__ void load_line(const LD& ld, int la, int lb, double* w) {
   if constexpr (AXIS == 0) {
     load_xwin(ld, la, lb, w);
+  } else if constexpr (PAIR_B && LD::VEC) {
+    const int g = (SZ ? thread_y() : thread_z()) & 1;
+    const int bw = lb - g;
+    double v[2 * R + 2];
+#pragma unroll
+    for (int i = 0; i < 2 * R + 2; ++i) v[i] = ld.at(la, bw - R + i);  // both centres needed
+#pragma unroll
+    for (int q = 0; q < 2 * R + 1; ++q) w[q] = q == R ? 0.0 : (g ? v[q + 1] : v[q]);
   } else {
 #pragma unroll
     for (int q = 0; q < BMB + 2 * R; ++q) {
@@ -1838,19 +1906,32 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
       for (int m = 0; m < R; ++m) ta[m] = tp + cu[m];
       tmem_ld_issue<R>(ta, tp + 2 * R + cs, q);
     };
-    // the ring of point 0 is in flight while the in-plane part is computed; the ring of
-    // point pt + 1 while point pt is finished (one-deep TMEM load pipeline)
-    TmQ<R> q0, q1;
-    if (j >= R) issue(0, q0);
+    // TMEM loads in flight while the in-plane part is computed: every point's ring when
+    // they fit the register budget (TM_ALL), else point 0's, then point pt + 1's while
+    // point pt is finished (one-deep pipeline)
+    constexpr bool TM_ALL = NPT * (2 * R + 2) <= 48;
+    TmQ<R> qa[TM_ALL ? NPT : 2];
+    if (j >= R) {
+      if constexpr (TM_ALL) static_for<0, NPT>([&](auto PP) { issue(decltype(PP)::value, qa[decltype(PP)::value]); });
+      else issue(0, qa[0]);
+    }
     double ip[NCB][NCA], cen[NCB][NCA];
     if (need_a) star_inplane_rows(C, ld, la, lb, ip, cen);
     else load_centres(ld, la, lb, cen);
+    if constexpr (TM_ALL) {
+      if (j >= R) {
+        tmem_wait_ld();
+        static_for<0, NPT>([&](auto PP) { tmem_pin(qa[decltype(PP)::value].r); });
+      }
+    }
     auto finish = [&](auto PP, TmQ<R>& q, TmQ<R>& qn) {
       constexpr int pt = decltype(PP)::value, ib = pt / NCA, ia = pt % NCA;
       const u32 tp = tq + (u32)(pt * TM_PCOLS);
       if (j >= R) {
-        tmem_ld_wait<R>(q);
-        if constexpr (pt + 1 < NPT) issue(pt + 1, qn);
+        if constexpr (!TM_ALL) {
+          tmem_ld_wait<R>(q);
+          if constexpr (pt + 1 < NPT) issue(pt + 1, qn);
+        }
         if (need_a) {  // A(p) = ip(p) + sum_{k=-R..-1} ws[k] u(p+k)
           double a = ip[ib][ia];
 #pragma unroll
@@ -1873,8 +1954,10 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
       tmem_st_d(tp + cs, cen[ib][ia]);
     };
     static_for<0, NPT>([&](auto PP) {
-      if constexpr (decltype(PP)::value % 2 == 0) finish(PP, q0, q1);
-      else finish(PP, q1, q0);
+      constexpr int pt = decltype(PP)::value;
+      if constexpr (TM_ALL) finish(PP, qa[pt], qa[pt]);
+      else if constexpr (pt % 2 == 0) finish(PP, qa[0], qa[1]);
+      else finish(PP, qa[1], qa[0]);
     });
     tmem_wait_st();  // the next plane reads these slots
     __syncthreads();
@@ -2043,14 +2126,17 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 #define CST_TM_NTHR (CST_TBX * CST_TBY * CST_TBZ)
 #if CST_KIND == 3
 #define CST_TM_REGS 168  // hypterm: ring of 25 doubles + in-plane windows, one point
-#else
-#define CST_TM_REGS (96 + 4 * CST_TM_NPT)
+#else  // star: + every point's ring in flight when it fits 48 registers (TM_ALL)
+#define CST_TM_REGS (96 + 4 * CST_TM_NPT + \
+                     (CST_TM_NPT * (2 * CST_R + 2) <= 48 ? CST_TM_NPT * (2 * CST_R + 2) : 0))
 #endif
 #ifndef CST_TM_MINB
 #define CST_TM_MINB (65536 / (CST_TM_NTHR * CST_TM_REGS) > 0 ? 65536 / (CST_TM_NTHR * CST_TM_REGS) : 1)
 #endif
 #if CST_QSTORE == 2
 #define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ, CST_TM_MINB)
+#elif defined(CST_MINB)  // experiment hook (CST_NVRTC_DEFINES="-DCST_MINB=n")
+#define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ, CST_MINB)
 #else
 #define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ)
 #endif
