@@ -599,47 +599,11 @@ __device__ __forceinline__ void load_centres(const LD& ld, const int* la, const 
 // of its row and y-terms of the rows within R — so no per-point temporaries stay live.
 // Logical accumulator m of a point = output plane p - R + m (phys (m + U) % W); the
 // in-plane part belongs to m = R.
-// Paired b-rows (shared-memory traffic of the y-windows): with TB_x = 16 a warp holds two
-// b-row groups of the tile (lanes 0-15 and 16-31, g = tb & 1).  Instead of each lane
-// loading its own 2R halo rows (every lane a distinct address: 4 wavefronts per LDS.128),
-// all lanes load the union of both groups' rows, row by row with the same address in the
-// two groups (2 wavefronts), and each lane then selects its rows (shift BM_b * g).
-// 2 BM_b + 2R row loads at half cost replace 2R at full cost: -40 % of the y-window
-// wavefronts at BM_b = 2, for 2R double2 selects.  Arithmetic and its order unchanged.
-constexpr bool PAIR_ROWS = KIND == 1 && BMA == 2 && CMA == 1 && CMB == 1 && TBA == 16 &&
-                           TBB % 2 == 0 && STAGING >= 2;
-
-template <class LD>
-__device__ __forceinline__ void load_pair_halo(const LD& ld, int la0, int lb0,
-                                               double (&top)[R][2], double (&bot)[R][2],
-                                               double (&mid)[BMB][2]) {
-  const int g = (SZ ? thread_y() : thread_z()) & 1;
-  const int bw = lb0 - BMB * g;  // group 0's first block row
-  constexpr int NR = 2 * BMB + 2 * R;
-  double2 v[NR];  // rows bw - R .. bw + 2 BMB + R - 1
-#pragma unroll
-  for (int i = 0; i < NR; ++i) v[i] = ld.at2(la0, bw - R + i);
-#pragma unroll
-  for (int t = 0; t < R; ++t) {
-    const double2 a = g ? v[BMB + t] : v[t];                  // row lb0 - R + t
-    const double2 b = g ? v[2 * BMB + R + t] : v[BMB + R + t];  // row lb0 + BMB + t
-    top[t][0] = a.x; top[t][1] = a.y;
-    bot[t][0] = b.x; bot[t][1] = b.y;
-  }
-#pragma unroll
-  for (int t = 0; t < BMB; ++t) {  // the block rows' own pair (centre of their x-window)
-    const double2 c = g ? v[BMB + R + t] : v[R + t];
-    mid[t][0] = c.x; mid[t][1] = c.y;
-  }
-}
-
 template <int U, class LD>
 __device__ __forceinline__ void star_retimed_plane(const Ctx& C, const LD& ld, const int* la,
                                                    const int* lb,
                                                    double (&acc)[NCB][NCA][W]) {
   constexpr int MR = (R + U) % W;
-  double top[R][2], bot[R][2], mid[BMB][2];
-  if constexpr (PAIR_ROWS && LD::VEC) load_pair_halo(ld, la[0], lb[0], top, bot, mid);
 #pragma unroll
   for (int cb = 0; cb < CMB; ++cb) {
     const int lb0 = lb[cb * BMB];
@@ -650,21 +614,7 @@ __device__ __forceinline__ void star_retimed_plane(const Ctx& C, const LD& ld, c
       for (int wr = -R; wr < BMB + R; ++wr) {
         if (wr >= 0 && wr < BMB) {
           double w[BMA + 2 * XR];
-          if constexpr (PAIR_ROWS && LD::VEC) {  // centre pair from the shared rows
-#pragma unroll
-            for (int q = 0; q < BMA / 2 + XR; ++q) {
-              if (q == XR / 2) {
-                w[XR] = mid[wr][0];
-                w[XR + 1] = mid[wr][1];
-                continue;
-              }
-              const double2 t = ld.at2(la0 - XR + 2 * q, lb0 + wr);
-              w[2 * q] = t.x;
-              w[2 * q + 1] = t.y;
-            }
-          } else {
-            load_xwin(ld, la0, lb0 + wr, w);
-          }
+          load_xwin(ld, la0, lb0 + wr, w);
 #pragma unroll
           for (int b = 0; b < BMA; ++b) {
             double(&A)[W] = acc[cb * BMB + wr][ca * BMA + b];
@@ -687,10 +637,7 @@ __device__ __forceinline__ void star_retimed_plane(const Ctx& C, const LD& ld, c
           }
         } else {
           double v[BMA];
-          if constexpr (PAIR_ROWS && LD::VEC) {
-#pragma unroll
-            for (int b = 0; b < BMA; ++b) v[b] = wr < 0 ? top[wr + R][b] : bot[wr - BMB][b];
-          } else if constexpr (LD::VEC && (BMA % 2 == 0)) {
+          if constexpr (LD::VEC && (BMA % 2 == 0)) {
 #pragma unroll
             for (int b = 0; b < BMA; b += 2) {
               const double2 t = ld.at2(la0 + b, lb0 + wr);
@@ -1004,25 +951,10 @@ constexpr int DA = 0, DB = SZ ? 1 : 2, DS = SZ ? 2 : 1;  // direction (0 x, 1 y,
 
 // load a line of values through the point block: along a (x-window of row lb, starting
 // la - XR, length BMA + 2XR) or along b (column la, rows lb - R .., length BMB + 2R)
-// hypterm b-lines with paired b-rows (TB_a = 16: a warp = two b-row groups, g = tb & 1):
-// all lanes load rows bw - R .. bw + R + 1 (bw = group 0's row) with the same address in
-// both groups — one wavefront per load instead of two — and group 1 takes them shifted by
-// one.  2R + 2 half-cost loads replace 2R full-cost ones (-37 % of the b-line wavefronts).
-constexpr bool PAIR_B = KIND == 3 && TBA == 16 && TBB % 2 == 0 && BMA == 1 && BMB == 1 &&
-                        CMA == 1 && CMB == 1 && STAGING >= 2;
-
 template <int AXIS, class LD>
 __device__ __forceinline__ void load_line(const LD& ld, int la, int lb, double* w) {
   if constexpr (AXIS == 0) {
     load_xwin(ld, la, lb, w);
-  } else if constexpr (PAIR_B && LD::VEC) {
-    const int g = (SZ ? thread_y() : thread_z()) & 1;
-    const int bw = lb - g;
-    double v[2 * R + 2];
-#pragma unroll
-    for (int i = 0; i < 2 * R + 2; ++i) v[i] = ld.at(la, bw - R + i);  // both centres needed
-#pragma unroll
-    for (int q = 0; q < 2 * R + 1; ++q) w[q] = q == R ? 0.0 : (g ? v[q + 1] : v[q]);
   } else {
 #pragma unroll
     for (int q = 0; q < BMB + 2 * R; ++q) {

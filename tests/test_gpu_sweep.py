@@ -77,12 +77,8 @@ PATH_SETTINGS = [
     ("tile3d-tma", S(tb_x=16, tb_y=2, tb_z=2, staging=3, **NOSTREAM)),
     ("tile3d-tma-merge", S(tb_x=16, tb_y=2, tb_z=1, staging=3, bm_z=2, cm_y=2, uf_z=2, **NOSTREAM)),
     ("tile3d-retimed", S(tb_x=16, tb_y=2, tb_z=2, staging=2, use_retiming=2, **NOSTREAM)),
-    # paired b-rows (TB_x = 16, BM_x = 2): shared halo-row loads + per-group selection
-    ("pair-rows-tma", S(tb_x=16, tb_y=4, bm_x=2, bm_y=2)),
-    ("pair-rows-ldst", S(tb_x=16, tb_y=4, bm_x=2, bm_y=2, staging=2)),
-    ("pair-rows-bmy1", S(tb_x=16, tb_y=4, bm_x=2, bm_y=1)),
-    ("pair-rows-bmy4", S(tb_x=16, tb_y=2, bm_x=2, bm_y=4)),
-    ("pair-rows-sd-y", S(tb_x=16, tb_y=1, tb_z=4, sd=2, bm_x=2, bm_z=2)),
+    ("tb16-bm2x2", S(tb_x=16, tb_y=4, bm_x=2, bm_y=2)),
+    ("tb16-bm2x4", S(tb_x=16, tb_y=2, bm_x=2, bm_y=4)),
 ]
 
 
