@@ -366,11 +366,35 @@ def main():
     C.cst_fill_uniform(grid, u.data_ptr(), SEED, 0, N, N, z0, float("nan"), stream.cuda_stream)
     C.cst_fill_uniform(grid, v.data_ptr(), SEED, 0, N, N, z0, float("nan"), stream.cuda_stream)
     dist_h = None
+    halo_used = args.halo
     if world > 1 and args.halo == "p2p":
-        # boundary kernels store straight into the neighbours' halos (NVLink peer stores)
+        # boundary kernels store straight into the neighbours' halos (NVLink peer stores).
+        # Every rank must take the same transport: export, all-gather (ok, blob), import,
+        # agree by MIN-reduce; any failure anywhere -> all ranks fall back to NCCL.
         dist_h = C.cst_dist_create(h, world, rank, None)
-        C.cst_dist_p2p_setup(dist_h, rank, world, [u.data_ptr()], [v.data_ptr()])
-    elif world > 1:
+        ok, why, mine = True, "", None
+        try:
+            mine = C.cst_dist_p2p_export(dist_h, [u.data_ptr()], [v.data_ptr()])
+        except C.CstError as e:
+            ok, why = False, str(e)
+        blobs = [None] * world
+        dist.all_gather_object(blobs, (ok, mine))
+        if ok and all(b[0] for b in blobs):
+            try:
+                for peer in (rank - 1, rank + 1):
+                    if 0 <= peer < world:
+                        C.cst_dist_p2p_import(dist_h, peer, blobs[peer][1])
+            except C.CstError as e:
+                ok, why = False, str(e)
+        else:
+            ok, why = False, why or "a peer could not export"
+        flag = torch.tensor([1 if ok else 0], device="cuda")
+        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+        if int(flag.item()) == 0:
+            C.cst_dist_destroy(dist_h)
+            dist_h = None
+            halo_used = "nccl (p2p setup failed: %s)" % (why or "on another rank")[:120]
+    if world > 1 and dist_h is None:
         uid = C.cst_dist_nccl_unique_id() if rank == 0 else None
         obj = [uid]
         dist.broadcast_object_list(obj, src=0)
@@ -461,8 +485,9 @@ def main():
                 "config": {"workload": "star25: order-4 25-point star (FD Laplacian /5040), "
                                        "512^3 FP64 interior per GPU (BASELINE configs[1])"
                                        + (("; z-slab weak scaling, halo exchange: "
-                                           + ("fused peer-memory stores" if args.halo == "p2p"
-                                              else "NCCL send/recv")) if world > 1 else ""),
+                                           + ("fused peer-memory stores" if halo_used == "p2p"
+                                              else "NCCL send/recv" if halo_used == "nccl"
+                                              else halo_used)) if world > 1 else ""),
                            "grid": [N, N, N * world], "halo": R,
                            "setting": s.as_dict(), "setting_source": s_src,
                            "l2": "inputs larger than L2 (2 x %.2f GB per GPU), no flush"
