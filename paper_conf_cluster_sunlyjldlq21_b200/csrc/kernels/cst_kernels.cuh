@@ -31,6 +31,9 @@
 #ifndef CST_QSTORE
 #define CST_QSTORE 1  // streamed-direction state: 1 registers, 2 tensor memory (TMEM)
 #endif
+#ifndef CST_TM_LATE
+#define CST_TM_LATE 1  // hypterm TMEM ring loaded after the in-plane terms (measured best)
+#endif
 
 // ------------------------------------------------------------------ configuration
 constexpr int KIND = CST_KIND;  // 1 star, 2 box, 3 hypterm, 4 rhs4center-like
@@ -1977,7 +1980,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
       constexpr int ib = 0, ia = 0;
       const u32 tp = tq;
       u32 re[R][10], ra[10];
-      if (j >= R) {  // ring in flight while the products and in-plane terms are computed
+      auto issue_ring = [&]() {
 #pragma unroll
         for (int m = 0; m < R; ++m) {
           tmem_ld_x8(tp + ce[m], re[m]);
@@ -1985,7 +1988,10 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
         }
         tmem_ld_x8(tp + ca, ra);
         tmem_ld_x2(tp + ca + 8, ra + 8);
-      }
+      };
+      // CST_TM_LATE (experiment hook): issue the ring after the in-plane terms — 50 fewer
+      // live registers, the load latency then hidden by other warps only
+      if (!CST_TM_LATE && j >= R) issue_ring();  // in flight while products/T are computed
       double E[5][NCB][NCA];
       hyp_products(ld, la, lb, E);
       double A[5];
@@ -1999,6 +2005,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
         for (int f = 0; f < 5; ++f) A[f] -= t[f][0][0];
       }
       if (j >= R) {
+        if (CST_TM_LATE) issue_ring();
         tmem_wait_ld();
 #pragma unroll
         for (int m = 0; m < R; ++m) tmem_pin(re[m]);
@@ -2056,7 +2063,9 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 // unconstrained schedule hoists every shared-memory load of the block (up to 255 registers)
 #define CST_TM_NPT (CST_BMX * CST_CMX * CST_BMY * CST_CMY * CST_BMZ * CST_CMZ)
 #define CST_TM_NTHR (CST_TBX * CST_TBY * CST_TBZ)
-#if CST_KIND == 3
+#if CST_KIND == 3 && CST_TM_LATE
+#define CST_TM_REGS 120  // hypterm, ring loaded after the in-plane terms
+#elif CST_KIND == 3
 #define CST_TM_REGS 168  // hypterm: ring of 25 doubles + in-plane windows, one point
 #else  // star: + every point's ring in flight when it fits 48 registers (TM_ALL)
 #define CST_TM_REGS (96 + 4 * CST_TM_NPT + \
