@@ -31,6 +31,9 @@
 #ifndef CST_QSTORE
 #define CST_QSTORE 1  // streamed-direction state: 1 registers, 2 tensor memory (TMEM)
 #endif
+#ifndef CST_HYP_ROWS
+#define CST_HYP_ROWS 1  // TMEM hypterm: in-plane terms by row streaming
+#endif
 #ifndef CST_TM_LATE
 #define CST_TM_LATE 1  // hypterm TMEM ring loaded after the in-plane terms (measured best)
 #endif
@@ -406,6 +409,32 @@ constexpr int PA = TA + 2 * XR, PB = TB + 2 * R;
 constexpr int PL = PA * PB;
 constexpr int SLOT = round_slot(PL);
 
+// Per-array halos of the hypterm TMA fast path (HTRIM): each input is staged with only the
+// halos its terms read (Table III hypterm): cons1..4 and q4 enter the
+// derivatives along every direction (a- and b-halos), q_a only along a, q_b only along b,
+// q_s only through the streamed-direction products (no in-plane halo).  Every other path
+// stages NIN uniform (PA x PB) slots; the layout functions then reduce to a * SLOT.
+// Mirrored by the host (cst_api.cpp: TMA boxes; space.cpp: kernel_smem_bytes).
+constexpr bool HTRIM = KIND == 3 && STAGING == 3 && STREAM && TS == 1 && CST_BT == 1;
+constexpr int Q_A = 4, Q_B = SZ ? 5 : 6;  // q index of direction a (x) and b (y or z)
+__host__ __device__ constexpr bool arr_halo_a(int a) { return !HTRIM || a < 4 || a == 7 || a == Q_A; }
+__host__ __device__ constexpr bool arr_halo_b(int a) { return !HTRIM || a < 4 || a == 7 || a == Q_B; }
+__host__ __device__ constexpr int arr_wa(int a) { return TA + (arr_halo_a(a) ? 2 * XR : 0); }
+__host__ __device__ constexpr int arr_wb(int a) { return TB + (arr_halo_b(a) ? 2 * R : 0); }
+__host__ __device__ constexpr int arr_off(int a) {
+  int o = 0;
+  for (int i = 0; i < a; ++i) o += round_slot(arr_wa(i) * arr_wb(i));
+  return o;
+}
+__host__ __device__ constexpr int arr_txb(int n) {
+  int b = 0;
+  for (int i = 0; i < n; ++i) b += arr_wa(i) * arr_wb(i) * 8;
+  return b;
+}
+constexpr int RSLOT = arr_off(NIN);      // elements of one ring slot (all arrays)
+constexpr int TX_BYTES = arr_txb(NIN);   // TMA bytes of one plane (all arrays)
+static_assert(HTRIM || (RSLOT == NIN * SLOT && TX_BYTES == NIN * PL * 8), "uniform layout");
+
 struct SGeo {
   int n_a, n_b, n_s;
   long long st_b, st_s;  // element strides of b and s
@@ -432,12 +461,11 @@ __device__ __forceinline__ void tma_plane(const cst_kparams& P, const SGeo& g, d
                                           u64* bar, int p) {
 #pragma unroll
   for (int a = 0; a < NIN; ++a) {
+    const int oa = g.a0 - (arr_halo_a(a) ? XR : 0), ob = g.b0 - (arr_halo_b(a) ? R : 0);
     if constexpr (SZ)
-      tma_load_3d(dst + a * SLOT, &P.tma[a], bar, P.tox + g.a0 - XR, P.toy + g.b0 - R,
-                  P.toz + p);
+      tma_load_3d(dst + arr_off(a), &P.tma[a], bar, P.tox + oa, P.toy + ob, P.toz + p);
     else
-      tma_load_3d(dst + a * SLOT, &P.tma[a], bar, P.tox + g.a0 - XR, P.toy + p,
-                  P.toz + g.b0 - R);
+      tma_load_3d(dst + arr_off(a), &P.tma[a], bar, P.tox + oa, P.toy + p, P.toz + ob);
   }
 }
 
@@ -459,11 +487,18 @@ __device__ __forceinline__ void ldst_plane(const cst_kparams& P, const SGeo& g, 
 struct SmemPlane {
   static constexpr bool VEC = true;
   const double* base;  // slot base of one array
-  __device__ __forceinline__ double at(int la, int lb) const { return base[(lb + R) * PA + la + XR]; }
+  int pitch = PA;            // row pitch (elements)
+  int org = R * PA + XR;     // element offset of tile point (0, 0)
+  __device__ __forceinline__ double at(int la, int lb) const { return base[org + lb * pitch + la]; }
   __device__ __forceinline__ double2 at2(int la, int lb) const {
-    return *reinterpret_cast<const double2*>(base + (lb + R) * PA + la + XR);
+    return *reinterpret_cast<const double2*>(base + org + lb * pitch + la);
   }
 };
+// array a of the ring slot at `slot_base` (per-array layout; uniform unless HTRIM)
+__device__ __forceinline__ SmemPlane splane(const double* slot_base, int a) {
+  return SmemPlane{slot_base + arr_off(a), arr_wa(a),
+                   (arr_halo_b(a) ? R : 0) * arr_wa(a) + (arr_halo_a(a) ? XR : 0)};
+}
 struct GlobPlane {
   static constexpr bool VEC = false;
   const double* base;  // &u(a0, b0, p)
@@ -726,7 +761,7 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
   const int n_planes = (g.s_end - g.s_start) + 2 * R;
   const double* __restrict__ in = P.in[0];
   double* __restrict__ out = P.out[0];
-  u64* bars = (u64*)(smem + NP * NIN * SLOT);
+  u64* bars = (u64*)(smem + NP * RSLOT);
 
   int la[NCA], lb[NCB];
 #pragma unroll
@@ -760,8 +795,8 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
     __syncthreads();
     if (tid == 0) {
       for (int j = 0; j < D && j < n_planes; ++j) {
-        mbar_arrive_expect_tx(&bars[j % NP], NIN * PL * 8);
-        tma_plane(P, g, smem + (j % NP) * NIN * SLOT, &bars[j % NP], g.s_start - R + j);
+        mbar_arrive_expect_tx(&bars[j % NP], TX_BYTES);
+        tma_plane(P, g, smem + (j % NP) * RSLOT, &bars[j % NP], g.s_start - R + j);
       }
     }
   } else if constexpr (STAGING == 2) {
@@ -783,7 +818,7 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
     if constexpr (STAGING == 1)
       return GlobPlane{in + col0 + (long long)p * g.st_s, g.st_b};
     else
-      return SmemPlane{smem + slot * NIN * SLOT};
+      return SmemPlane{smem + slot * RSLOT};
   };
   auto store = [&](int ib, int ia, int po, double v) {
     if (g.a0 + la[ia] < g.n_a && g.b0 + lb[ib] < g.n_b)
@@ -909,13 +944,13 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
           const int sl = (j + D) % NP;
 #endif
           fence_proxy_async();
-          mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
-          tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);
+          mbar_arrive_expect_tx(&bars[sl], TX_BYTES);
+          tma_plane(P, g, smem + sl * RSLOT, &bars[sl], p + D);
         }
       } else if constexpr (STAGING == 2) {
         __syncthreads();
         if (j + 1 < n_planes) {
-          double* dst = smem + ((j + 1) % NP) * NIN * SLOT;
+          double* dst = smem + ((j + 1) % NP) * RSLOT;
           if constexpr (D == 1) {
             ldst_plane(P, g, dst, p + 1);
           } else {
@@ -1086,7 +1121,7 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   const int tb = SZ ? thread_y() : thread_z();
   const int tid = threadIdx.x;
   const int n_planes = (g.s_end - g.s_start) + 2 * R;
-  u64* bars = (u64*)(smem + NP * NIN * SLOT);
+  u64* bars = (u64*)(smem + NP * RSLOT);
 
   int la[NCA], lb[NCB];
 #pragma unroll
@@ -1124,8 +1159,8 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
     __syncthreads();
     if (tid == 0) {
       for (int j = 0; j < D && j < n_planes; ++j) {
-        mbar_arrive_expect_tx(&bars[j % NP], NIN * PL * 8);
-        tma_plane(P, g, smem + (j % NP) * NIN * SLOT, &bars[j % NP], g.s_start - R + j);
+        mbar_arrive_expect_tx(&bars[j % NP], TX_BYTES);
+        tma_plane(P, g, smem + (j % NP) * RSLOT, &bars[j % NP], g.s_start - R + j);
       }
     }
   } else if constexpr (STAGING == 2) {
@@ -1149,7 +1184,7 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
       if constexpr (STAGING == 1)
         out8[a] = GlobPlane{P.in[a] + col0 + (long long)p * g.st_s, g.st_b};
       else
-        out8[a] = SmemPlane{smem + (slot * NIN + a) * SLOT};
+        out8[a] = splane(smem + slot * RSLOT, a);
     }
   };
   using LDT = typename Cond<STAGING == 1, GlobPlane, SmemPlane>::type;
@@ -1284,13 +1319,13 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
           const int sl = (j + D) % NP;
 #endif
           fence_proxy_async();
-          mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
-          tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);
+          mbar_arrive_expect_tx(&bars[sl], TX_BYTES);
+          tma_plane(P, g, smem + sl * RSLOT, &bars[sl], p + D);
         }
       } else if constexpr (STAGING == 2) {
         __syncthreads();
         if (j + 1 < n_planes) {
-          double* dst = smem + ((j + 1) % NP) * NIN * SLOT;
+          double* dst = smem + ((j + 1) % NP) * RSLOT;
           if constexpr (D == 1) {
             ldst_plane(P, g, dst, p + 1);
           } else {
@@ -1332,7 +1367,7 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
   const int n_out = g.s_end - g.s_start;
   const int n_planes = n_out + 2 * R;
   const int steps = (n_out + TS - 1) / TS;
-  u64* bars = (u64*)(smem + NP * NIN * SLOT);
+  u64* bars = (u64*)(smem + NP * RSLOT);
 
   auto issue = [&](int j) {  // load plane j (sequence index) into its slot
     if (j >= n_planes) return;
@@ -1340,11 +1375,11 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
     if constexpr (STAGING == 3) {
       if (tid == 0) {
         fence_proxy_async();
-        mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
-        tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], g.s_start - R + j);
+        mbar_arrive_expect_tx(&bars[sl], TX_BYTES);
+        tma_plane(P, g, smem + sl * RSLOT, &bars[sl], g.s_start - R + j);
       }
     } else if constexpr (STAGING == 2) {
-      ldst_plane(P, g, smem + sl * NIN * SLOT, g.s_start - R + j);
+      ldst_plane(P, g, smem + sl * RSLOT, g.s_start - R + j);
     }
   };
 
@@ -1383,7 +1418,7 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
           const int jp = s - g.s_start + R;
           auto U2 = [&](int arr, int dx, int dy, int dz) {
             const int db = SZ ? dy : dz, ds = SZ ? dz : dy;
-            const double* row = smem + ((jp + ds) % NP) * NIN * SLOT + arr * SLOT +
+            const double* row = smem + ((jp + ds) % NP) * RSLOT + arr * SLOT +
                                 (lbp + R + db) * PA + lap + XR;
             if ((dx & 1) == 0) {
               const double2 v = *reinterpret_cast<const double2*>(row + dx);
@@ -1418,7 +1453,7 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
             const int jp = s - g.s_start + R;  // sequence index of the point's plane
             auto U = [&](int arr, int dx, int dy, int dz) {
               const int da = dx, db = SZ ? dy : dz, ds = SZ ? dz : dy;
-              return smem[((jp + ds) % NP) * NIN * SLOT + arr * SLOT + (lbp + R + db) * PA +
+              return smem[((jp + ds) % NP) * RSLOT + arr * SLOT + (lbp + R + db) * PA +
                           lap + XR + da];
             };
             point(C, U, o);
@@ -1911,6 +1946,130 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
 
 
 // =============================================================================
+// hypterm in-plane terms by row streaming (TMEM path, one point per thread)
+//
+// Every in-plane derivative contributes  sum_{k=-R..R, k!=0} wd[k] E^d_f(p + k e_d)  to flux f,
+// wd[k] = -sign(k) dxinv_d a_|k| (the bank's ws tables, one per direction), E^d_f the
+// pointwise products of direction d.  Instead of loading a window per array and point, the
+// lanes walk the union of their windows one position at a time (six loads, five products,
+// five FMAs per position; few live registers):
+//  * along a (x): lanes 2i, 2i+1 share each 16-B chunk of the 2R+2 positions starting at the
+//    even element la - XR - (la & 1); a lane's weight at position j is wd[j - XR - (la & 1)],
+//    chosen by a select between two uniform constants;
+//  * along b, when a warp holds two b-rows (T_a = 16): both half-warps read the same row at a
+//    time (16 distinct doubles, one wavefront instead of two), 2R+2 rows per pair, the weight
+//    again selected by the lane's row parity; otherwise each lane walks its own 2R rows.
+// Positions outside a lane's window (beyond its halo) are predicated off, never weighted by
+// zero, so halo garbage past the radius cannot leak in as 0 * NaN.
+// =============================================================================
+constexpr bool HPAIR = TBA == 16 && TBB % 2 == 0;  // two b-rows per warp
+
+__host__ __device__ constexpr int ws_base(int dir) { return 7 + (dir == 2 ? 0 : (dir == 1 ? 8 : 16)); }
+
+// E^d_f at one position from v = {cons1..4, q_d, q4}
+template <int DIR>
+__device__ __forceinline__ void hyp_e(const double (&v)[6], double (&E)[5]) {
+  E[0] = v[DIR];
+#pragma unroll
+  for (int m = 0; m < 3; ++m) E[m + 1] = m == DIR ? fma(v[m], v[4], v[5]) : v[m] * v[4];
+  E[4] = fma(v[3], v[4], v[5] * v[4]);
+}
+
+// A_f += w E_f with the lane's weight for offsets k0 (parity 0) / k1 (parity 1)
+template <int DIR, int K0, int K1>
+__device__ __forceinline__ void hyp_acc(const Ctx& C, bool par, const double (&E)[5],
+                                        double (&A)[5]) {
+  constexpr bool V0 = K0 != 0 && K0 >= -R && K0 <= R, V1 = K1 != 0 && K1 >= -R && K1 <= R;
+  constexpr int I0 = V0 ? ws_base(DIR) + (K0 < 0 ? K0 + R : K0 + R - 1) : 0;
+  constexpr int I1 = V1 ? ws_base(DIR) + (K1 < 0 ? K1 + R : K1 + R - 1) : 0;
+  if constexpr (V0 && V1) {
+    const double w = par ? C.coef(I1) : C.coef(I0);
+#pragma unroll
+    for (int f = 0; f < 5; ++f) A[f] = fma(w, E[f], A[f]);
+  } else if constexpr (V0) {
+    if (!par) {
+#pragma unroll
+      for (int f = 0; f < 5; ++f) A[f] = fma(C.coef(I0), E[f], A[f]);
+    }
+  } else if constexpr (V1) {
+    if (par) {
+#pragma unroll
+      for (int f = 0; f < 5; ++f) A[f] = fma(C.coef(I1), E[f], A[f]);
+    }
+  }
+}
+
+// x-direction terms into A; the point's own cons1..4 and q4 into cen
+template <class LD>
+__device__ __forceinline__ void hyp_rows_a(const Ctx& C, const LD* ld, int la, int lb,
+                                           double (&A)[5], double (&cen)[5]) {
+  static_assert(XR == R, "even order");
+  const bool odd = la & 1;
+  const int e0 = la - XR - (int)odd;
+  static_for<0, R + 1>([&](auto CC) {
+    constexpr int c = decltype(CC)::value;
+    double2 v2[6];
+#pragma unroll
+    for (int m = 0; m < 4; ++m) v2[m] = ld[m].at2(e0 + 2 * c, lb);
+    v2[4] = ld[Q_A].at2(e0 + 2 * c, lb);
+    v2[5] = ld[7].at2(e0 + 2 * c, lb);
+    static_for<0, 2>([&](auto HH) {
+      constexpr int h = decltype(HH)::value, j = 2 * c + h;
+      double v[6];
+#pragma unroll
+      for (int m = 0; m < 6; ++m) v[m] = h ? v2[m].y : v2[m].x;
+      if constexpr (j == XR) {
+#pragma unroll
+        for (int m = 0; m < 4; ++m) cen[m] = v[m];
+        cen[4] = v[5];
+      } else if constexpr (j == XR + 1) {
+#pragma unroll
+        for (int m = 0; m < 4; ++m) cen[m] = odd ? v[m] : cen[m];
+        cen[4] = odd ? v[5] : cen[4];
+      }
+      double E[5];
+      hyp_e<DA>(v, E);
+      hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A);
+    });
+  });
+}
+
+// b-direction terms into A
+template <class LD>
+__device__ __forceinline__ void hyp_rows_b(const Ctx& C, const LD* ld, int la, int lb,
+                                           double (&A)[5]) {
+  if constexpr (HPAIR) {
+    const bool odd = lb & 1;
+    const int b0 = lb - (int)odd - R;
+    static_for<0, 2 * R + 2>([&](auto QQ) {
+      constexpr int q = decltype(QQ)::value;
+      double v[6];
+#pragma unroll
+      for (int m = 0; m < 4; ++m) v[m] = ld[m].at(la, b0 + q);
+      v[4] = ld[Q_B].at(la, b0 + q);
+      v[5] = ld[7].at(la, b0 + q);
+      double E[5];
+      hyp_e<DB>(v, E);
+      hyp_acc<DB, q - R, q - R - 1>(C, odd, E, A);
+    });
+  } else {
+    static_for<0, 2 * R + 1>([&](auto QQ) {
+      constexpr int q = decltype(QQ)::value;
+      if constexpr (q != R) {
+        double v[6];
+#pragma unroll
+        for (int m = 0; m < 4; ++m) v[m] = ld[m].at(la, lb - R + q);
+        v[4] = ld[Q_B].at(la, lb - R + q);
+        v[5] = ld[7].at(la, lb - R + q);
+        double E[5];
+        hyp_e<DB>(v, E);
+        hyp_acc<DB, q - R, q - R>(C, false, E, A);
+      }
+    });
+  }
+}
+
+// =============================================================================
 // hypterm-like, streamed-direction state in tensor memory (qstore = 2)
 //
 // The retimed hypterm kernel keeps 5 fluxes x (2R+1) pending planes = 45 doubles per point
@@ -1935,7 +2094,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
   const int tb = SZ ? thread_y() : thread_z();
   const int tid = threadIdx.x, warp = tid / 32;
   const int n_planes = (g.s_end - g.s_start) + 2 * R;
-  u64* bars = (u64*)(smem + NP * NIN * SLOT);
+  u64* bars = (u64*)(smem + NP * RSLOT);
   u32* tslot = (u32*)(bars + NP);  // spare mbarrier words (kernel_smem_bytes reserves 2 NP)
 
   int la[NCA], lb[NCB];
@@ -1958,8 +2117,8 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
   const u32 tq = *tslot + ((u32)((warp & 3) * 32) << 16) + (u32)((warp >> 2) * NPT * TM_PCOLS);
   if (tid == 0)
     for (int j = 0; j < D && j < n_planes; ++j) {
-      mbar_arrive_expect_tx(&bars[j % NP], NIN * PL * 8);
-      tma_plane(P, g, smem + (j % NP) * NIN * SLOT, &bars[j % NP], g.s_start - R + j);
+      mbar_arrive_expect_tx(&bars[j % NP], TX_BYTES);
+      tma_plane(P, g, smem + (j % NP) * RSLOT, &bars[j % NP], g.s_start - R + j);
     }
 
 #pragma unroll 1
@@ -1970,7 +2129,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
     mbar_wait(&bars[slot], (u32)((j / NP) & 1));
     SmemPlane ld[NIN];
 #pragma unroll
-    for (int a = 0; a < NIN; ++a) ld[a] = SmemPlane{smem + (slot * NIN + a) * SLOT};
+    for (int a = 0; a < NIN; ++a) ld[a] = splane(smem + slot * RSLOT, a);
     const bool need_a = j >= R && j < n_planes - R;  // A(p) feeds an interior output
     u32 ce[R];  // column offset of E slot of plane p - R + m
 #pragma unroll
@@ -1993,8 +2152,28 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
       // live registers, the load latency then hidden by other warps only
       if (!CST_TM_LATE && j >= R) issue_ring();  // in flight while products/T are computed
       double E[5][NCB][NCA];
-      hyp_products(ld, la, lb, E);
       double A[5];
+#if CST_HYP_ROWS
+      {
+        double cen[5];
+        if (need_a) {
+#pragma unroll
+          for (int f = 0; f < 5; ++f) A[f] = 0.0;
+          hyp_rows_a(C, ld, la[0], lb[0], A, cen);
+          hyp_rows_b(C, ld, la[0], lb[0], A);
+        } else {
+#pragma unroll
+          for (int m = 0; m < 4; ++m) cen[m] = ld[m].at(la[0], lb[0]);
+          cen[4] = ld[7].at(la[0], lb[0]);
+        }
+        const double v[6] = {cen[0], cen[1], cen[2], cen[3], ld[4 + DS].at(la[0], lb[0]), cen[4]};
+        double e[5];
+        hyp_e<DS>(v, e);
+#pragma unroll
+        for (int f = 0; f < 5; ++f) E[f][0][0] = e[f];
+      }
+#else
+      hyp_products(ld, la, lb, E);
       if (need_a) {
         double t[5][NCB][NCA];
         hyp_inplane<0>(C, ld, la, lb, t);
@@ -2004,6 +2183,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 #pragma unroll
         for (int f = 0; f < 5; ++f) A[f] -= t[f][0][0];
       }
+#endif
       if (j >= R) {
         if (CST_TM_LATE) issue_ring();
         tmem_wait_ld();
@@ -2045,8 +2225,8 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
     if (tid == 0 && j + D < n_planes) {
       const int sl = (j + D) % NP;
       fence_proxy_async();
-      mbar_arrive_expect_tx(&bars[sl], NIN * PL * 8);
-      tma_plane(P, g, smem + sl * NIN * SLOT, &bars[sl], p + D);
+      mbar_arrive_expect_tx(&bars[sl], TX_BYTES);
+      tma_plane(P, g, smem + sl * RSLOT, &bars[sl], p + D);
     }
   }
   tmem_fence_before_sync();

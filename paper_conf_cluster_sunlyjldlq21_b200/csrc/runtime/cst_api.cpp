@@ -184,7 +184,8 @@ extern "C" cst_status cst_stencil_create(const cst_stencil_desc* desc, const cst
   h->coeffs.assign(desc->coeffs, desc->coeffs + desc->n_coeffs);
   h->desc.coeffs = h->coeffs.data();
   // kernel coefficient bank: the user's coefficients, plus for hypterm the streamed-
-  // direction weights ws[k] = -sign(k) dxinv_s a_|k| (k = -4..-1, 1..4) for s = z, then y
+  // direction weights ws[k] = -sign(k) dxinv_d a_|k| (k = -4..-1, 1..4) for d = z, y, x
+  // (z and y: the streamed direction; all three: the row-streamed in-plane terms)
   h->kcoef = h->coeffs;
   if (kind == CST_RHS4) {
     // s_d^2 / 6 for the V terms, s_d s_i / 144 for the mixed pairs (0,1), (0,2), (1,2)
@@ -194,7 +195,7 @@ extern "C" cst_status cst_stencil_create(const cst_stencil_desc* desc, const cst
     h->kcoef.push_back(h->coeffs[1] * h->coeffs[2] / 144.0);
   }
   if (kind == CST_HYPTERM)
-    for (int sdir : {2, 1})
+    for (int sdir : {2, 1, 0})
       for (int k = -4; k <= 4; ++k) {
         if (k == 0) continue;
         const double a = h->coeffs[(k > 0 ? k : -k) - 1];
@@ -251,12 +252,15 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
   const int64_t* M = h->info.M;
   // measured-good starting points on B200, shrunk to fit small grids:
   // streaming along z, TMA staging, retimed accumulators; star/box 64x8 tiles of 2x2
-  // register blocks; hypterm/rhs4 16x8 tiles, one point per thread (rhs4: 128-plane
-  // blocks, 2-deep TMA ring — 24.5 vs 23.4 GSt/s at 320^3 over pf 1).
+  // register blocks; rhs4 16x8 tiles, one point per thread (128-plane blocks, 2-deep TMA
+  // ring — 24.5 vs 23.4 GSt/s at 320^3 over pf 1); hypterm 16x16 tiles, one point per
+  // thread, streamed state in TMEM, 2-deep ring, coefficients in __constant__ (3.50 ms vs
+  // 3.68 ms for the best register-path setting at 512^3).
   const bool hyp = h->info.kind == CST_HYPTERM || h->info.kind == CST_RHS4;
+  const bool hyp_tm = h->info.kind == CST_HYPTERM;
   cst_setting c{};
   c.tb[0] = hyp ? 16 : 32;
-  c.tb[1] = hyp ? 8 : 4;
+  c.tb[1] = hyp_tm ? 16 : (hyp ? 8 : 4);
   c.tb[2] = 1;
   c.staging = 3;
   c.use_constant = 1;
@@ -268,15 +272,18 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
   c.bm[1] = hyp ? 1 : 2;
   c.use_retiming = 2;
   c.bt = 1;
-  c.qstore = 1;
-  c.prefetch = (h->info.kind == CST_BOX || h->info.kind == CST_RHS4) ? 2 : 3;
+  c.qstore = hyp_tm ? 2 : 1;
+  if (hyp_tm) c.use_constant = 2;
+  c.prefetch = (h->info.kind == CST_BOX || h->info.kind == CST_RHS4 || hyp_tm) ? 2 : 3;
   for (int tries = 0; tries < 12 && check_rules(h->info, to_tuple(c)); ++tries) {
+    if (c.qstore == 2 && c.staging != 3) { c.qstore = 1; continue; }  // R15 needs TMA
     // shrink the tile until it fits the grid (coverage) and the thread floor
     if (c.bm[0] > 1 && (int64_t)c.tb[0] * c.bm[0] > M[0]) c.bm[0] /= 2;
     else if (c.bm[1] > 1 && (int64_t)c.tb[1] * c.bm[1] > M[1]) c.bm[1] /= 2;
     else if (c.tb[0] > 1 && c.tb[0] > M[0]) { c.tb[0] /= 2; c.tb[1] *= 2; }
     else if (c.tb[1] > 1 && c.tb[1] > M[1]) { c.tb[1] /= 2; }
     else if (c.tb[0] * c.bm[0] % 2) { c.staging = 2; }
+    else if (c.qstore == 2) { c.qstore = 1; }
     else break;
   }
   if (!check_rules(h->info, to_tuple(c))) {
@@ -475,7 +482,14 @@ cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* 
   for (int a = 0; a < nin; ++a) {
     P.in[a] = in[a] + origin;
     if (t[F_STAGING] == 3) {
-      st = tmap_for(h, in[a], g.box, G.nz + 2 * (int64_t)G.halo, &P.tma[a]);
+      int box[3] = {g.box[0], g.box[1], g.box[2]};
+      if (t[F_STREAM] == 2 && hyp_trimmed(h->info.kind, t)) {  // per-array halos (HTRIM)
+        int64_t wa, wb;
+        stream_array_box(h->info.kind, h->info.r, t, a, &wa, &wb);
+        box[0] = (int)wa;
+        box[t[F_SD] == 3 ? 1 : 2] = (int)wb;
+      }
+      st = tmap_for(h, in[a], box, G.nz + 2 * (int64_t)G.halo, &P.tma[a]);
       if (st != CST_OK) return st;
     }
   }

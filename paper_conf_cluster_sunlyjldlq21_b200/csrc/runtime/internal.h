@@ -54,6 +54,8 @@ int64_t model_regs(int kind, int r, const Tuple& t);
 int tmem_cols_alloc(int kind, int r, const Tuple& t);
 // Dynamic shared memory the kernel variant actually uses (<= model for fast paths).
 int64_t kernel_smem_bytes(int kind, int r, const Tuple& t);
+bool hyp_trimmed(int kind, const Tuple& t);
+void stream_array_box(int kind, int r, const Tuple& t, int a, int64_t* wa, int64_t* wb);
 
 // ------------------------------------------------------------------ space
 class Space {

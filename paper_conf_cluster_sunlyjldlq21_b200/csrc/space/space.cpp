@@ -161,6 +161,28 @@ int64_t model_smem_bytes(int kind, int r, const Tuple& t) {
   return n_arrays(kind) * NP * plane;
 }
 
+// Per-array halos of the hypterm TMA fast path (HTRIM in csrc/kernels/cst_kernels.cuh):
+// array a's staged in-plane box is (T_a + 2 XR h_a) x (T_b + 2 r h_b) with h_a = 0 for q_b
+// and q_s, h_b = 0 for q_a and q_s (inputs: cons1..4 = 0..3, q1..q3 = 4..6, q4 = 7).
+bool hyp_trimmed(int kind, const Tuple& t) {
+  if (kind != CST_HYPTERM || t[F_STAGING] != 3 || t[F_STREAM] != 2 || t[F_BT] != 1) return false;
+  const int sd = t[F_SD] - 1;
+  return (int64_t)t[F_TBX + sd] * t[F_BMX + sd] * t[F_CMX + sd] == 1;
+}
+
+void stream_array_box(int kind, int r, const Tuple& t, int a, int64_t* wa, int64_t* wb) {
+  int64_t T[3];
+  tiles(t, T);
+  const int sd = t[F_SD] - 1;
+  const int b = sd == 2 ? 1 : 2;
+  const int q_a = 4, q_b = 4 + b;
+  const bool trim = hyp_trimmed(kind, t);
+  const bool ha = !trim || a < 4 || a == 7 || a == q_a;
+  const bool hb = !trim || a < 4 || a == 7 || a == q_b;
+  *wa = T[0] + (ha ? 2 * xr_of(r) : 0);
+  *wb = T[b] + (hb ? 2 * (int64_t)r : 0);
+}
+
 int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
   // mirrors csrc/kernels/cst_kernels.cuh: x halo XR = r rounded up to even
   if (t[F_STAGING] == 1) return 0;
@@ -184,6 +206,15 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
   }
   const int64_t plane = (plane_elems * 8 + 127) / 128 * 128;
   const int64_t bars = t[F_STAGING] == 3 ? 2 * NP * 8 : 0;  // full (+ optional empty) mbarriers
+  if (t[F_STREAM] == 2 && hyp_trimmed(kind, t)) {
+    int64_t slot = 0;
+    for (int a = 0; a < n_arrays(kind); ++a) {
+      int64_t wa, wb;
+      stream_array_box(kind, r, t, a, &wa, &wb);
+      slot += rnd128(wa * wb * 8);
+    }
+    return NP * slot + bars;
+  }
   return n_arrays(kind) * NP * plane + bars;
 }
 

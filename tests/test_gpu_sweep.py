@@ -265,3 +265,31 @@ def test_host_path_multistep_and_chunked():
     C.cst_sweep_host(h, s, [t.data_ptr() for t in hin], [t.data_ptr() for t in hout], 2)
     H.assert_parity(L, hin[0].numpy(), win[0], "host T=2")
     C.cst_stencil_destroy(h)
+
+
+# hypterm-like register path over every staging of the fast streaming kernel; the TMA cases
+# use the per-array halo layout (q_a: a-halo only, q_b: b-halo only, q_s: none)
+HYP_PATHS = [
+    ("tma-z-32x4", S(tb_x=32, tb_y=4, sb=8, prefetch=2)),
+    ("tma-z-16x8-pf3", S(tb_x=16, tb_y=8, sb=8, prefetch=3)),
+    ("tma-z-32x8", S(tb_x=32, tb_y=8, sb=8, prefetch=2)),
+    ("tma-y-16x1x8", S(tb_x=16, tb_y=1, tb_z=8, sd=2, sb=8, prefetch=3)),
+    ("tma-y-32x1x4-sb16", S(tb_x=32, tb_y=1, tb_z=4, sd=2, sb=16, prefetch=2)),
+    ("tma-z-gather", S(tb_x=32, tb_y=4, sb=8, use_retiming=1, prefetch=2)),
+    ("tma-z-const-pf4", S(tb_x=16, tb_y=8, sb=8, use_constant=2, prefetch=4)),
+    ("ldst-z", S(tb_x=32, tb_y=4, sb=8, staging=2, prefetch=1)),
+    ("none-y", S(tb_x=16, tb_y=1, tb_z=8, sd=2, sb=8, staging=1, prefetch=1)),
+]
+
+
+@pytest.mark.parametrize("name,setting", HYP_PATHS, ids=[p[0] for p in HYP_PATHS])
+def test_hypterm_paths_ragged(name, setting):
+    kind, r = 3, 4
+    L = H.layout((37, 29, 26), r + 1)
+    c = H.coeffs(kind, r, "random", seed=5)
+    ins = H.inputs(kind, L, seed=17, poison_beyond=r)
+    _, want = H.oracle_outputs(kind, r, c, L, ins)
+    _, got = run_gpu(kind, r, c, L, ins, setting)
+    for o in range(5):
+        H.assert_parity(L, got[o], want[o], f"{name} out{o}")
+        H.assert_halo_untouched(L, got[o], np.full(L.numel, np.nan))

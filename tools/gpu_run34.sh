@@ -1,0 +1,14 @@
+#!/bin/bash
+# re-entry pass (session 3): build, smoke, GPU suite, hypterm TMEM sweep, bench
+cd "$GRAFT_REPO_ROOT" 2>/dev/null || cd /root/repo
+mkdir -p gpurun_out
+nvidia-smi > gpurun_out/smi.txt 2>&1
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout -k 10 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1
+echo "smoke rc=$?" >> gpurun_out/smoke.log
+timeout -k 10 1500 python -m pytest tests -m gpu -q --timeout 400 -p no:cacheprovider > gpurun_out/pytest_gpu.log 2>&1
+echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
+timeout -k 10 900 python tools/explore.py --kind 3 --order 4 --settings tools/hyp_tmem_late_explore.json --reps 5 > gpurun_out/explore_hyp_late.log 2>&1
+timeout -k 10 900 python tools/explore.py --kind 3 --order 4 --settings tools/hyp_tmem_big_explore.json --reps 5 > gpurun_out/explore_hyp_big.log 2>&1
+timeout -k 10 900 python bench.py > gpurun_out/bench.log 2>&1
+echo done

@@ -1,0 +1,12 @@
+#!/bin/bash
+# trimmed-halo hypterm + TMEM default: full GPU suite, smoke, hypterm re-tune, bench
+cd "$GRAFT_REPO_ROOT" 2>/dev/null || cd /root/repo
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout -k 10 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1
+echo "smoke rc=$?" >> gpurun_out/smoke.log
+timeout -k 10 1500 python -m pytest tests -m gpu -q --timeout 400 -p no:cacheprovider > gpurun_out/pytest_gpu.log 2>&1
+echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
+timeout -k 10 900 python tools/tune.py --config hypterm --budget 240 > gpurun_out/tune_hyp.log 2>&1
+timeout -k 10 900 python bench.py > gpurun_out/bench.log 2>&1
+echo done

@@ -23,8 +23,12 @@ if arg == "default":
     s = C.cst_setting_default(h)
 elif arg.endswith(".json") and os.path.exists(os.path.join(ROOT, arg)):
     s = C.cst_setting.from_dict(json.load(open(os.path.join(ROOT, arg)))["setting"])
-else:
-    s = C.cst_setting.from_dict(json.loads(arg))
+else:  # partial dicts are completed from explore.py's base setting
+    d = dict(tb_x=64, tb_y=4, tb_z=1, staging=3, use_constant=1, use_streaming=2, sd=3, sb=128,
+             uf_x=1, uf_y=1, uf_z=1, cm_x=1, cm_y=1, cm_z=1, bm_x=1, bm_y=1, bm_z=1,
+             use_retiming=2, prefetch=3, bt=1)
+    d.update(json.loads(arg))
+    s = C.cst_setting.from_dict(d)
 ins = [torch.empty(g.numel, dtype=torch.float64, device="cuda") for _ in range(C.N_IN[kind])]
 outs = [torch.empty(g.numel, dtype=torch.float64, device="cuda") for _ in range(C.N_OUT[kind])]
 for a, t in enumerate(ins):
