@@ -106,9 +106,10 @@ typedef struct {
                            * memory (TMEM)}: B200 extension of retiming — a ring of R
                            * (value, partial output) pairs per point in TMEM frees the
                            * registers for larger register blocks.  Rule
-                           * R15: qstore = 2 needs the star, streaming with T_SD = 1, TMA
+                           * R15: qstore = 2 needs the star or hypterm (hypterm: one point
+                           * along x, BM_b <= 2, CM = 1), streaming with T_SD = 1, TMA
                            * staging, retiming, bt = 1, and ceil(threads/128) * points per
-                           * thread * 4r <= 512 TMEM columns. */
+                           * thread * (4r star, 20r hypterm) <= 512 TMEM columns. */
 } cst_setting;
 
 typedef struct cst_stencil cst_stencil;     /* opaque: JIT modules, TMA descriptors, space */

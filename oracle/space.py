@@ -35,8 +35,9 @@ R10 modelled smem <= SMEM_LIMIT; R11 modelled registers <= 255; R12 TMA box: T_x
 every box extent <= 256; R14 bt > 1 only for the temporally blocked path: star / box,
 streaming along z with T_SD = 1, TMA staging, retimed accumulators, no cyclic merging,
 BM_x, BM_y <= 2, every UF = 1 (reading Q23); R15 qstore = 2 only for the
-TMEM path: star, streaming with T_SD = 1, TMA staging, retimed, bt = 1, and
-ceil(threads/128) * points per thread * 4r <= 512 TMEM columns.
+TMEM path: star or hypterm (hypterm: one point along x, BM_b <= 2 along the other in-plane
+dim, no cyclic merging), streaming with T_SD = 1, TMA staging, retimed, bt = 1, and
+ceil(threads/128) * points per thread * (4r star, 20r hypterm) <= 512 TMEM columns.
 """
 from __future__ import annotations
 
@@ -151,15 +152,19 @@ def qs_path_ok(kind: int, r: int, s: dict) -> bool:
         return False
     if tiles(s)[s["sd"] - 1] != 1:
         return False
-    if kind == HYPTERM and points_per_thread(s) != 1:
-        return False
+    if kind == HYPTERM:
+        # one point along a (x), up to two stacked along b (the in-plane non-x dim)
+        b = "y" if s["sd"] == 3 else "z"
+        for d in "xyz":
+            if s["cm_" + d] != 1 or s["bm_" + d] > 2 or (d != b and s["bm_" + d] != 1):
+                return False
     return tmem_columns(r, s, kind) <= 512
 
 
 def est_regs(kind: int, r: int, s: dict) -> int:
     if s["qstore"] == 2 and kind == HYPTERM:
-        # products, partial fluxes, the ring of one point, the in-plane windows
-        return 32 + 2 * (5 * (r + 1) + 5 + 5 + 30)
+        # products, partial fluxes, the ring of one point, the in-plane row values
+        return 32 + 2 * (5 * (r + 1) + 10 * points_per_thread(s) + 30)
     if s["qstore"] == 2:
         # in-plane part + centre per point, one point's ring, the block's column windows
         return 32 + 2 * (2 * points_per_thread(s) + (r + 1) + 2 * r)

@@ -34,9 +34,6 @@
 #ifndef CST_HYP_ROWS
 #define CST_HYP_ROWS 1  // TMEM hypterm: in-plane terms by row streaming
 #endif
-#ifndef CST_TM_LATE
-#define CST_TM_LATE 1  // hypterm TMEM ring loaded after the in-plane terms (measured best)
-#endif
 
 // ------------------------------------------------------------------ configuration
 constexpr int KIND = CST_KIND;  // 1 star, 2 box, 3 hypterm, 4 rhs4center-like
@@ -1956,13 +1953,21 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
 //  * along a (x): lanes 2i, 2i+1 share each 16-B chunk of the 2R+2 positions starting at the
 //    even element la - XR - (la & 1); a lane's weight at position j is wd[j - XR - (la & 1)],
 //    chosen by a select between two uniform constants;
-//  * along b, when a warp holds two b-rows (T_a = 16): both half-warps read the same row at a
-//    time (16 distinct doubles, one wavefront instead of two), 2R+2 rows per pair, the weight
-//    again selected by the lane's row parity; otherwise each lane walks its own 2R rows.
+//  * along b each lane walks its own 2R rows.  (CST_HYP_HPAIR = 1, experiment: when a warp
+//    holds two b-rows (T_a = 16) both half-warps read the same row at a time, 2R+2 rows per
+//    pair, the weight selected by the row parity — measured slower: 3.85 vs 3.53 ms at
+//    512^3; the shared 8-byte loads of the two half-warps are not merged into one wavefront.)
 // Positions outside a lane's window (beyond its halo) are predicated off, never weighted by
 // zero, so halo garbage past the radius cannot leak in as 0 * NaN.
 // =============================================================================
-constexpr bool HPAIR = TBA == 16 && TBB % 2 == 0;  // two b-rows per warp
+#ifndef CST_HYP_HPAIR
+#define CST_HYP_HPAIR 0
+#endif
+constexpr bool HPAIR = CST_HYP_HPAIR && TBA == 16 && TBB % 2 == 0;  // two b-rows per warp
+#ifndef CST_TM_EARLY
+#define CST_TM_EARLY (CST_BMX * CST_BMY * CST_BMZ > 1)  // TMEM hypterm: ring fetch before in-plane
+#endif
+constexpr bool TM_EARLY = CST_TM_EARLY;
 
 __host__ __device__ constexpr int ws_base(int dir) { return 7 + (dir == 2 ? 0 : (dir == 1 ? 8 : 16)); }
 
@@ -2069,6 +2074,30 @@ __device__ __forceinline__ void hyp_rows_b(const Ctx& C, const LD* ld, int la, i
   }
 }
 
+// b-direction terms of NP2 points stacked along b (rows lb0 .. lb0 + NP2 - 1, register
+// blocking BM_b): the union of their windows is walked once, each row's products
+// feeding every point it neighbours (2R + NP2 rows instead of 2R per point)
+template <int NP2, class LD>
+__device__ __forceinline__ void hyp_rows_bn(const Ctx& C, const LD* ld, int la, int lb0,
+                                            double (&A)[NP2][5]) {
+  static_for<0, 2 * R + NP2>([&](auto QQ) {
+    constexpr int q = decltype(QQ)::value;
+    if constexpr (NP2 > 1 || q != R) {
+      double v[6];
+#pragma unroll
+      for (int m = 0; m < 4; ++m) v[m] = ld[m].at(la, lb0 - R + q);
+      v[4] = ld[Q_B].at(la, lb0 - R + q);
+      v[5] = ld[7].at(la, lb0 - R + q);
+      double E[5];
+      hyp_e<DB>(v, E);
+      static_for<0, NP2>([&](auto PP) {
+        constexpr int pt = decltype(PP)::value;
+        hyp_acc<DB, q - R - pt, q - R - pt>(C, false, E, A[pt]);
+      });
+    }
+  });
+}
+
 // =============================================================================
 // hypterm-like, streamed-direction state in tensor memory (qstore = 2)
 //
@@ -2084,8 +2113,9 @@ __device__ __forceinline__ void hyp_rows_b(const Ctx& C, const LD* ld, int la, i
 // =============================================================================
 template <int DUMMY>
 __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* smem) {
-  static_assert(DUMMY != 0 || (KIND == 3 && STAGING == 3 && TS == 1 && NCA == 1 && NCB == 1),
-                "TMEM hypterm: TMA, T_SD = 1, one point per thread");
+  static_assert(DUMMY != 0 || (KIND == 3 && STAGING == 3 && TS == 1 && NCA == 1 && CMB == 1 &&
+                               NCB <= 2),
+                "TMEM hypterm: TMA, T_SD = 1, one point along a, up to two along b");
   static_assert(DUMMY != 0 || TM_USED <= 512, "TMEM ring exceeds 512 columns");
   Ctx C{P};
   constexpr int D = PF, NP = PF;
@@ -2135,91 +2165,104 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 #pragma unroll
     for (int m = 0; m < R; ++m) ce[m] = (u32)(10 * ((u + m) % R));
     const u32 ca = (u32)(10 * (R + u));  // A slot of plane p - R (read) / p (written)
-    {  // one point per thread (R15: BM = CM = 1 in-plane for the hypterm TMEM path)
-      constexpr int ib = 0, ia = 0;
-      const u32 tp = tq;
-      u32 re[R][10], ra[10];
-      auto issue_ring = [&]() {
+    {  // NCB points stacked along b (R15: BM_a = CM = 1, BM_b <= 2)
+      constexpr int ia = 0;
+      double E[NCB][5];
+      double A[NCB][5];
+      // ring slots of every point; with two points the CTA is TMEM-bound to 8 warps per SM
+      // and registers are plentiful, so the rings are fetched before the in-plane terms
+      // (load latency hidden by them); one point: fetched after them (fewer live registers)
+      constexpr bool EARLY = TM_EARLY;
+      u32 re[NCB][R][10], ra[NCB][10];
+      auto issue_ring = [&](int ib) {
+        const u32 tp = tq + (u32)(ib * TM_PCOLS);
 #pragma unroll
         for (int m = 0; m < R; ++m) {
-          tmem_ld_x8(tp + ce[m], re[m]);
-          tmem_ld_x2(tp + ce[m] + 8, re[m] + 8);
+          tmem_ld_x8(tp + ce[m], re[ib][m]);
+          tmem_ld_x2(tp + ce[m] + 8, re[ib][m] + 8);
         }
-        tmem_ld_x8(tp + ca, ra);
-        tmem_ld_x2(tp + ca + 8, ra + 8);
+        tmem_ld_x8(tp + ca, ra[ib]);
+        tmem_ld_x2(tp + ca + 8, ra[ib] + 8);
       };
-      // CST_TM_LATE (experiment hook): issue the ring after the in-plane terms — 50 fewer
-      // live registers, the load latency then hidden by other warps only
-      if (!CST_TM_LATE && j >= R) issue_ring();  // in flight while products/T are computed
-      double E[5][NCB][NCA];
-      double A[5];
-#if CST_HYP_ROWS
-      {
-        double cen[5];
-        if (need_a) {
+      if (EARLY && j >= R) {
 #pragma unroll
-          for (int f = 0; f < 5; ++f) A[f] = 0.0;
-          hyp_rows_a(C, ld, la[0], lb[0], A, cen);
-          hyp_rows_b(C, ld, la[0], lb[0], A);
+        for (int ib = 0; ib < NCB; ++ib) issue_ring(ib);
+      }
+      {
+        double cen[NCB][5];
+        if (need_a) {
+          // separate x and b partial sums: two independent FMA chains per flux
+          double Ab[NCB][5];
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int f = 0; f < 5; ++f) A[ib][f] = Ab[ib][f] = 0.0;
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib) hyp_rows_a(C, ld, la[0], lb[ib], A[ib], cen[ib]);
+          if constexpr (NCB == 1 && HPAIR)
+            hyp_rows_b(C, ld, la[0], lb[0], Ab[0]);
+          else
+            hyp_rows_bn<NCB>(C, ld, la[0], lb[0], Ab);
+#pragma unroll
+          for (int ib = 0; ib < NCB; ++ib)
+#pragma unroll
+            for (int f = 0; f < 5; ++f) A[ib][f] += Ab[ib][f];
         } else {
 #pragma unroll
-          for (int m = 0; m < 4; ++m) cen[m] = ld[m].at(la[0], lb[0]);
-          cen[4] = ld[7].at(la[0], lb[0]);
-        }
-        const double v[6] = {cen[0], cen[1], cen[2], cen[3], ld[4 + DS].at(la[0], lb[0]), cen[4]};
-        double e[5];
-        hyp_e<DS>(v, e);
+          for (int ib = 0; ib < NCB; ++ib) {
 #pragma unroll
-        for (int f = 0; f < 5; ++f) E[f][0][0] = e[f];
-      }
-#else
-      hyp_products(ld, la, lb, E);
-      if (need_a) {
-        double t[5][NCB][NCA];
-        hyp_inplane<0>(C, ld, la, lb, t);
-#pragma unroll
-        for (int f = 0; f < 5; ++f) A[f] = -t[f][0][0];
-        hyp_inplane<1>(C, ld, la, lb, t);
-#pragma unroll
-        for (int f = 0; f < 5; ++f) A[f] -= t[f][0][0];
-      }
-#endif
-      if (j >= R) {
-        if (CST_TM_LATE) issue_ring();
-        tmem_wait_ld();
-#pragma unroll
-        for (int m = 0; m < R; ++m) tmem_pin(re[m]);
-        tmem_pin(ra);
-        auto ev = [&](int m, int f) { return tmem_d(re[m][2 * f], re[m][2 * f + 1]); };
-        if (need_a) {
-#pragma unroll
-          for (int f = 0; f < 5; ++f)
-#pragma unroll
-            for (int m = 0; m < R; ++m) A[f] = fma(ws(m - R), ev(m, f), A[f]);
-          tmem_st_5d(tp + ca, A);
-        }
-        if (j >= 2 * R) {
-          double v[5];
-#pragma unroll
-          for (int f = 0; f < 5; ++f) {
-            double o = tmem_d(ra[2 * f], ra[2 * f + 1]);
-#pragma unroll
-            for (int k = 1; k < R; ++k) o = fma(ws(k), ev(k, f), o);
-            v[f] = fma(ws(R), E[f][0][0], o);
-          }
-          if (g.a0 + la[ia] < g.n_a && g.b0 + lb[ib] < g.n_b) {
-            const long long off =
-                col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)(p - R) * g.st_s;
-#pragma unroll
-            for (int f = 0; f < 5; ++f) put(P, f, off, v[f]);
+            for (int m = 0; m < 4; ++m) cen[ib][m] = ld[m].at(la[0], lb[ib]);
+            cen[ib][4] = ld[7].at(la[0], lb[ib]);
           }
         }
-      }
-      double e5[5];
 #pragma unroll
-      for (int f = 0; f < 5; ++f) e5[f] = E[f][0][0];
-      tmem_st_5d(tp + 10 * u, e5);
+        for (int ib = 0; ib < NCB; ++ib) {
+          const double v[6] = {cen[ib][0], cen[ib][1], cen[ib][2], cen[ib][3],
+                               ld[4 + DS].at(la[0], lb[ib]), cen[ib][4]};
+          hyp_e<DS>(v, E[ib]);
+        }
+      }
+      // streamed-direction state, one point at a time (ring loaded after the in-plane terms)
+#pragma unroll
+      for (int ib = 0; ib < NCB; ++ib) {
+        const u32 tp = tq + (u32)(ib * TM_PCOLS);
+        if (j >= R) {
+          if (!EARLY) issue_ring(ib);
+          if (!EARLY || ib == 0) tmem_wait_ld();
+#pragma unroll
+          for (int m = 0; m < R; ++m) tmem_pin(re[ib][m]);
+          tmem_pin(ra[ib]);
+          auto ev = [&](int m, int f) { return tmem_d(re[ib][m][2 * f], re[ib][m][2 * f + 1]); };
+          if (need_a) {
+#pragma unroll
+            for (int f = 0; f < 5; ++f)
+#pragma unroll
+              for (int m = 0; m < R; ++m) A[ib][f] = fma(ws(m - R), ev(m, f), A[ib][f]);
+            tmem_st_5d(tp + ca, A[ib]);
+          }
+          if (j >= 2 * R) {
+            double v[5];
+#pragma unroll
+            for (int f = 0; f < 5; ++f) {
+              double o = tmem_d(ra[ib][2 * f], ra[ib][2 * f + 1]);
+#pragma unroll
+              for (int k = 1; k < R; ++k) o = fma(ws(k), ev(k, f), o);
+              v[f] = fma(ws(R), E[ib][f], o);
+            }
+            if (g.a0 + la[ia] < g.n_a && g.b0 + lb[ib] < g.n_b) {
+              const long long off =
+                  col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)(p - R) * g.st_s;
+#pragma unroll
+              for (int f = 0; f < 5; ++f) put(P, f, off, v[f]);
+            }
+          }
+        }
+        tmem_st_5d(tp + 10 * u, E[ib]);
+      }
     }
+#if !CST_HYP_ROWS
+#error "CST_HYP_ROWS = 0 (window path) was removed from the TMEM hypterm kernel"
+#endif
     tmem_wait_st();  // the next plane reads these slots
     __syncthreads();
     if (tid == 0 && j + D < n_planes) {
@@ -2243,10 +2286,8 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 // unconstrained schedule hoists every shared-memory load of the block (up to 255 registers)
 #define CST_TM_NPT (CST_BMX * CST_CMX * CST_BMY * CST_CMY * CST_BMZ * CST_CMZ)
 #define CST_TM_NTHR (CST_TBX * CST_TBY * CST_TBZ)
-#if CST_KIND == 3 && CST_TM_LATE
-#define CST_TM_REGS 120  // hypterm, ring loaded after the in-plane terms
-#elif CST_KIND == 3
-#define CST_TM_REGS 168  // hypterm: ring of 25 doubles + in-plane windows, one point
+#if CST_KIND == 3
+#define CST_TM_REGS (CST_TM_NPT == 1 ? 120 : 255)  // hypterm (two points: TMEM-bound to 8 warps/SM)
 #else  // star: + every point's ring in flight when it fits 48 registers (TM_ALL)
 #define CST_TM_REGS (96 + 4 * CST_TM_NPT + \
                      (CST_TM_NPT * (2 * CST_R + 2) <= 48 ? CST_TM_NPT * (2 * CST_R + 2) : 0))

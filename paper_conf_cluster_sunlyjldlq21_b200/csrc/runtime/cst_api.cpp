@@ -4,6 +4,7 @@
 #include <chrono>
 #include <cmath>
 #include <cstring>
+#include <cstdlib>
 #include <mutex>
 
 #include "internal.h"
@@ -253,14 +254,14 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
   // measured-good starting points on B200, shrunk to fit small grids:
   // streaming along z, TMA staging, retimed accumulators; star/box 64x8 tiles of 2x2
   // register blocks; rhs4 16x8 tiles, one point per thread (128-plane blocks, 2-deep TMA
-  // ring — 24.5 vs 23.4 GSt/s at 320^3 over pf 1); hypterm 16x16 tiles, one point per
-  // thread, streamed state in TMEM, 2-deep ring, coefficients in __constant__ (3.50 ms vs
-  // 3.68 ms for the best register-path setting at 512^3).
+  // ring — 24.5 vs 23.4 GSt/s at 320^3 over pf 1); hypterm 32x4 threads with two points
+  // stacked along y each, streamed state in TMEM, 3-deep ring, coefficients in __constant__
+  // (3.16-3.19 ms vs 3.53 ms for the best register-path setting at 512^3).
   const bool hyp = h->info.kind == CST_HYPTERM || h->info.kind == CST_RHS4;
   const bool hyp_tm = h->info.kind == CST_HYPTERM;
   cst_setting c{};
-  c.tb[0] = hyp ? 16 : 32;
-  c.tb[1] = hyp_tm ? 16 : (hyp ? 8 : 4);
+  c.tb[0] = hyp && !hyp_tm ? 16 : 32;
+  c.tb[1] = hyp && !hyp_tm ? 8 : 4;
   c.tb[2] = 1;
   c.staging = 3;
   c.use_constant = 1;
@@ -269,12 +270,12 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
   c.sb = p2floor(M[2], h->info.kind == CST_HYPTERM ? 256 : 128);
   for (int d = 0; d < 3; ++d) c.uf[d] = c.cm[d] = c.bm[d] = 1;
   c.bm[0] = hyp ? 1 : 2;
-  c.bm[1] = hyp ? 1 : 2;
+  c.bm[1] = hyp && !hyp_tm ? 1 : 2;
   c.use_retiming = 2;
   c.bt = 1;
   c.qstore = hyp_tm ? 2 : 1;
   if (hyp_tm) c.use_constant = 2;
-  c.prefetch = (h->info.kind == CST_BOX || h->info.kind == CST_RHS4 || hyp_tm) ? 2 : 3;
+  c.prefetch = (h->info.kind == CST_BOX || h->info.kind == CST_RHS4) ? 2 : 3;
   for (int tries = 0; tries < 12 && check_rules(h->info, to_tuple(c)); ++tries) {
     if (c.qstore == 2 && c.staging != 3) { c.qstore = 1; continue; }  // R15 needs TMA
     // shrink the tile until it fits the grid (coverage) and the thread floor
@@ -447,10 +448,14 @@ static cst_status tmap_for(cst_stencil* h, const double* base, const int box[3],
                                  (cuuint64_t)h->grid.pitch_x * h->grid.pitch_y * 8};
   const cuuint32_t boxd[3] = {(cuuint32_t)box[0], (cuuint32_t)box[1], (cuuint32_t)box[2]};
   const cuuint32_t estr[3] = {1, 1, 1};
+  // L2 promotion of the TMA fetches (experiment hook CST_TMA_PROMO = 0 none, 1 64B,
+  // 2 128B, 3 256B; default 256B)
+  CUtensorMapL2promotion promo = CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+  if (const char* e = std::getenv("CST_TMA_PROMO")) promo = (CUtensorMapL2promotion)std::atoi(e);
   st = cu_check(d->cuTensorMapEncodeTiled(
                     (CUtensorMap*)&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, (void*)base, dims,
                     strides, boxd, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                    CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_SWIZZLE_NONE, promo,
                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE),
                 "cuTensorMapEncodeTiled");
   if (st != CST_OK) return st;

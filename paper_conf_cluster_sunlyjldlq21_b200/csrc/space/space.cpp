@@ -94,7 +94,7 @@ static int64_t tb_smem_bytes(int r, const Tuple& t) {
 }
 
 // R15: the TMEM streamed-state path (qstore = 2): star or hypterm, streaming with
-// T_SD = 1, TMA, retimed, bt = 1 (hypterm: one point per thread); ceil(threads / 128) warps
+// T_SD = 1, TMA, retimed, bt = 1 (hypterm: one point along x, BM_b <= 2, CM = 1); ceil(threads / 128) warps
 // share a TMEM lane quarter, each thread keeps 4r (star) or 20r (hypterm: 5 products + 5
 // partial fluxes per ring slot) columns per point, 512 columns per SM (mirrors TM_* in
 // csrc/kernels/cst_kernels.cuh)
@@ -118,9 +118,11 @@ static bool qs_path_ok(int kind, int r, const Tuple& t) {
     return false;
   const int sd = t[F_SD] - 1;
   if ((int64_t)t[F_TBX + sd] * t[F_BMX + sd] * t[F_CMX + sd] != 1) return false;
-  if (kind == CST_HYPTERM)
+  if (kind == CST_HYPTERM) {  // one point along a (x), up to two stacked along b
+    const int b = sd == 2 ? 1 : 2;
     for (int d = 0; d < 3; ++d)
-      if (t[F_BMX + d] * t[F_CMX + d] != 1) return false;
+      if (t[F_CMX + d] != 1 || (d != b && t[F_BMX + d] != 1) || t[F_BMX + d] > 2) return false;
+  }
   return tmem_cols_kind(kind, r, t) <= 512;
 }
 
@@ -219,8 +221,11 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
 }
 
 int64_t model_regs(int kind, int r, const Tuple& t) {
-  if (t[F_QS] == 2 && kind == CST_HYPTERM)  // products, partial fluxes, ring, windows
-    return 32 + 2 * (5 * (r + 1) + 5 + 5 + 30);
+  if (t[F_QS] == 2 && kind == CST_HYPTERM) {  // products, partial fluxes, ring, row values
+    int64_t ppt = 1;
+    for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
+    return 32 + 2 * (5 * (r + 1) + 10 * ppt + 30);
+  }
   if (t[F_QS] == 2) {
     // TMEM path: in-plane part + centre per point, one point's ring (r + 1 doubles) and
     // the column windows of the block in flight

@@ -101,6 +101,10 @@ HYP_CASES = [
     ("y-16x1x16-const", Q(tb_x=16, tb_y=1, tb_z=16, sd=2, bm_x=1, bm_y=1, sb=16,
                           use_constant=2, prefetch=3)),
     ("sb1-pf1", Q(tb_x=32, tb_y=4, bm_x=1, bm_y=1, sb=1, prefetch=1)),
+    # two points stacked along b (BM_b = 2): union of the b-windows, per-point TMEM rings
+    ("z-32x4-bmy2", Q(tb_x=32, tb_y=4, bm_x=1, bm_y=2, sb=8)),
+    ("z-16x8-bmy2-pf3", Q(tb_x=16, tb_y=8, bm_x=1, bm_y=2, prefetch=3, sb=16, use_constant=2)),
+    ("y-32x1x4-bmz2", Q(tb_x=32, tb_y=1, tb_z=4, sd=2, bm_x=1, bm_y=1, bm_z=2, sb=8)),
 ]
 
 
