@@ -484,17 +484,35 @@ __device__ __forceinline__ void ldst_plane(const cst_kparams& P, const SGeo& g, 
 struct SmemPlane {
   static constexpr bool VEC = true;
   const double* base;  // slot base of one array
-  int pitch = PA;            // row pitch (elements)
-  int org = R * PA + XR;     // element offset of tile point (0, 0)
+  __device__ __forceinline__ double at(int la, int lb) const { return base[(lb + R) * PA + la + XR]; }
+  __device__ __forceinline__ double2 at2(int la, int lb) const {
+    return *reinterpret_cast<const double2*>(base + (lb + R) * PA + la + XR);
+  }
+};
+// HTRIM slots: per-array pitch and origin (compile-time constants once the array loop is
+// unrolled); a separate type so the uniform paths keep their one-pointer accessor
+struct SmemPlaneV {
+  static constexpr bool VEC = true;
+  const double* base;
+  int pitch;  // row pitch (elements)
+  int org;    // element offset of tile point (0, 0)
   __device__ __forceinline__ double at(int la, int lb) const { return base[org + lb * pitch + la]; }
   __device__ __forceinline__ double2 at2(int la, int lb) const {
     return *reinterpret_cast<const double2*>(base + org + lb * pitch + la);
   }
 };
+using SPlane = typename Cond<HTRIM, SmemPlaneV, SmemPlane>::type;
 // array a of the ring slot at `slot_base` (per-array layout; uniform unless HTRIM)
-__device__ __forceinline__ SmemPlane splane(const double* slot_base, int a) {
-  return SmemPlane{slot_base + arr_off(a), arr_wa(a),
-                   (arr_halo_b(a) ? R : 0) * arr_wa(a) + (arr_halo_a(a) ? XR : 0)};
+__device__ __forceinline__ SmemPlaneV splane_v(const double* slot_base, int a) {
+  return SmemPlaneV{slot_base + arr_off(a), arr_wa(a),
+                    (arr_halo_b(a) ? R : 0) * arr_wa(a) + (arr_halo_a(a) ? XR : 0)};
+}
+__device__ __forceinline__ SmemPlane splane_u(const double* slot_base, int a) {
+  return SmemPlane{slot_base + arr_off(a)};
+}
+__device__ __forceinline__ auto splane(const double* slot_base, int a) {
+  if constexpr (HTRIM) return splane_v(slot_base, a);
+  else return splane_u(slot_base, a);
 }
 struct GlobPlane {
   static constexpr bool VEC = false;
@@ -1184,7 +1202,7 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
         out8[a] = splane(smem + slot * RSLOT, a);
     }
   };
-  using LDT = typename Cond<STAGING == 1, GlobPlane, SmemPlane>::type;
+  using LDT = typename Cond<STAGING == 1, GlobPlane, SPlane>::type;
   auto store5 = [&](int ib, int ia, int po, double (&v)[5]) {
     if (g.a0 + la[ia] < g.n_a && g.b0 + lb[ib] < g.n_b) {
       const long long off = col0 + la[ia] + (long long)lb[ib] * g.st_b + (long long)po * g.st_s;
@@ -1964,6 +1982,9 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
 #define CST_HYP_HPAIR 0
 #endif
 constexpr bool HPAIR = CST_HYP_HPAIR && TBA == 16 && TBB % 2 == 0;  // two b-rows per warp
+#ifndef CST_HYP_XSPLIT
+#define CST_HYP_XSPLIT 0  // experiment: x-walk into two partial sums (even / odd positions)
+#endif
 #ifndef CST_TM_EARLY
 #define CST_TM_EARLY (CST_BMX * CST_BMY * CST_BMZ > 1)  // TMEM hypterm: ring fetch before in-plane
 #endif
@@ -2011,6 +2032,7 @@ __device__ __forceinline__ void hyp_rows_a(const Ctx& C, const LD* ld, int la, i
   static_assert(XR == R, "even order");
   const bool odd = la & 1;
   const int e0 = la - XR - (int)odd;
+  double A2[5] = {0.0, 0.0, 0.0, 0.0, 0.0};
   static_for<0, R + 1>([&](auto CC) {
     constexpr int c = decltype(CC)::value;
     double2 v2[6];
@@ -2034,9 +2056,16 @@ __device__ __forceinline__ void hyp_rows_a(const Ctx& C, const LD* ld, int la, i
       }
       double E[5];
       hyp_e<DA>(v, E);
-      hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A);
+      if constexpr (CST_HYP_XSPLIT && h == 1)  // experiment: second chain for odd positions
+        hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A2);
+      else
+        hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A);
     });
   });
+  if constexpr (CST_HYP_XSPLIT) {
+#pragma unroll
+    for (int f = 0; f < 5; ++f) A[f] += A2[f];
+  }
 }
 
 // b-direction terms into A
@@ -2157,7 +2186,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
     const int slot = j % NP;
     const int u = j % R;
     mbar_wait(&bars[slot], (u32)((j / NP) & 1));
-    SmemPlane ld[NIN];
+    SPlane ld[NIN];
 #pragma unroll
     for (int a = 0; a < NIN; ++a) ld[a] = splane(smem + slot * RSLOT, a);
     const bool need_a = j >= R && j < n_planes - R;  // A(p) feeds an interior output
