@@ -1002,6 +1002,16 @@ __device__ __forceinline__ void kernel_stream1(const cst_kparams& P, double* sme
 // =============================================================================
 constexpr int DA = 0, DB = SZ ? 1 : 2, DS = SZ ? 2 : 1;  // direction (0 x, 1 y, 2 z)
 
+// derivative weight of offset k along direction dir (hypterm, R = 4):
+//   w_d[k] = -sign(k) dxinv_d a_|k|, from the bank's products P_d[j] = dxinv_d a_j
+//   (j = 1..R; host cst_api.cpp: after the 7 user coefficients, d = z, y, x); the
+//   negation is exact, so every use is bit-identical to a stored signed table
+__host__ __device__ constexpr int ws_base(int dir) { return 7 + R * (dir == 2 ? 0 : (dir == 1 ? 1 : 2)); }
+__device__ __forceinline__ double hws(const Ctx& C, int dir, int k) {
+  const double p = C.coef(ws_base(dir) + (k < 0 ? -k : k) - 1);
+  return k > 0 ? -p : p;
+}
+
 // load a line of values through the point block: along a (x-window of row lb, starting
 // la - XR, length BMA + 2XR) or along b (column la, rows lb - R .., length BMB + 2R)
 template <int AXIS, class LD>
@@ -1148,7 +1158,7 @@ __device__ __forceinline__ void kernel_hyp_stream1(const cst_kparams& P, double*
   // streamed-direction weights ws[k] = -sign(k) dxinv_s a_|k| (host-precomputed, in the
   // constant bank after the 7 user coefficients: 8 for s = z, then 8 for s = y):
   // plane p contributes ws[p-o] * E_f(p) to flux_f(o)
-  auto ws = [&](int k) { return C.coef(7 + (DS == 1 ? 8 : 0) + (k < 0 ? k + R : k + R - 1)); };
+  auto ws = [&](int k) { return hws(C, DS, k); };
 
   double acc[5][NCB][NCA][W];  // retimed: pending fluxes ; gather: queue of E_f
 #pragma unroll
@@ -1982,15 +1992,11 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
 #define CST_HYP_HPAIR 0
 #endif
 constexpr bool HPAIR = CST_HYP_HPAIR && TBA == 16 && TBB % 2 == 0;  // two b-rows per warp
-#ifndef CST_HYP_XSPLIT
-#define CST_HYP_XSPLIT 0  // experiment: x-walk into two partial sums (even / odd positions)
-#endif
 #ifndef CST_TM_EARLY
 #define CST_TM_EARLY (CST_BMX * CST_BMY * CST_BMZ > 1)  // TMEM hypterm: ring fetch before in-plane
 #endif
 constexpr bool TM_EARLY = CST_TM_EARLY;
 
-__host__ __device__ constexpr int ws_base(int dir) { return 7 + (dir == 2 ? 0 : (dir == 1 ? 8 : 16)); }
 
 // E^d_f at one position from v = {cons1..4, q_d, q4}
 template <int DIR>
@@ -2006,21 +2012,23 @@ template <int DIR, int K0, int K1>
 __device__ __forceinline__ void hyp_acc(const Ctx& C, bool par, const double (&E)[5],
                                         double (&A)[5]) {
   constexpr bool V0 = K0 != 0 && K0 >= -R && K0 <= R, V1 = K1 != 0 && K1 >= -R && K1 <= R;
-  constexpr int I0 = V0 ? ws_base(DIR) + (K0 < 0 ? K0 + R : K0 + R - 1) : 0;
-  constexpr int I1 = V1 ? ws_base(DIR) + (K1 < 0 ? K1 + R : K1 + R - 1) : 0;
-  if constexpr (V0 && V1) {
-    const double w = par ? C.coef(I1) : C.coef(I0);
+  if constexpr (V0 && V1) {  // K1 = K0 - 1: both on the same side of 0, same sign
+    static_assert((K0 > 0) == (K1 > 0), "weights of one sign");
+    constexpr int I0 = ws_base(DIR) + (K0 < 0 ? -K0 : K0) - 1;
+    constexpr int I1 = ws_base(DIR) + (K1 < 0 ? -K1 : K1) - 1;
+    const double p = par ? C.coef(I1) : C.coef(I0);
+    const double w = K0 > 0 ? -p : p;
 #pragma unroll
     for (int f = 0; f < 5; ++f) A[f] = fma(w, E[f], A[f]);
   } else if constexpr (V0) {
     if (!par) {
 #pragma unroll
-      for (int f = 0; f < 5; ++f) A[f] = fma(C.coef(I0), E[f], A[f]);
+      for (int f = 0; f < 5; ++f) A[f] = fma(hws(C, DIR, K0), E[f], A[f]);
     }
   } else if constexpr (V1) {
     if (par) {
 #pragma unroll
-      for (int f = 0; f < 5; ++f) A[f] = fma(C.coef(I1), E[f], A[f]);
+      for (int f = 0; f < 5; ++f) A[f] = fma(hws(C, DIR, K1), E[f], A[f]);
     }
   }
 }
@@ -2032,7 +2040,6 @@ __device__ __forceinline__ void hyp_rows_a(const Ctx& C, const LD* ld, int la, i
   static_assert(XR == R, "even order");
   const bool odd = la & 1;
   const int e0 = la - XR - (int)odd;
-  double A2[5] = {0.0, 0.0, 0.0, 0.0, 0.0};
   static_for<0, R + 1>([&](auto CC) {
     constexpr int c = decltype(CC)::value;
     double2 v2[6];
@@ -2056,16 +2063,9 @@ __device__ __forceinline__ void hyp_rows_a(const Ctx& C, const LD* ld, int la, i
       }
       double E[5];
       hyp_e<DA>(v, E);
-      if constexpr (CST_HYP_XSPLIT && h == 1)  // experiment: second chain for odd positions
-        hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A2);
-      else
-        hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A);
+      hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A);
     });
   });
-  if constexpr (CST_HYP_XSPLIT) {
-#pragma unroll
-    for (int f = 0; f < 5; ++f) A[f] += A2[f];
-  }
 }
 
 // b-direction terms into A
@@ -2163,7 +2163,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
   for (int i = 0; i < NCB; ++i) lb[i] = merged_pos(i, tb, TBB, BMB);
   const long long col0 = (long long)g.a0 + (long long)g.b0 * g.st_b;
   // streamed-direction weights (as kernel_hyp_stream1): plane p adds ws[p-o] E_f(p) to o
-  auto ws = [&](int k) { return C.coef(7 + (DS == 1 ? 8 : 0) + (k < 0 ? k + R : k + R - 1)); };
+  auto ws = [&](int k) { return hws(C, DS, k); };
 
   if (warp == 0) tmem_alloc(tslot, TM_COLS);
   if (tid == 0) {

@@ -5,7 +5,7 @@
 
 #define CST_MAX_IN 8
 #define CST_MAX_OUT 5
-#define CST_MAX_COEF 32
+#define CST_MAX_COEF 27
 
 // Opaque CUtensorMap (128 bytes, 64-byte aligned), filled by cuTensorMapEncodeTiled.
 struct __attribute__((aligned(64))) cst_tmap {

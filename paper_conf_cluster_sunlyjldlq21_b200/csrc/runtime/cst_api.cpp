@@ -184,9 +184,9 @@ extern "C" cst_status cst_stencil_create(const cst_stencil_desc* desc, const cst
   h->desc = *desc;
   h->coeffs.assign(desc->coeffs, desc->coeffs + desc->n_coeffs);
   h->desc.coeffs = h->coeffs.data();
-  // kernel coefficient bank: the user's coefficients, plus for hypterm the streamed-
-  // direction weights ws[k] = -sign(k) dxinv_d a_|k| (k = -4..-1, 1..4) for d = z, y, x
-  // (z and y: the streamed direction; all three: the row-streamed in-plane terms)
+  // kernel coefficient bank: the user's coefficients, plus for hypterm the derivative
+  // weight magnitudes P_d[j] = dxinv_d a_j (j = 1..4) for d = z, y, x — the kernels apply
+  // w_d[k] = -sign(k) P_d[|k|] (streamed direction and row-streamed in-plane terms)
   h->kcoef = h->coeffs;
   if (kind == CST_RHS4) {
     // s_d^2 / 6 for the V terms, s_d s_i / 144 for the mixed pairs (0,1), (0,2), (1,2)
@@ -197,11 +197,7 @@ extern "C" cst_status cst_stencil_create(const cst_stencil_desc* desc, const cst
   }
   if (kind == CST_HYPTERM)
     for (int sdir : {2, 1, 0})
-      for (int k = -4; k <= 4; ++k) {
-        if (k == 0) continue;
-        const double a = h->coeffs[(k > 0 ? k : -k) - 1];
-        h->kcoef.push_back((k > 0 ? -1.0 : 1.0) * (h->coeffs[4 + sdir] * a));
-      }
+      for (int j = 1; j <= 4; ++j) h->kcoef.push_back(h->coeffs[4 + sdir] * h->coeffs[j - 1]);
   h->grid = *g;
   h->device = device;
   {

@@ -42,6 +42,9 @@ CASES = [
     (3, 4, (512, 512, 512), None, False),                      # hypterm default (TMEM)
     (3, 4, (512, 512, 512), dict(qstore=1, bm_y=1, tb_y=8, prefetch=3), False),
     (4, 2, (320, 320, 320), None, False),                      # rhs4 default
+    # hypterm register path with ld/st staging (tests/test_gpu_sweep.py "ldst-z")
+    (3, 4, (37, 29, 26), dict(tb_x=32, tb_y=4, bm_y=1, qstore=1, staging=2, prefetch=1,
+                              sb=8, use_constant=1), False),
 ]
 
 
