@@ -8,11 +8,14 @@ if absent).  A step = one sweep (one kernel launch) over inputs resident in HBM;
 1.18 GB arrays exceed the 126 MB L2, so no flush is needed between steps.
 N>1 (torchrun, one rank per GPU): weak scaling of the z-slab decomposition — every rank owns
 a 512^3 slab of a (512*N) x 512 x 512 grid and exchanges 4-plane halos with its neighbours
-(cst_dist_sweep, NCCL) every step.  value = all ranks' points / max-over-ranks time.
+every step (cst_dist_sweep: by default the boundary kernels store straight into the
+neighbours' halos over peer memory, --halo nccl selects NCCL send/recv overlapped with the
+interior).  value = all ranks' points / max-over-ranks time.
 
 Extra keys: roofline (dominant kernel = the sweep), cpu_baseline (the oracle on a bounded
 sample, rank 0 at N=1), e2e (cst_sweep_host: H2D + sweep + D2H through the C ABI), clocks
-(nvidia-smi during the timed region), gpu_launches.
+(NVML polled every 2 ms during the timed region, nvidia-smi as fallback), gpu_launches,
+other_configs (configs[0], [2], [3] and the NEXT rows, reported beside the headline).
 """
 from __future__ import annotations
 
@@ -76,7 +79,7 @@ class ClockSampler:
         self.thread = None
         self.proc = None
         self.rows = []
-        self.poll_s = float(os.environ.get("CST_BENCH_CLOCK_POLL_MS", "20")) / 1e3
+        self.poll_s = float(os.environ.get("CST_BENCH_CLOCK_POLL_MS", "2")) / 1e3
 
     def start(self):
         try:
@@ -329,7 +332,7 @@ def run_reference(args, rank, world):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="cst", choices=["cst", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -339,7 +342,6 @@ def main():
                     choices=["p2p", "nccl"],
                     help="N > 1: fused peer-memory halo stores (default) or NCCL send/recv")
     args = ap.parse_args()
-    assert args.warmup >= 3 or args.impl == "reference" or True
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))

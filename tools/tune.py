@@ -43,6 +43,10 @@ def main():
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--fix", action="append", default=[],
+                    help="field=value: tune the sub-space with this field fixed (e.g. "
+                         "staging=1); other candidates get fitness 0 through the evaluation "
+                         "callback (SURVEY §8(d) C3: each staging mode best-of-tuned)")
     args = ap.parse_args()
     kind, r, coeffs, n, seed = config(args.config)
     g = C.make_grid(*n, r)
@@ -57,10 +61,32 @@ def main():
     o.time_budget_s = args.budget
     o.reps = args.reps
     os.makedirs(os.path.join(ROOT, "tuned", "logs"), exist_ok=True)
-    log = os.path.join(ROOT, "tuned", "logs", f"{args.config}_seed{args.seed}.json")
+    tag = "".join(f"_{kv.replace('=', '')}" for kv in args.fix)
+    log = os.path.join(ROOT, "tuned", "logs", f"{args.config}{tag}_seed{args.seed}.json")
     o.log_path = log.encode()
+    fixed = {kv.split("=")[0]: int(kv.split("=")[1]) for kv in args.fix}
+    eval_fn = None
+    if fixed:
+        stream0 = torch.cuda.current_stream().cuda_stream
+
+        def eval_fn(settings):
+            ms = []
+            for st in settings:
+                d = st.as_dict()
+                if any(d[k] != v for k, v in fixed.items()):
+                    ms.append(float("inf"))
+                    continue
+                try:
+                    ms.append(C.cst_time_setting(h, st, [t.data_ptr() for t in ins],
+                                                 [t.data_ptr() for t in outs], 2, args.reps,
+                                                 stream0))
+                except C.CstError:
+                    ms.append(float("inf"))
+            return ms
+        o.warm_start = 0
     t0 = time.time()
-    best, rep = C.cst_tune(h, o, [t.data_ptr() for t in ins], [t.data_ptr() for t in outs])
+    best, rep = C.cst_tune(h, o, [t.data_ptr() for t in ins], [t.data_ptr() for t in outs],
+                           eval_fn)
     wall = time.time() - t0
     # re-time the winner and the default setting on the same buffers
     stream = torch.cuda.current_stream().cuda_stream
@@ -74,8 +100,9 @@ def main():
            "tuned_ms": rep.best_ms, "retimed_ms": ms_best, "gstencils": pts / (ms_best * 1e-3) / 1e9,
            "default_setting": dflt.as_dict(), "default_ms": ms_def,
            "report": {f: getattr(rep, f) for f, _ in rep._fields_}, "wall_s": wall,
-           "log": os.path.relpath(log, ROOT), "seed": args.seed, "budget_s": args.budget}
-    out = args.out or os.path.join(ROOT, "tuned", f"{args.config}_{n[0]}.json")
+           "log": os.path.relpath(log, ROOT), "seed": args.seed, "budget_s": args.budget,
+           "fixed": fixed}
+    out = args.out or os.path.join(ROOT, "tuned", f"{args.config}_{n[0]}{tag}.json")
     with open(out, "w") as f:
         json.dump(res, f, indent=1)
     print(json.dumps(res))
