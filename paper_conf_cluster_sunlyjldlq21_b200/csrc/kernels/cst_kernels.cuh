@@ -1992,6 +1992,9 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
 #define CST_HYP_HPAIR 0
 #endif
 constexpr bool HPAIR = CST_HYP_HPAIR && TBA == 16 && TBB % 2 == 0;  // two b-rows per warp
+#ifndef CST_HYP_WXPRE
+#define CST_HYP_WXPRE 1  // TMEM hypterm: per-lane x weights selected once per thread
+#endif
 #ifndef CST_TM_EARLY
 #define CST_TM_EARLY (CST_BMX * CST_BMY * CST_BMZ > 1)  // TMEM hypterm: ring fetch before in-plane
 #endif
@@ -2033,10 +2036,38 @@ __device__ __forceinline__ void hyp_acc(const Ctx& C, bool par, const double (&E
   }
 }
 
+// the lane's x weights at the walk positions where both parities have one (positions
+// 1..R-1 and R+2..2R: w = -sign(k) P_x[|k|] with k = j - XR - parity), selected once per
+// thread (CST_HYP_WXPRE) instead of once per position and plane
+struct HypWx {
+  double w[2 * R - 2 > 0 ? 2 * R - 2 : 1];
+};
+__device__ __forceinline__ HypWx hyp_wx(const Ctx& C, bool odd) {
+  HypWx W;
+  int n = 0;
+#pragma unroll
+  for (int j = 0; j < 2 * R + 2; ++j) {
+    const int k0 = j - XR, k1 = j - XR - 1;
+    const bool v0 = k0 != 0 && k0 >= -R && k0 <= R, v1 = k1 != 0 && k1 >= -R && k1 <= R;
+    if (v0 && v1) W.w[n++] = odd ? hws(C, DA, k1) : hws(C, DA, k0);
+  }
+  return W;
+}
+constexpr int hyp_wx_slot(int j) {  // index into HypWx::w of walk position j, -1 if none
+  int n = 0;
+  for (int i = 0; i < j; ++i) {
+    const int k0 = i - XR, k1 = i - XR - 1;
+    if (k0 != 0 && k0 >= -R && k0 <= R && k1 != 0 && k1 >= -R && k1 <= R) ++n;
+  }
+  const int k0 = j - XR, k1 = j - XR - 1;
+  return (k0 != 0 && k0 >= -R && k0 <= R && k1 != 0 && k1 >= -R && k1 <= R) ? n : -1;
+}
+
 // x-direction terms into A; the point's own cons1..4 and q4 into cen
 template <class LD>
 __device__ __forceinline__ void hyp_rows_a(const Ctx& C, const LD* ld, int la, int lb,
-                                           double (&A)[5], double (&cen)[5]) {
+                                           double (&A)[5], double (&cen)[5],
+                                           const HypWx* wx = nullptr) {
   static_assert(XR == R, "even order");
   const bool odd = la & 1;
   const int e0 = la - XR - (int)odd;
@@ -2063,7 +2094,13 @@ __device__ __forceinline__ void hyp_rows_a(const Ctx& C, const LD* ld, int la, i
       }
       double E[5];
       hyp_e<DA>(v, E);
-      hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A);
+      constexpr int ws_i = hyp_wx_slot(j);
+      if (ws_i >= 0 && wx != nullptr) {
+#pragma unroll
+        for (int f = 0; f < 5; ++f) A[f] = fma(wx->w[ws_i < 0 ? 0 : ws_i], E[f], A[f]);
+      } else {
+        hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A);
+      }
     });
   });
 }
@@ -2174,6 +2211,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
   __syncthreads();
   tmem_fence_after_sync();
   const u32 tq = *tslot + ((u32)((warp & 3) * 32) << 16) + (u32)((warp >> 2) * NPT * TM_PCOLS);
+  const HypWx wxl = hyp_wx(C, la[0] & 1);
   if (tid == 0)
     for (int j = 0; j < D && j < n_planes; ++j) {
       mbar_arrive_expect_tx(&bars[j % NP], TX_BYTES);
@@ -2227,7 +2265,8 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 #pragma unroll
             for (int f = 0; f < 5; ++f) A[ib][f] = Ab[ib][f] = 0.0;
 #pragma unroll
-          for (int ib = 0; ib < NCB; ++ib) hyp_rows_a(C, ld, la[0], lb[ib], A[ib], cen[ib]);
+          for (int ib = 0; ib < NCB; ++ib)
+            hyp_rows_a(C, ld, la[0], lb[ib], A[ib], cen[ib], CST_HYP_WXPRE ? &wxl : nullptr);
           if constexpr (NCB == 1 && HPAIR)
             hyp_rows_b(C, ld, la[0], lb[0], Ab[0]);
           else
