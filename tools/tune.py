@@ -43,6 +43,9 @@ def main():
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--refine", action="store_true",
+                    help="after cst_tune: hill-climb the winner over its SB and prefetch "
+                         "neighbours, re-timed (ours, not the paper's; reported separately)")
     ap.add_argument("--fix", action="append", default=[],
                     help="field=value: tune the sub-space with this field fixed (e.g. "
                          "staging=1); other candidates get fitness 0 through the evaluation "
@@ -95,13 +98,40 @@ def main():
     dflt = C.cst_setting_default(h)
     ms_def = C.cst_time_setting(h, dflt, [t.data_ptr() for t in ins], [t.data_ptr() for t in outs],
                                 3, 20, stream)
+    refine = None
+    if args.refine:
+        def timed(st):
+            try:
+                C.cst_setting_check(h, st)
+                return C.cst_time_setting(h, st, [t.data_ptr() for t in ins],
+                                          [t.data_ptr() for t in outs], 3, 20, stream)
+            except C.CstError:
+                return float("inf")
+        cur, cur_ms, steps = best.as_dict(), ms_best, []
+        for _ in range(3):
+            cands = []
+            for f, vals in (("sb", (cur["sb"] // 2, cur["sb"] * 2)),
+                            ("prefetch", (cur["prefetch"] - 1, cur["prefetch"] + 1))):
+                for v in vals:
+                    if v >= 1:
+                        cands.append(dict(cur, **{f: v}))
+            timed_c = [(timed(C.cst_setting.from_dict(d)), d) for d in cands]
+            ms_c, d_c = min(timed_c, key=lambda x: x[0])
+            steps.append({"from_ms": cur_ms, "neighbours": [[m, {k: d[k] for k in ("sb", "prefetch")}]
+                                                            for m, d in timed_c]})
+            if ms_c < 0.99 * cur_ms:
+                cur, cur_ms = d_c, ms_c
+            else:
+                break
+        refine = {"tuned_setting": best.as_dict(), "tuned_retimed_ms": ms_best, "steps": steps}
+        best, ms_best = C.cst_setting.from_dict(cur), cur_ms
     pts = n[0] * n[1] * n[2]
     res = {"config": args.config, "grid": list(n), "setting": best.as_dict(),
            "tuned_ms": rep.best_ms, "retimed_ms": ms_best, "gstencils": pts / (ms_best * 1e-3) / 1e9,
            "default_setting": dflt.as_dict(), "default_ms": ms_def,
            "report": {f: getattr(rep, f) for f, _ in rep._fields_}, "wall_s": wall,
            "log": os.path.relpath(log, ROOT), "seed": args.seed, "budget_s": args.budget,
-           "fixed": fixed}
+           "fixed": fixed, "refine": refine}
     out = args.out or os.path.join(ROOT, "tuned", f"{args.config}_{n[0]}{tag}.json")
     with open(out, "w") as f:
         json.dump(res, f, indent=1)
