@@ -4,6 +4,8 @@ tuned setting (used by bench.py) plus the tuner's stage-by-stage JSON report.
     python tools/tune.py --config star25      # BASELINE configs[1]: order-4 star, 512^3
     python tools/tune.py --config box27       # configs[2]
     python tools/tune.py --config hypterm     # configs[3]
+    python tools/tune.py --config star25 --start tuned/star25_512.json --refine-all
+                                              # hill climb from a recorded setting
 """
 import argparse
 import json
@@ -19,6 +21,10 @@ import torch  # noqa: E402
 from paper_conf_cluster_sunlyjldlq21_b200 import cst as C  # noqa: E402
 
 D2_R4 = [-9, 128, -1008, 8064, -14350, 8064, -1008, 128, -9]
+
+
+SIZE_FIELDS = {"tb_x", "tb_y", "tb_z", "sb", "uf_x", "uf_y", "uf_z", "cm_x", "cm_y", "cm_z",
+               "bm_x", "bm_y", "bm_z", "bt"}
 
 
 def config(name):
@@ -46,6 +52,12 @@ def main():
     ap.add_argument("--refine", action="store_true",
                     help="after cst_tune: hill-climb the winner over its SB and prefetch "
                          "neighbours, re-timed (ours, not the paper's; reported separately)")
+    ap.add_argument("--refine-all", action="store_true",
+                    help="with --refine: the neighbourhood is every field one step away "
+                         "(x2 / /2 for sizes, +-1 for enumerated fields), not only SB/prefetch")
+    ap.add_argument("--start", default=None,
+                    help="tuned JSON to refine from: skips cst_tune and hill-climbs from its "
+                         "setting (implies --refine)")
     ap.add_argument("--fix", action="append", default=[],
                     help="field=value: tune the sub-space with this field fixed (e.g. "
                          "staging=1); other candidates get fitness 0 through the evaluation "
@@ -88,8 +100,14 @@ def main():
             return ms
         o.warm_start = 0
     t0 = time.time()
-    best, rep = C.cst_tune(h, o, [t.data_ptr() for t in ins], [t.data_ptr() for t in outs],
-                           eval_fn)
+    if args.start:
+        with open(args.start) as f:
+            best = C.cst_setting.from_dict(json.load(f)["setting"])
+        rep = None
+        args.refine = True
+    else:
+        best, rep = C.cst_tune(h, o, [t.data_ptr() for t in ins], [t.data_ptr() for t in outs],
+                               eval_fn)
     wall = time.time() - t0
     # re-time the winner and the default setting on the same buffers
     stream = torch.cuda.current_stream().cuda_stream
@@ -102,23 +120,29 @@ def main():
     if args.refine:
         def timed(st):
             try:
+                st = C.cst_setting.from_dict(st) if isinstance(st, dict) else st
                 C.cst_setting_check(h, st)
                 return C.cst_time_setting(h, st, [t.data_ptr() for t in ins],
                                           [t.data_ptr() for t in outs], 3, 20, stream)
-            except C.CstError:
+            except (C.CstError, ValueError, OverflowError):
                 return float("inf")
         cur, cur_ms, steps = best.as_dict(), ms_best, []
         for _ in range(3):
             cands = []
-            for f, vals in (("sb", (cur["sb"] // 2, cur["sb"] * 2)),
-                            ("prefetch", (cur["prefetch"] - 1, cur["prefetch"] + 1))):
+            moves = (("sb", (cur["sb"] // 2, cur["sb"] * 2)),
+                     ("prefetch", (cur["prefetch"] - 1, cur["prefetch"] + 1)))
+            if args.refine_all:
+                moves = [(f, (v // 2, v * 2) if f in SIZE_FIELDS else (v - 1, v + 1))
+                         for f, v in cur.items() if f not in fixed]
+            for f, vals in moves:
                 for v in vals:
-                    if v >= 1:
+                    if v >= 1 or (f not in SIZE_FIELDS and v >= 0):
                         cands.append(dict(cur, **{f: v}))
-            timed_c = [(timed(C.cst_setting.from_dict(d)), d) for d in cands]
+            timed_c = [(timed(d), d) for d in cands]
             ms_c, d_c = min(timed_c, key=lambda x: x[0])
-            steps.append({"from_ms": cur_ms, "neighbours": [[m, {k: d[k] for k in ("sb", "prefetch")}]
-                                                            for m, d in timed_c]})
+            steps.append({"from_ms": cur_ms,
+                          "neighbours": [[m, {k: v for k, v in d.items() if cur[k] != v}]
+                                         for m, d in timed_c]})
             if ms_c < 0.99 * cur_ms:
                 cur, cur_ms = d_c, ms_c
             else:
@@ -127,11 +151,14 @@ def main():
         best, ms_best = C.cst_setting.from_dict(cur), cur_ms
     pts = n[0] * n[1] * n[2]
     res = {"config": args.config, "grid": list(n), "setting": best.as_dict(),
-           "tuned_ms": rep.best_ms, "retimed_ms": ms_best, "gstencils": pts / (ms_best * 1e-3) / 1e9,
+           "tuned_ms": rep.best_ms if rep else None, "retimed_ms": ms_best, "gstencils": pts / (ms_best * 1e-3) / 1e9,
            "default_setting": dflt.as_dict(), "default_ms": ms_def,
-           "report": {f: getattr(rep, f) for f, _ in rep._fields_}, "wall_s": wall,
+           "report": {f: getattr(rep, f) for f, _ in rep._fields_} if rep else None,
+           "wall_s": wall, "start": args.start,
            "log": os.path.relpath(log, ROOT), "seed": args.seed, "budget_s": args.budget,
            "fixed": fixed, "refine": refine}
+    if args.start:
+        tag += "_refined"
     out = args.out or os.path.join(ROOT, "tuned", f"{args.config}_{n[0]}{tag}.json")
     with open(out, "w") as f:
         json.dump(res, f, indent=1)
