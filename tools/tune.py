@@ -27,6 +27,23 @@ SIZE_FIELDS = {"tb_x", "tb_y", "tb_z", "sb", "uf_x", "uf_y", "uf_z", "cm_x", "cm
                "bm_x", "bm_y", "bm_z", "bt"}
 
 
+def neighbours(cur, fixed=(), full=False):
+    """Settings one step away from `cur`: SB x2 / /2 and prefetch +-1, or (full) every field
+    not in `fixed` (sizes x2 / /2, enumerated fields +-1). Validity is left to
+    cst_setting_check; only values below a field's minimum are dropped here."""
+    moves = [("sb", (cur["sb"] // 2, cur["sb"] * 2)),
+             ("prefetch", (cur["prefetch"] - 1, cur["prefetch"] + 1))]
+    if full:
+        moves = [(f, (v // 2, v * 2) if f in SIZE_FIELDS else (v - 1, v + 1))
+                 for f, v in cur.items() if f not in fixed]
+    out = []
+    for f, vals in moves:
+        for v in vals:
+            if v != cur[f] and (v >= 1 or (f not in SIZE_FIELDS and v >= 0)):
+                out.append(dict(cur, **{f: v}))
+    return out
+
+
 def config(name):
     if name == "star25":
         w = [v / 5040.0 for v in D2_R4]
@@ -128,16 +145,7 @@ def main():
                 return float("inf")
         cur, cur_ms, steps = best.as_dict(), ms_best, []
         for _ in range(3):
-            cands = []
-            moves = (("sb", (cur["sb"] // 2, cur["sb"] * 2)),
-                     ("prefetch", (cur["prefetch"] - 1, cur["prefetch"] + 1)))
-            if args.refine_all:
-                moves = [(f, (v // 2, v * 2) if f in SIZE_FIELDS else (v - 1, v + 1))
-                         for f, v in cur.items() if f not in fixed]
-            for f, vals in moves:
-                for v in vals:
-                    if v >= 1 or (f not in SIZE_FIELDS and v >= 0):
-                        cands.append(dict(cur, **{f: v}))
+            cands = neighbours(cur, fixed, args.refine_all)
             timed_c = [(timed(d), d) for d in cands]
             ms_c, d_c = min(timed_c, key=lambda x: x[0])
             steps.append({"from_ms": cur_ms,
