@@ -3,8 +3,8 @@
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl cst|reference]
 
 N=1 workload: order-4 25-point star (FD Laplacian, weights /5040), 512^3 FP64 interior,
-halo 4, the tuned setting from tuned/star25_512.json (cst_tune output; the default setting
-if absent).  A step = one sweep (one kernel launch) over inputs resident in HBM; the two
+halo 4, the tuned setting from tuned/star25_512.json (cst_tune output, then the A/B-checked
+hill climb of tools/tune.py --refine-all; the default setting if absent).  A step = one sweep (one kernel launch) over inputs resident in HBM; the two
 1.18 GB arrays exceed the 126 MB L2, so no flush is needed between steps.
 N>1 (torchrun, one rank per GPU): weak scaling of the z-slab decomposition — every rank owns
 a 512^3 slab of a (512*N) x 512 x 512 grid and exchanges 4-plane halos with its neighbours
