@@ -148,6 +148,13 @@ cst_status cst_kernel_info_get(cst_stencil* h, const cst_setting* s, cst_kernel_
 /* Code generation only: generate and NVRTC-compile the sm_100a variant of a valid
  * setting into the cubin cache; needs no GPU.  *compile_s = seconds (0 on a cache hit). */
 cst_status cst_variant_compile(const cst_stencil* h, const cst_setting* s, double* compile_s);
+/* The generated code itself: copy the sm_100a cubin of a valid setting's variant
+ * (compiled if needed; no GPU) into buf[cap].  *size = cubin bytes, always set; if cap is
+ * smaller than that nothing is copied and CST_E_INVALID is returned (call with cap = 0 to
+ * size the buffer).  remote = 1 selects the fused-halo twin (CST_REMOTE).  Used to audit
+ * that distinct settings generate distinct code (tests/test_codegen_distinct.py). */
+cst_status cst_variant_cubin(const cst_stencil* h, const cst_setting* s, int32_t remote,
+                             void* buf, int64_t cap, int64_t* size);
 
 /* One sweep (nsteps = 1) or nsteps ping-pong sweeps over DEVICE buffers, asynchronous on
  * `stream`.  in[n_inputs], out[n_outputs].  nsteps = 1: only interior points of out[] are

@@ -29,15 +29,18 @@ Space (readings Q14/Q15 of SURVEY.md §8(c)):
 
 Rules: paper R1 prod TB <= 1024; R2 SD=SB=1 when streaming off; R3 UF_SD <= SB when
 streaming on.  Ours (Q15): R4 prod TB >= 32; R5 T_d = TB_d*BM_d*CM_d <= E_d (E_d = M_d,
-E_SD = SB when streaming); R6 UF_d <= trip_d (trip_d = BM_d*CM_d; trip_SD = SB / T_SD when
-streaming); R7 prod(BM*CM) <= 16; R8 streaming => SD != 1; R9 prefetch > 1 => streaming;
+E_SD = SB when streaming); R6 UF_d <= trip_d, the trip count of the loop the kernel path
+unrolls along d (uf_trip; 1 where there is none); R7 prod(BM*CM) <= 16; R8 streaming =>
+SD != 1; R9 prefetch > 1 => streaming with staging (nothing to prefetch into otherwise);
 R10 modelled smem <= SMEM_LIMIT; R11 modelled registers <= 255; R12 TMA box: T_x even and
 every box extent <= 256; R14 bt > 1 only for the temporally blocked path: star / box,
 streaming along z with T_SD = 1, TMA staging, retimed accumulators, no cyclic merging,
 BM_x, BM_y <= 2, every UF = 1 (reading Q23); R15 qstore = 2 only for the
 TMEM path: star or hypterm (hypterm: one point along x, BM_b <= 2 along the other in-plane
 dim, no cyclic merging), streaming with T_SD = 1, TMA staging, retimed, bt = 1, and
-ceil(threads/128) * points per thread * (4r star, 20r hypterm) <= 512 TMEM columns.
+ceil(threads/128) * points per thread * (4r star, 20r hypterm) <= 512 TMEM columns;
+R16 rhs4: use_retiming = 1 (its kernels have one summation form).  R6/R9/R16 keep every
+field a kernel path does not read at its canonical value (round 2; tools/knob_audit.py).
 """
 from __future__ import annotations
 
@@ -187,6 +190,30 @@ def est_regs(kind: int, r: int, s: dict) -> int:
     return 32 + 2 * ppt * live_doubles_per_point(kind, r) + 2 * pf
 
 
+def uf_trip(kind: int, s: dict, d: int) -> int:
+    """R6: trip count of the per-thread loop that the setting's kernel path unrolls along
+    dim d (loop unrolling), 1 where that path has no such loop (UF_d then stays at
+    its canonical 1, so no two settings generate the same code — tools/knob_audit.py):
+      streaming off (3-D tiles) and generic streaming (T_SD > 1, or rhs4): the merged-point
+        loop, BM_d * CM_d;
+      fast streaming paths (star / box / hypterm, T_SD = 1): no in-plane loop (the block is
+        register-unrolled); along SD the plane loop, SB planes, which the compiler unrolls
+        for star / box with TMA or no staging (not ld/st staging, not the hypterm, TMEM or
+        temporally blocked kernels)."""
+    a = "xyz"[d]
+    bmcm = s["bm_" + a] * s["cm_" + a]
+    if s["use_streaming"] == 1:
+        return bmcm
+    sd = s["sd"] - 1
+    if not (kind in (STAR, BOX, HYPTERM) and tiles(s)[sd] == 1):
+        return bmcm
+    if d != sd:
+        return 1
+    if kind in (STAR, BOX) and s["qstore"] == 1 and s["bt"] == 1 and s["staging"] != 2:
+        return s["sb"]
+    return 1
+
+
 def tma_ok(r: int, s: dict) -> bool:
     T = tiles(s)
     if T[0] % 2:
@@ -222,20 +249,21 @@ def check(kind: int, r: int, M, s: dict):
     if stream and s["uf_" + "xyz"[sd]] > s["sb"]:
         return "R3"
     for d in range(3):
-        trip = s["sb"] // T[d] if (stream and d == sd) else s["bm_" + "xyz"[d]] * s["cm_" + "xyz"[d]]
-        if s["uf_" + "xyz"[d]] > trip:
+        if s["uf_" + "xyz"[d]] > uf_trip(kind, s, d):
             return "R6"
     ppt = 1
     for d in "xyz":
         ppt *= s["bm_" + d] * s["cm_" + d]
     if ppt > 16:
         return "R7"
-    if s["prefetch"] > 1 and not stream:
+    if s["prefetch"] > 1 and (not stream or s["staging"] == 1):
         return "R9"
     if s["bt"] > 1 and not tb_path_ok(kind, s):
         return "R14"
     if s["qstore"] == 2 and not qs_path_ok(kind, r, s):
         return "R15"
+    if kind == RHS4 and s["use_retiming"] != 1:
+        return "R16"
     if smem_bytes(kind, r, s) > SMEM_LIMIT:
         return "R10"
     if est_regs(kind, r, s) > REG_LIMIT:

@@ -267,7 +267,7 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
   for (int d = 0; d < 3; ++d) c.uf[d] = c.cm[d] = c.bm[d] = 1;
   c.bm[0] = hyp ? 1 : 2;
   c.bm[1] = hyp && !hyp_tm ? 1 : 2;
-  c.use_retiming = 2;
+  c.use_retiming = h->info.kind == CST_RHS4 ? 1 : 2;  // R16: rhs4 has one summation form
   c.bt = 1;
   c.qstore = hyp_tm ? 2 : 1;
   if (hyp_tm) c.use_constant = 2;
@@ -401,6 +401,22 @@ extern "C" cst_status cst_variant_compile(const cst_stencil* h, const cst_settin
   if (rule) return fail(CST_E_CONSTRAINT, std::string("setting violates ") + rule);
   std::string cubin;
   return jit_cubin(h->info, t, &cubin, compile_s);
+}
+
+extern "C" cst_status cst_variant_cubin(const cst_stencil* h, const cst_setting* s,
+                                        int32_t remote, void* buf, int64_t cap, int64_t* size) {
+  if (!h || !s || !size || (cap > 0 && !buf)) return fail(CST_E_INVALID, "null argument");
+  const Tuple t = to_tuple(*s);
+  const char* rule = check_rules(h->info, t);
+  if (rule) return fail(CST_E_CONSTRAINT, std::string("setting violates ") + rule);
+  std::string cubin;
+  double cs = 0;
+  const cst_status st = jit_cubin(h->info, t, &cubin, &cs, remote != 0);
+  if (st != CST_OK) return st;
+  *size = (int64_t)cubin.size();
+  if (cap < (int64_t)cubin.size()) return fail(CST_E_INVALID, "cst_variant_cubin: buffer too small");
+  std::memcpy(buf, cubin.data(), cubin.size());
+  return CST_OK;
 }
 
 extern "C" cst_status cst_kernel_info_get(cst_stencil* h, const cst_setting* s,

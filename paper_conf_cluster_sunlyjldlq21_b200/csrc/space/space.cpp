@@ -272,6 +272,26 @@ static bool tma_ok(int r, const Tuple& t) {
   return true;
 }
 
+// R6: trip count of the per-thread loop the kernel path unrolls along dim d (loop
+// unrolling); 1 where the path has no such loop, so UF_d stays at its canonical 1
+// and no two settings generate the same code (tools/knob_audit.py).  Streaming off and
+// generic streaming (T_SD > 1, rhs4): the merged-point loop BM_d*CM_d.  Fast streaming
+// paths (star/box/hypterm, T_SD = 1): no in-plane loop; along SD the plane loop (SB), which
+// is unrolled for star/box with TMA or no staging in the register-state, unfused kernel.
+int64_t uf_trip(int kind, const Tuple& t, int d) {
+  const int64_t bmcm = (int64_t)t[F_BMX + d] * t[F_CMX + d];
+  if (t[F_STREAM] != 2) return bmcm;
+  const int sd = t[F_SD] - 1;
+  const bool fast = (kind == CST_STAR || kind == CST_BOX || kind == CST_HYPTERM) &&
+                    (int64_t)t[F_TBX + sd] * t[F_BMX + sd] * t[F_CMX + sd] == 1;
+  if (!fast) return bmcm;
+  if (d != sd) return 1;
+  if ((kind == CST_STAR || kind == CST_BOX) && t[F_QS] == 1 && t[F_BT] == 1 &&
+      t[F_STAGING] != 2)
+    return t[F_SB];
+  return 1;
+}
+
 static bool is_p2(int64_t v) { return v >= 1 && (v & (v - 1)) == 0; }
 
 const char* check_rules(const StencilInfo& st, const Tuple& t) {
@@ -309,17 +329,15 @@ const char* check_rules(const StencilInfo& st, const Tuple& t) {
     if (T[d] > E) return "R5";
   }
   if (stream && t[F_UFX + sd] > t[F_SB]) return "R3";
-  for (int d = 0; d < 3; ++d) {
-    const int64_t trip = (stream && d == sd) ? t[F_SB] / T[d]
-                                             : (int64_t)t[F_BMX + d] * t[F_CMX + d];
-    if (t[F_UFX + d] > trip) return "R6";
-  }
+  for (int d = 0; d < 3; ++d)
+    if (t[F_UFX + d] > uf_trip(st.kind, t, d)) return "R6";
   int64_t ppt = 1;
   for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
   if (ppt > 16) return "R7";
-  if (t[F_PF] > 1 && !stream) return "R9";
+  if (t[F_PF] > 1 && (!stream || t[F_STAGING] == 1)) return "R9";
   if (t[F_BT] > 1 && !tb_path_ok(st.kind, t)) return "R14";
   if (t[F_QS] == 2 && !qs_path_ok(st.kind, st.r, t)) return "R15";
+  if (st.kind == CST_RHS4 && t[F_RET] != 1) return "R16";
   if (model_smem_bytes(st.kind, st.r, t) > SMEM_LIMIT) return "R10";
   if (model_regs(st.kind, st.r, t) > REG_LIMIT) return "R11";
   if (t[F_STAGING] == 3 && !tma_ok(st.r, t)) return "R12";
@@ -379,9 +397,8 @@ void Space::cores_for(const int32_t* pre, std::vector<Core>* cores) const {
                   for (int d = 0; d < 3; ++d) {
                     c.cm[d] = cm[d];
                     c.bm[d] = bm[d];
-                    const int64_t Td = (int64_t)pre[F_TBX + d] * cm[d] * bm[d];
-                    const int64_t trip = (stream && d == sd) ? pre[F_SB] / Td
-                                                             : (int64_t)cm[d] * bm[d];
+                    int64_t trip = uf_trip(st_.kind, t, d);
+                    if (stream && d == sd) trip = std::min<int64_t>(trip, pre[F_SB]);  // R3
                     c.nuf[d] = bt > 1 ? 1 : count_le(p2_[d], trip);
                   }
                   c.ret = ret;

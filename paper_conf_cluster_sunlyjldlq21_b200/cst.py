@@ -164,6 +164,8 @@ _decl("cst_space_at", _S, _P, ctypes.c_uint64, ctypes.POINTER(cst_setting))
 _decl("cst_space_rank", _S, _P, ctypes.POINTER(cst_setting), ctypes.POINTER(ctypes.c_uint64))
 _decl("cst_kernel_info_get", _S, _P, ctypes.POINTER(cst_setting), ctypes.POINTER(cst_kernel_info))
 _decl("cst_variant_compile", _S, _P, ctypes.POINTER(cst_setting), ctypes.POINTER(ctypes.c_double))
+_decl("cst_variant_cubin", _S, _P, ctypes.POINTER(cst_setting), ctypes.c_int32, _P, ctypes.c_int64,
+      ctypes.POINTER(ctypes.c_int64))
 _decl("cst_sweep", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP, ctypes.c_int32, _P)
 _decl("cst_sweep_host", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP, ctypes.c_int32)
 _decl("cst_sync", _S, _P)
@@ -272,6 +274,16 @@ def cst_variant_compile(h, s: cst_setting) -> float:
     t = ctypes.c_double()
     check(_lib.cst_variant_compile(h, ctypes.byref(s), ctypes.byref(t)))
     return t.value
+
+
+def cst_variant_cubin(h, s: cst_setting, remote: bool = False) -> bytes:
+    n = ctypes.c_int64()
+    rc = _lib.cst_variant_cubin(h, ctypes.byref(s), int(remote), None, 0, ctypes.byref(n))
+    if rc not in (0, 1) or n.value == 0:
+        check(rc)
+    buf = ctypes.create_string_buffer(n.value)
+    check(_lib.cst_variant_cubin(h, ctypes.byref(s), int(remote), buf, n.value, ctypes.byref(n)))
+    return buf.raw[:n.value]
 
 
 def cst_sweep(h, s: cst_setting, in_ptrs, out_ptrs, nsteps: int = 1, stream: int = 0) -> None:

@@ -66,11 +66,11 @@ PATH_SETTINGS = [
     ("const-mem", S(use_constant=2)),
     ("sd-y", S(tb_y=1, tb_z=4, sd=2)),
     ("sd-y-ldst-gather", S(tb_y=1, tb_z=4, sd=2, staging=2, use_retiming=1)),
-    ("merge-bm-cm", S(tb_x=16, cm_x=2, bm_y=2, uf_y=2)),
+    ("merge-bm-cm", S(tb_x=16, cm_x=2, bm_y=2)),
     ("sb1", S(sb=1, prefetch=1)),
     ("generic-TS2-tma", S(tb_y=2, tb_z=2)),
     ("generic-TS2-ldst", S(tb_y=2, tb_z=2, staging=2)),
-    ("generic-TS2-none", S(tb_y=2, tb_z=2, staging=1)),
+    ("generic-TS2-none", S(tb_y=2, tb_z=2, staging=1, prefetch=1)),
     ("generic-bmz2", S(bm_z=2, uf_z=1, sb=8)),
     ("tile3d-none", S(tb_x=16, tb_y=2, tb_z=2, staging=1, **NOSTREAM)),
     ("tile3d-ldst", S(tb_x=16, tb_y=2, tb_z=2, staging=2, **NOSTREAM)),
@@ -154,7 +154,7 @@ def test_rhs4_paired_points_ragged(name, kw):
     c = H.coeffs(kind, r, "random", seed=9)
     ins = H.inputs(kind, L, seed=13, poison_beyond=r)
     _, want = H.oracle_outputs(kind, r, c, L, ins)
-    _, got = run_gpu(kind, r, c, L, ins, S(sb=8, uf_z=1, **kw))
+    _, got = run_gpu(kind, r, c, L, ins, S(sb=8, uf_z=1, use_retiming=1, **kw))
     for o in range(ost.N_OUT[kind]):
         H.assert_parity(L, got[o], want[o], f"{name} out{o}")
         H.assert_halo_untouched(L, got[o], np.full(L.numel, np.nan))

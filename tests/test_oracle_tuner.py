@@ -154,6 +154,24 @@ def test_space_rules_spot_checks():
     assert S.check(1, 4, M, dict(base, tb_x=8, tb_y=2)) == "R4"
     assert S.check(1, 4, M, dict(base, tb_z=2, bm_z=64)) == "R5"
     assert S.check(1, 4, M, dict(base, uf_x=2)) == "R6"
+    # R6 with the path's loop (round 2, tools/knob_audit.py): on the fast streaming path the
+    # in-plane block is register-unrolled (no UF_x / UF_y loop) even when BM > 1; along z the
+    # plane loop (<= SB) is unrolled for star/box with TMA, but not with ld/st staging, TMEM or
+    # for the hypterm; the generic path (T_z > 1) unrolls the merged-point loop BM_z * CM_z
+    assert S.check(1, 4, M, dict(base, bm_y=2, uf_y=2)) == "R6"
+    assert S.check(1, 4, M, dict(base, uf_z=64)) is None
+    assert S.check(1, 4, M, dict(base, uf_z=2, staging=2)) == "R6"
+    assert S.check(1, 4, M, dict(base, uf_z=2, qstore=2)) == "R6"
+    assert S.check(3, 4, M, dict(base, uf_z=2)) == "R6"
+    assert S.check(1, 4, M, dict(base, tb_y=2, tb_z=2, uf_z=2)) == "R6"
+    assert S.check(1, 4, M, dict(base, tb_y=2, tb_z=2, bm_z=2, uf_z=2)) is None
+    assert S.check(1, 4, M, dict(base, use_streaming=1, sd=1, sb=1, prefetch=1, bm_y=2,
+                                 uf_y=2)) is None
+    # R9: no staging -> nothing to prefetch; R16: rhs4 has one summation form
+    assert S.check(1, 4, M, dict(base, staging=1)) == "R9"
+    assert S.check(1, 4, M, dict(base, staging=1, prefetch=1)) is None
+    assert S.check(4, 2, M, dict(base, tb_x=16, tb_y=8)) == "R16"
+    assert S.check(4, 2, M, dict(base, tb_x=16, tb_y=8, use_retiming=1)) is None
     assert S.check(1, 4, M, dict(base, bm_y=8, cm_y=4)) == "R7"
     assert S.check(1, 4, M, dict(base, sd=1)) == "R8"
     assert S.check(1, 4, M, dict(base, use_streaming=1, sd=1, sb=1, prefetch=2)) == "R9"
@@ -169,7 +187,7 @@ def test_space_rules_spot_checks():
     assert S.check(2, 1, M, dict(tb, staging=2)) == "R14"
     assert S.check(2, 1, M, dict(tb, use_retiming=1)) == "R14"
     assert S.check(2, 1, M, dict(tb, sd=2, sb=64)) == "R14"
-    assert S.check(2, 1, M, dict(tb, uf_z=2)) == "R14"
+    assert S.check(2, 1, M, dict(tb, uf_z=2)) == "R6"          # the fused kernel unrolls no plane loop
     assert S.check(2, 1, M, dict(tb, bm_x=4, tb_x=16)) == "R14"
     assert S.check(2, 1, M, dict(tb, cm_x=2, tb_x=16)) == "R14"
     # box r=1, tile 64x8, bt=2, 2 stages: input box (64+2*2*2)x(8+2*2) = 72x12 doubles
