@@ -238,18 +238,29 @@ typedef struct {
                                 fitness is ms per step.  With nsteps = 1 a setting is
                                 timed as its bt = 1 twin; with nsteps > 1 the built-in
                                 evaluator times ping-pong on its own device copies   */
+  int32_t noise_reps;        /* 8: re-evaluate the dataset's best setting this many
+                                times; the CV of those fitness values (timing noise)
+                                sets the approximation threshold to
+                                max(cv_threshold, 2 * noise CV) (Q18); 0 =
+                                cv_threshold as given                                */
+  int32_t filter_threads;    /* host threads streaming the whole valid space through
+                                the PMNF threshold filter (0 = all cores)             */
 } cst_tune_opts;
 
 typedef struct {
   double best_ms;            /* median ms of the best setting                   */
   double best_gstencils;     /* interior points / best time                     */
   uint64_t space_count;      /* valid settings                                   */
-  uint64_t sampled_count;    /* settings kept by the PMNF threshold filter       */
+  uint64_t sampled_count;    /* settings of the whole valid space kept by the PMNF
+                                threshold filter (counted exactly)        */
   uint64_t evaluations;      /* distinct settings timed (incl. dataset)          */
   uint64_t jit_compiles;
   double wall_s, eval_s, jit_s, preproc_s;
   int32_t n_groups;
   int32_t generations;
+  int32_t phases_cv_stop;    /* GA phases ended by the CV_top-n approximation */
+  double noise_cv;           /* CV of the noise_reps re-evaluations (0 if none)      */
+  double cv_threshold_used;  /* the approximation threshold applied               */
 } cst_tune_report;
 
 void cst_tune_opts_default(cst_tune_opts* o);

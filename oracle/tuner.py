@@ -18,7 +18,10 @@ Readings (restated in DESIGN.md §2):
       exactly one collected metric joins that metric's collection; otherwise skipped.
 * Q12 PMNF (Eq. 3): f = sum_k c_k prod_{l in G_k} P_l^i log2(P_l)^j, raw values, no
       intercept; least squares; RSE = sqrt(SSR / (m - rank)); min RSE over I x J.
-* Q13 thresholds: one common order-statistic index t over a quantile sample of the space.
+* Q13 thresholds: one common order-statistic index t over a quantile sample of the space
+      (the smallest t whose pass fraction is >= the sampling ratio); the sampled space is
+      then every setting of the whole valid space that passes (sampled_space), and the GA's
+      gene tables are its per-group projections (gene_tables).
 """
 from __future__ import annotations
 
@@ -291,6 +294,24 @@ def threshold_filter(preds: np.ndarray, directions, ratio: float):
         else:
             lo = mid + 1
     return lo, thr(lo)
+
+
+def sampled_space(X: np.ndarray, groups, chosen_fits, directions, th) -> np.ndarray:
+    """P:290-292 ("filter out inappropriate parameter settings during the sampling
+    process"), reading Q13: every setting of the WHOLE valid space (rows of X, raw values)
+    whose predicted selected metrics all pass their thresholds (pred <= th for a metric
+    that grows with time, >= th otherwise).  Returns the boolean keep mask."""
+    keep = np.ones(X.shape[0], bool)
+    for fit, d, t in zip(chosen_fits, directions, th):
+        p = pmnf_predict(groups, X, fit)
+        keep &= (p <= t) if d > 0 else (p >= t)
+    return keep
+
+
+def gene_tables(groups, X_kept: np.ndarray):
+    """P:308-310 / Fig. 7: per group, the distinct value tuples of its fields over the
+    sampled space, in ascending order (index = re-indexed gene value)."""
+    return [sorted(set(tuple(int(v) for v in row) for row in X_kept[:, g])) for g in groups]
 
 
 def passes(pred_row, directions, th) -> bool:

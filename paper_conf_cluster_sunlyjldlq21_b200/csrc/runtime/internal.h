@@ -65,6 +65,12 @@ class Space {
   uint64_t count() const { return total_; }
   bool at(uint64_t rank, Tuple* out) const;
   bool rank(const Tuple& t, uint64_t* out) const;
+  // Stream the valid settings of prefixes [p0, p1) in rank order: f(rank, tuple).  The
+  // prefixes (first 8 fields) partition the space, so threads can split them.
+  size_t n_prefixes() const { return prefixes_.size(); }
+  uint64_t prefix_start(size_t i) const { return prefixes_[i].start; }
+  template <class F>
+  void for_each(size_t p0, size_t p1, F&& f) const;
 
  private:
   struct Core {  // (CM x3, BM x3, ret, pf, bt, qs) and its per-dim UF bounds (counts)
@@ -78,10 +84,42 @@ class Space {
   };
   void cores_for(const int32_t* prefix, std::vector<Core>* cores) const;
   StencilInfo st_;
+  uint64_t id_;                 // unique per Space (keys at()'s per-thread core cache)
   std::vector<Prefix> prefixes_;
   uint64_t total_ = 0;
   std::vector<int32_t> p2_[3];  // powers of two <= M_d
 };
+
+template <class F>
+void Space::for_each(size_t p0, size_t p1, F&& f) const {
+  std::vector<Core> cores;
+  for (size_t pi = p0; pi < p1 && pi < prefixes_.size(); ++pi) {
+    const Prefix& P = prefixes_[pi];
+    cores_for(P.v, &cores);
+    Tuple t{};
+    for (int i = 0; i < 8; ++i) t[i] = P.v[i];
+    uint64_t rk = P.start;
+    // canonical order within a prefix: UF_x, UF_y, UF_z, then the cores (see Space::at)
+    for (int32_t u0 = 0; u0 < (int32_t)p2_[0].size(); ++u0)
+      for (int32_t u1 = 0; u1 < (int32_t)p2_[1].size(); ++u1)
+        for (int32_t u2 = 0; u2 < (int32_t)p2_[2].size(); ++u2)
+          for (const Core& c : cores) {
+            if (u0 >= c.nuf[0] || u1 >= c.nuf[1] || u2 >= c.nuf[2]) continue;
+            t[F_UFX] = p2_[0][u0];
+            t[F_UFY] = p2_[1][u1];
+            t[F_UFZ] = p2_[2][u2];
+            for (int d = 0; d < 3; ++d) {
+              t[F_CMX + d] = c.cm[d];
+              t[F_BMX + d] = c.bm[d];
+            }
+            t[F_RET] = c.ret;
+            t[F_PF] = c.pf;
+            t[F_BT] = c.bt;
+            t[F_QS] = c.qs;
+            f(rk++, t);
+          }
+  }
+}
 
 // Copy the logical halo of one array (fill.cu).  Multi-step sweeps use in[]'s halo as the
 // boundary condition of every step.

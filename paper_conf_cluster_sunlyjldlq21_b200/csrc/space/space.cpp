@@ -8,6 +8,7 @@
 // Canonical order: lexicographic over the 21 fields (Table I row order, bt, qstore), values
 // ascending.  count / rank / unrank are exact (bit-exact with oracle/space.py).
 #include <algorithm>
+#include <atomic>
 #include <cstring>
 
 #include "../runtime/internal.h"
@@ -417,7 +418,9 @@ void Space::cores_for(const int32_t* pre, std::vector<Core>* cores) const {
   });
 }
 
-Space::Space(const StencilInfo& st) : st_(st) {
+static std::atomic<uint64_t> g_space_ids{0};
+
+Space::Space(const StencilInfo& st) : st_(st), id_(++g_space_ids) {
   for (int d = 0; d < 3; ++d) p2_[d] = p2_upto(st.M[d]);
   const std::vector<int32_t> tbxy = p2_upto(1024), tbz = p2_upto(64);
   std::vector<Core> cores;
@@ -468,8 +471,16 @@ bool Space::at(uint64_t rank, Tuple* out) const {
   }
   const Prefix& P = prefixes_[lo];
   uint64_t q = rank - P.start;
-  std::vector<Core> cores;
-  cores_for(P.v, &cores);
+  // the cores of the last prefix unranked on this thread are reused (sorted rank batches,
+  // e.g. the tuner's quantile sample, mostly stay within one prefix)
+  thread_local uint64_t c_space = 0;
+  thread_local size_t c_prefix = (size_t)-1;
+  thread_local std::vector<Core> cores;
+  if (c_space != id_ || c_prefix != lo) {
+    cores_for(P.v, &cores);
+    c_space = id_;
+    c_prefix = lo;
+  }
   Tuple t{};
   for (int i = 0; i < 8; ++i) t[i] = P.v[i];
   // UF_x, UF_y, UF_z in turn: candidate value index u_d (0-based) allowed iff u_d < nuf[d]

@@ -22,6 +22,7 @@
 #include <set>
 #include <sstream>
 #include <thread>
+#include <unordered_set>
 
 #include "../runtime/internal.h"
 
@@ -394,6 +395,8 @@ extern "C" void cst_tune_opts_default(cst_tune_opts* o) {
   o->warm_start = 1;
   o->metrics_mode = 0;
   o->nsteps = 1;
+  o->noise_reps = 8;
+  o->filter_threads = 0;
 }
 
 namespace {
@@ -437,6 +440,36 @@ struct Evaluator {
   Tuple effective(Tuple t) const {
     if (o->nsteps <= 1 && check_rules(h->info, t) == nullptr) t[F_BT] = 1;
     return t;
+  }
+
+  // timing noise (Q18): n independent re-evaluations of one setting, bypassing
+  // the memo; returns their fitness values
+  cst_status repeat(const Tuple& t0, int n, std::vector<double>* fit) {
+    fit->clear();
+    const Tuple t = effective(t0);
+    if (n <= 0 || check_rules(h->info, t) != nullptr) return CST_OK;
+    std::vector<cst_setting> ss(n, from_tuple(t));
+    std::vector<double> ms(n, INFINITY);
+    const auto t0c = std::chrono::steady_clock::now();
+    if (cb) {
+      std::vector<double> met;
+      if (o->n_user_metrics > 0) met.assign((size_t)n * o->n_user_metrics, 0.0);
+      if (cb(user, ss.data(), n, ms.data(), o->n_user_metrics > 0 ? met.data() : nullptr) != 0)
+        return fail(CST_E_INTERNAL, "tuner: evaluation callback failed");
+    } else {
+      if (o->nsteps > 1) return CST_OK;  // multi-step timing copies its input: skip
+      for (int i = 0; i < n; ++i) {
+        double m = INFINITY;
+        const cst_status st = cst_time_setting(h, &ss[i], in, out, 1, o->warmup,
+                                               std::max(1, o->reps), stream, &m);
+        if (st == CST_E_CUDA) return st;
+        ms[i] = st == CST_OK ? m : INFINITY;
+      }
+    }
+    eval_s += std::chrono::duration<double>(std::chrono::steady_clock::now() - t0c).count();
+    for (double m : ms)
+      if (m > 0 && std::isfinite(m)) fit->push_back(1.0 / m);
+    return CST_OK;
   }
 
   // evaluate (memoised) a batch; invalid settings (rules) get ms = inf without timing
@@ -710,9 +743,13 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
     allfits.push_back(fits);
   }
 
-  // ---- 5. threshold filter over a quantile sample of the space (Q13)
+  // ---- 5. threshold filter -> sampled space (reading Q13)
+  // 5a. thresholds: one common order-statistic index t over a seeded quantile sample of
+  // the valid space (the whole space if it is small), the smallest t for which at least
+  // the sampling ratio of the sample passes every selected metric's threshold
   const uint64_t nq = std::min<uint64_t>(count, (uint64_t)std::max(16, o->quantile_sample));
-  const std::vector<uint64_t> qranks = sample_ranks(o->seed ^ 0x51A7E5ULL, count, nq);
+  std::vector<uint64_t> qranks = sample_ranks(o->seed ^ 0x51A7E5ULL, count, nq);
+  std::sort(qranks.begin(), qranks.end());  // order is irrelevant to t; sorted = fast unrank
   std::vector<Tuple> qset(qranks.size());
   for (size_t i = 0; i < qranks.size(); ++i) S.at(qranks[i], &qset[i]);
   const size_t K = selected.size();
@@ -742,21 +779,111 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
     else lo = mid + 1;
   }
   const int64_t tstar = lo;
-  std::vector<Tuple> kept;
-  for (int64_t i = 0; i < nqs; ++i)
-    if (passes((size_t)i, tstar)) kept.push_back(qset[i]);
-  const uint64_t sampled_count =
-      (uint64_t)std::llround((double)kept.size() / (double)nqs * (double)count);
+  std::vector<double> thv(K);
+  for (size_t k = 0; k < K; ++k) thv[k] = thr_at(tstar, k);
 
-  // ---- 6. re-index each group's valid value tuples (Fig. 7)
-  std::vector<std::vector<std::vector<int32_t>>> tables;
-  for (const auto& g : groups) {
-    std::set<std::vector<int32_t>> vals;
-    for (const Tuple& t : kept) {
-      std::vector<int32_t> v;
-      for (int f : g) v.push_back(t[f]);
-      vals.insert(v);
+  // 5b. "filter out inappropriate parameter settings during the sampling process"
+  // (P:290-292): stream the WHOLE valid space through the surrogate and the thresholds,
+  // count the survivors exactly and keep, per group, the distinct value tuples they
+  // project to (all the GA needs).  Multi-threaded over contiguous rank ranges.
+  // The predictions use per-field tables of P^i and log2(P)^j with the same values and
+  // multiplication order as pmnf_predict, so they are bit-identical to it.
+  const auto filt0 = std::chrono::steady_clock::now();
+  int32_t vmax = 1024;
+  for (int d = 0; d < 3; ++d) vmax = std::max<int32_t>(vmax, (int32_t)h->info.M[d]);
+  std::vector<std::vector<std::vector<double>>> fa(K), fb(K);  // [k][field][value]
+  for (size_t k = 0; k < K; ++k) {
+    fa[k].assign(F_COUNT, std::vector<double>(vmax + 1, 0.0));
+    fb[k].assign(F_COUNT, std::vector<double>(vmax + 1, 0.0));
+    for (int f = 0; f < F_COUNT; ++f)
+      for (int32_t v = 1; v <= vmax; ++v) {
+        fa[k][f][v] = std::pow((double)v, chosen[k].i);
+        fb[k][f][v] = std::pow(std::log2((double)v), chosen[k].j);
+      }
+  }
+  auto pass_full = [&](const Tuple& t) {
+    for (size_t k = 0; k < K; ++k) {
+      double sum = 0;
+      for (size_t c = 0; c < groups.size(); ++c) {
+        double col = 1.0;
+        for (int l : groups[c]) col = col * fa[k][l][t[l]] * fb[k][l][t[l]];
+        sum += col * chosen[k].coef[c];
+      }
+      if (dirs[k] > 0 ? !(sum <= thv[k]) : !(sum >= thv[k])) return false;
     }
+    return true;
+  };
+  typedef unsigned __int128 u128;
+  struct H128 {
+    size_t operator()(u128 x) const {
+      return (size_t)(sm64((uint64_t)x) ^ (sm64((uint64_t)(x >> 64)) * 31));
+    }
+  };
+  auto code_of = [](int f, int32_t v) -> u128 {
+    if (!pow2_field(f)) return (u128)v;
+    int c = 0;
+    while ((1 << c) < v) ++c;
+    return (u128)c;
+  };
+  auto decode_of = [](int f, u128 c) -> int32_t {
+    return pow2_field(f) ? (int32_t)(1 << (int)c) : (int32_t)c;
+  };
+  const size_t G = groups.size();
+  unsigned nth = o->filter_threads > 0 ? (unsigned)o->filter_threads
+                                       : std::max(1u, std::thread::hardware_concurrency());
+  nth = std::min<unsigned>(nth, (unsigned)std::max<size_t>(1, S.n_prefixes()));
+  // contiguous prefix ranges with about count / nth settings each (rank order kept)
+  std::vector<size_t> bnd(nth + 1, S.n_prefixes());
+  bnd[0] = 0;
+  for (unsigned w = 1; w < nth; ++w) {
+    const uint64_t target = count / nth * w;
+    size_t lo2 = 0, hi2 = S.n_prefixes();
+    while (lo2 < hi2) {
+      const size_t mid = (lo2 + hi2) / 2;
+      if (S.prefix_start(mid) < target) lo2 = mid + 1;
+      else hi2 = mid;
+    }
+    bnd[w] = std::max(bnd[w - 1], lo2);
+  }
+  const uint64_t kLogKept = 200000;
+  std::vector<uint64_t> kept_n(nth, 0);
+  std::vector<std::vector<uint64_t>> kept_rk(nth);
+  std::vector<std::vector<std::unordered_set<u128, H128>>> proj(
+      nth, std::vector<std::unordered_set<u128, H128>>(G));
+  {
+    std::vector<std::thread> pool;
+    for (unsigned w = 0; w < nth; ++w)
+      pool.emplace_back([&, w] {
+        S.for_each(bnd[w], bnd[w + 1], [&](uint64_t rk, const Tuple& t) {
+          if (!pass_full(t)) return;
+          ++kept_n[w];
+          if (kept_rk[w].size() <= kLogKept) kept_rk[w].push_back(rk);
+          for (size_t g = 0; g < G; ++g) {
+            u128 key = 0;
+            for (size_t q = 0; q < groups[g].size(); ++q)
+              key |= code_of(groups[g][q], t[groups[g][q]]) << (5 * q);
+            proj[w][g].insert(key);
+          }
+        });
+      });
+    for (auto& th : pool) th.join();
+  }
+  uint64_t sampled_count = 0;
+  for (unsigned w = 0; w < nth; ++w) sampled_count += kept_n[w];
+  const double filter_s =
+      std::chrono::duration<double>(std::chrono::steady_clock::now() - filt0).count();
+
+  // ---- 6. re-index each group's valid value tuples (Fig. 7): ascending order
+  std::vector<std::vector<std::vector<int32_t>>> tables;
+  for (size_t g = 0; g < G; ++g) {
+    std::set<std::vector<int32_t>> vals;
+    for (unsigned w = 0; w < nth; ++w)
+      for (u128 key : proj[w][g]) {
+        std::vector<int32_t> v;
+        for (size_t q = 0; q < groups[g].size(); ++q)
+          v.push_back(decode_of(groups[g][q], (key >> (5 * q)) & 31));
+        vals.insert(v);
+      }
     tables.push_back(std::vector<std::vector<int32_t>>(vals.begin(), vals.end()));
   }
   const double preproc_s = std::chrono::duration<double>(std::chrono::steady_clock::now() - pre0).count();
@@ -799,21 +926,53 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
   js.o << tstar;
   js.key("quantile_sample");
   js.o << nqs;
-  js.key("kept_ranks");
+  js.key("thresholds");
   js.o << "[";
-  {
+  for (size_t k = 0; k < K; ++k) js.o << (k ? "," : "") << Json::num(thv[k]);
+  js.o << "]";
+  js.key("sampled_count");
+  js.o << sampled_count;
+  js.key("filter_s");
+  js.o << Json::num(filter_s);
+  js.key("filter_threads");
+  js.o << nth;
+  js.key("kept_ranks");
+  if (sampled_count <= kLogKept) {
+    js.o << "[";
     bool first = true;
-    for (int64_t i = 0; i < nqs; ++i)
-      if (passes((size_t)i, tstar)) {
-        js.o << (first ? "" : ",") << qranks[i];
+    for (unsigned w = 0; w < nth; ++w)
+      for (uint64_t rk : kept_rk[w]) {
+        js.o << (first ? "" : ",") << rk;
         first = false;
       }
+    js.o << "]";
+  } else {
+    js.o << "null";
   }
-  js.o << "]";
   js.key("table_sizes");
   js.o << "[";
-  for (size_t g = 0; g < tables.size(); ++g) js.o << (g ? "," : "") << tables[g].size();
+  size_t table_entries = 0;
+  for (size_t g = 0; g < tables.size(); ++g) {
+    js.o << (g ? "," : "") << tables[g].size();
+    table_entries += tables[g].size();
+  }
   js.o << "]";
+  js.key("tables");  // the re-indexed gene tables themselves, when small enough to log
+  if (table_entries <= 20000) {
+    js.o << "[";
+    for (size_t g = 0; g < tables.size(); ++g) {
+      js.o << (g ? "," : "") << "[";
+      for (size_t e = 0; e < tables[g].size(); ++e) {
+        js.o << (e ? "," : "") << "[";
+        for (size_t q = 0; q < tables[g][e].size(); ++q) js.o << (q ? "," : "") << tables[g][e][q];
+        js.o << "]";
+      }
+      js.o << "]";
+    }
+    js.o << "]";
+  } else {
+    js.o << "null";
+  }
 
   // ---- 7. group-wise GA with approximation
   int bi = valid[0];
@@ -821,9 +980,24 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
     if (fitness_of(res[i]) > fitness_of(res[bi])) bi = i;
   Tuple cur = rows[bi];
   double cur_ms = res[bi].ms;
+  // approximation threshold (reading Q18): the CV of the top-n fitness is compared with
+  // max(cv_threshold, 2 * timing-noise CV), the noise measured by re-evaluating the
+  // dataset's best setting noise_reps times — top-n settings whose fitness spread is
+  // within the measurement noise are "similar performance"
+  double noise_cv = 0.0;
+  {
+    std::vector<double> nf;
+    st = ev.repeat(cur, o->noise_reps, &nf);
+    if (st != CST_OK) return st;
+    if (nf.size() >= 2) noise_cv = cv(nf);
+  }
+  const double tau = std::max(o->cv_threshold, 2.0 * noise_cv);
+  js.key("noise");
+  js.o << "{\"reps\":" << o->noise_reps << ",\"cv\":" << Json::num(noise_cv)
+       << ",\"tau\":" << Json::num(tau) << "}";
   Rng rng(o->seed);
   const int pop = o->n_subpops * o->subpop_size;
-  int total_gens = 0;
+  int total_gens = 0, phases_cv_stop = 0;
   js.key("phases");
   js.o << "[";
   for (size_t g = 0; g < groups.size(); ++g) {
@@ -837,7 +1011,11 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
       return t;
     };
     std::map<Tuple, double> phase;  // distinct settings evaluated in this phase -> fitness
+    const Tuple start = cur;
+    const double start_ms = cur_ms;
     int gens = 0;
+    const char* stop = "exhaustive";
+    std::vector<double> cv_trace;
     bool exhaustive = (int)tab.size() <= pop;
     if (exhaustive) {
       // P:343 / P:405: fewer settings than the population -> exhaustive search
@@ -950,18 +1128,32 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
               }
             }
         }
-        // approximation stop: CV of the top-n fitness of this phase
+        // approximation stop: CV of the top-n fitness of the population's
+        // individuals (an individual "is evaluated by the fitness")
         std::vector<double> fs;
-        for (auto& kv : phase)
-          if (kv.second > 0) fs.push_back(kv.second);
+        for (int i = 0; i < pop; ++i)
+          if (fit[i] > 0) fs.push_back(fit[i]);
         std::sort(fs.rbegin(), fs.rend());
+        double cvn = -1.0;
         if ((int)fs.size() >= o->top_n) {
           fs.resize(o->top_n);
-          if (cv(fs) < o->cv_threshold) break;
+          cvn = cv(fs);
         }
-        if (o->time_budget_s > 0 && elapsed() - t_dataset > o->time_budget_s) break;
+        cv_trace.push_back(cvn);
+        if (cvn >= 0 && cvn < tau) {
+          stop = "cv_top_n";
+          ++phases_cv_stop;
+          break;
+        }
+        if (o->time_budget_s > 0 && elapsed() - t_dataset > o->time_budget_s) {
+          stop = "time_budget";
+          break;
+        }
       }
-      if (gens > o->max_generations) gens = o->max_generations;
+      if (gens > o->max_generations) {
+        gens = o->max_generations;
+        stop = "max_generations";
+      }
     }
     total_gens += gens;
     // adopt the best setting of the phase
@@ -972,7 +1164,15 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
       }
     js.o << (g ? "," : "") << "{\"group\":" << g << ",\"table\":" << tab.size()
          << ",\"exhaustive\":" << (exhaustive ? "true" : "false") << ",\"generations\":" << gens
-         << ",\"evaluated\":" << phase.size() << ",\"best_ms\":" << Json::num(cur_ms) << "}";
+         << ",\"evaluated\":" << phase.size() << ",\"stop\":\"" << stop << "\""
+         << ",\"start_ms\":" << Json::num(start_ms) << ",\"best_ms\":" << Json::num(cur_ms)
+         << ",\"start\":[";
+    for (int f = 0; f < F_COUNT; ++f) js.o << (f ? "," : "") << start[f];
+    js.o << "],\"best\":[";
+    for (int f = 0; f < F_COUNT; ++f) js.o << (f ? "," : "") << cur[f];
+    js.o << "],\"cv_top_n\":[";
+    for (size_t q = 0; q < cv_trace.size(); ++q) js.o << (q ? "," : "") << Json::num(cv_trace[q]);
+    js.o << "]}";
     if (o->time_budget_s > 0 && elapsed() - t_dataset > o->time_budget_s) break;
   }
   js.o << "]";
@@ -991,6 +1191,9 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
   rep->preproc_s = preproc_s;
   rep->n_groups = (int32_t)groups.size();
   rep->generations = total_gens;
+  rep->phases_cv_stop = phases_cv_stop;
+  rep->noise_cv = noise_cv;
+  rep->cv_threshold_used = tau;
   js.key("best");
   js.o << "{\"setting\": [";
   for (int f = 0; f < F_COUNT; ++f) js.o << (f ? "," : "") << cur[f];
@@ -1006,7 +1209,9 @@ extern "C" cst_status cst_tune(cst_stencil* h, const cst_tune_opts* o, const dou
        << ",\"jit_s\":" << Json::num(rep->jit_s) << ",\"preproc_s\":" << Json::num(preproc_s)
        << ",\"dataset_s\":" << Json::num(t_dataset) << ",\"evaluations\":" << rep->evaluations
        << ",\"jit_compiles\":" << rep->jit_compiles << ",\"space_count\":" << count
-       << ",\"sampled_count\":" << sampled_count << ",\"generations\":" << total_gens << "}";
+       << ",\"sampled_count\":" << sampled_count << ",\"generations\":" << total_gens
+       << ",\"phases_cv_stop\":" << phases_cv_stop << ",\"filter_s\":" << Json::num(filter_s)
+       << "}";
   js.o << "\n}\n";
   if (o->log_path && *o->log_path) {
     std::ofstream f(o->log_path);

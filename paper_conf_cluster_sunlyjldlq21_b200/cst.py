@@ -118,7 +118,8 @@ class cst_tune_opts(ctypes.Structure):
                 ("reps", ctypes.c_int32), ("warmup", ctypes.c_int32), ("log_path", ctypes.c_char_p),
                 ("n_user_metrics", ctypes.c_int32), ("quantile_sample", ctypes.c_int32),
                 ("warm_start", ctypes.c_int32), ("metrics_mode", ctypes.c_int32),
-                ("nsteps", ctypes.c_int32)]
+                ("nsteps", ctypes.c_int32), ("noise_reps", ctypes.c_int32),
+                ("filter_threads", ctypes.c_int32)]
 
 
 class cst_tune_report(ctypes.Structure):
@@ -127,7 +128,8 @@ class cst_tune_report(ctypes.Structure):
                 ("evaluations", ctypes.c_uint64), ("jit_compiles", ctypes.c_uint64),
                 ("wall_s", ctypes.c_double), ("eval_s", ctypes.c_double), ("jit_s", ctypes.c_double),
                 ("preproc_s", ctypes.c_double), ("n_groups", ctypes.c_int32),
-                ("generations", ctypes.c_int32)]
+                ("generations", ctypes.c_int32), ("phases_cv_stop", ctypes.c_int32),
+                ("noise_cv", ctypes.c_double), ("cv_threshold_used", ctypes.c_double)]
 
 
 class cst_halo_xfer(ctypes.Structure):
