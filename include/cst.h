@@ -313,6 +313,42 @@ cst_status cst_dist_sweep_loopback(cst_stencil* h, int32_t nslabs, const cst_set
                                    int32_t nsteps, void* stream);
 void cst_dist_destroy(cst_dist* d);
 
+/* ---------------------------------------------------- population-parallel tuning */
+/* cst_tune with each GA population (and the dataset) evaluated across the ranks of a
+ * cst_dist (the paper's multi-process GA): rank 0 runs the tuner
+ * (every stage of cst_tune, same options, same result for the same fitness values); every
+ * batch of candidates it asks for is broadcast, rank k evaluates candidates i with
+ * i % nranks == k on its own GPU, and the fitness (and metric) vectors are all-gathered.
+ * The GA's trajectory therefore does not depend on nranks.  COLLECTIVE: every rank of `d`
+ * calls it with the same opts.
+ *   in / scratch_out: this rank's replica of the evaluation grid (device buffers of the
+ *     handle's grid), used by the built-in evaluator (NVRTC code generation of the share
+ *     on host threads, then CUDA-event timing, Q20) when local_eval == NULL;
+ *   local_eval: optional caller evaluation of this rank's share (same contract as
+ *     cst_tune's eval callback; synthetic objectives in the tests);
+ *   best / rep: written on every rank (rank 0's result is broadcast); rep->evaluations
+ *     etc. are rank 0's.
+ * Transport: the handle's NCCL communicator (small device staging buffers on its
+ * communication stream), or the host collectives given to cst_dist_create_host.  Errors:
+ * if rank 0's tuner fails, every rank returns that status (the result message is always
+ * broadcast, so no rank blocks); a rank whose evaluation fails reports its candidates as
+ * invalid (fitness 0) and keeps serving. */
+typedef struct {
+  void* user;
+  /* broadcast `bytes` of host memory at buf from rank `root` (in place); 0 = success */
+  int (*bcast)(void* user, void* buf, int64_t bytes, int32_t root);
+  /* all-gather `bytes` from every rank: recv[k * bytes ...] = rank k's send; 0 = success */
+  int (*allgather)(void* user, const void* send, void* recv, int64_t bytes);
+} cst_collectives;
+/* A tuning-only handle (no device resources; cst_dist_sweep on it is CST_E_INVALID) whose
+ * collectives are the caller's (e.g. torch.distributed over gloo or NCCL).  `coll` is
+ * copied; its user pointer must stay valid for the handle's lifetime. */
+cst_status cst_dist_create_host(cst_stencil* h, int32_t nranks, int32_t rank,
+                                const cst_collectives* coll, cst_dist** out);
+cst_status cst_dist_tune(cst_dist* d, const cst_tune_opts* o, const double* const* in,
+                         double* const* scratch_out, cst_eval_fn local_eval, void* local_user,
+                         cst_setting* best, cst_tune_report* rep);
+
 /* Fused halo exchange over peer memory (no NCCL).  A handle created
  * with nccl_unique_id == NULL and nranks > 1 uses it: the boundary kernels of
  * cst_dist_sweep store every edge-plane value both locally and, through a CUDA IPC

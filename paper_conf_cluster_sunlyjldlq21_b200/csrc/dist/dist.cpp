@@ -11,11 +11,7 @@
 // result is bit-identical to the single-GPU sweep with the same setting.
 #include <cstring>
 
-#include "../runtime/internal.h"
-
-#ifdef CST_HAVE_NCCL
-#include <nccl.h>
-#endif
+#include "dist_internal.h"
 
 // Fused halo exchange over peer memory: no NCCL.  The boundary
 // launches store every edge-plane value both locally and, through a CUDA IPC mapping of
@@ -29,32 +25,6 @@
 // Per step (epoch e, one stream):  wait DONE >= e-1 | boundary launches with remote stores
 // | signal BND = e | interior | signal DONE = e | wait BND >= e.  Waits spin on an acquire
 // load with a 30 s bound (then trap: a dead peer is an error, not a hang).
-enum { F_BND_LO = 0, F_BND_HI = 1, F_DONE_LO = 2, F_DONE_HI = 3, F_WORDS = 16 };
-
-struct P2PPeer {
-  bool open = false;
-  double* buf[2][CST_MAX_IN] = {};  // the peer's ping-pong buffers (a, b), mapped here
-  unsigned long long* flags = nullptr;  // the peer's flag words, mapped here
-  std::vector<void*> bases;             // IPC mappings to close
-};
-
-struct cst_dist {
-  cst_stencil* h = nullptr;
-  int32_t nranks = 1, rank = 0;
-  cudaStream_t s_comm = nullptr;
-  cudaEvent_t ev_bnd = nullptr, ev_comm = nullptr;
-#ifdef CST_HAVE_NCCL
-  ncclComm_t comm = nullptr;
-#endif
-  // peer-memory transport
-  bool p2p = false;
-  unsigned long long* flags = nullptr;  // my flag words (F_WORDS x u64)
-  const double* mine[2][CST_MAX_IN] = {};  // my registered ping-pong buffers (a, b)
-  bool exported = false;
-  P2PPeer lo, hi;                        // rank - 1, rank + 1
-  unsigned long long epoch = 0;
-};
-
 using namespace cst;
 
 extern "C" cst_status cst_dist_halo_plan(int32_t nranks, int32_t rank, int64_t nz, int32_t r,
@@ -174,13 +144,17 @@ namespace {
 struct P2PBlob {
   uint64_t magic;
   int32_t nio, rank, nranks, device;
+  // geometry: the remote store offsets are computed from the LOCAL grid, so the peer's
+  // must be identical (a mismatch would put peer stores at wrong offsets)
+  int64_t nx, ny, nz, pitch_x, pitch_y;
+  int32_t halo, lead_x, order, kind;
   cudaIpcMemHandle_t buf[2][CST_MAX_IN];
   int64_t off[2][CST_MAX_IN];
   cudaIpcMemHandle_t flags;
   int64_t flags_off;
 };
 static_assert(sizeof(P2PBlob) <= CST_P2P_BLOB_BYTES, "blob size");
-const uint64_t kBlobMagic = 0x43535450325031ULL;  // "CSTP2P1"
+const uint64_t kBlobMagic = 0x43535450325032ULL;  // "CSTP2P2"
 
 cst_status ipc_handle(const void* p, cudaIpcMemHandle_t* hd, int64_t* off) {
   const Driver* d = nullptr;
@@ -209,6 +183,16 @@ extern "C" cst_status cst_dist_p2p_export(cst_dist* D, double* const* buf_a,
   b.rank = D->rank;
   b.nranks = D->nranks;
   b.device = D->h->device;
+  const cst_grid& G = D->h->grid;
+  b.nx = G.nx;
+  b.ny = G.ny;
+  b.nz = G.nz;
+  b.pitch_x = G.pitch_x;
+  b.pitch_y = G.pitch_y;
+  b.halo = G.halo;
+  b.lead_x = G.lead_x;
+  b.order = D->h->desc.order;
+  b.kind = D->h->desc.kind;
   for (int a = 0; a < nio; ++a) {
     if (!buf_a[a] || !buf_b[a]) return fail(CST_E_INVALID, "null buffer");
     cst_status st = ipc_handle(buf_a[a], &b.buf[0][a], &b.off[0][a]);
@@ -236,6 +220,14 @@ extern "C" cst_status cst_dist_p2p_import(cst_dist* D, int32_t peer, const void*
   if (b.magic != kBlobMagic || b.nio != D->h->desc.n_inputs || b.rank != peer ||
       b.nranks != D->nranks)
     return fail(CST_E_INVALID, "p2p blob does not belong to this decomposition / peer");
+  {
+    const cst_grid& G = D->h->grid;
+    if (b.nx != G.nx || b.ny != G.ny || b.nz != G.nz || b.pitch_x != G.pitch_x ||
+        b.pitch_y != G.pitch_y || b.halo != G.halo || b.lead_x != G.lead_x ||
+        b.order != D->h->desc.order || b.kind != D->h->desc.kind)
+      return fail(CST_E_INVALID, "p2p blob: the peer's grid geometry / stencil differs from "
+                                 "mine (nx, ny, nz, pitches, halo, lead_x, order, kind must match)");
+  }
   CST_CUDA(cudaSetDevice(D->h->device));
   P2PPeer& P = peer < D->rank ? D->lo : D->hi;
   for (void* base : P.bases) cudaIpcCloseMemHandle(base);
@@ -283,6 +275,15 @@ static cst_status dist_sweep_p2p(cst_dist* D, const cst_setting* s, const double
   }
   if (role < 0)
     return fail(CST_E_INVALID, "p2p transport: in/out must be the exported buffer sets (a, b)");
+  if (D->broken)
+    return fail(CST_E_INTERNAL, "p2p transport: an earlier step failed mid-protocol; the "
+                                "ranks cannot resynchronise (destroy and recreate the handle)");
+  // every variant this protocol launches is resolved before any epoch is published: a
+  // compile / R13 / load failure must not leave the neighbours waiting for this rank
+  {
+    cst_status st = cst_resolve_variant(h, s, has_lo || has_hi);
+    if (st != CST_OK) return st;
+  }
   const int64_t pz = G.pitch_x * G.pitch_y;
   const int64_t origin0 = ((int64_t)G.halo * G.pitch_y + G.halo) * G.pitch_x + G.lead_x;
   const double* cin[CST_MAX_IN];
@@ -299,7 +300,7 @@ static cst_status dist_sweep_p2p(cst_dist* D, const cst_setting* s, const double
     // WAR: both neighbours finished step e-1 (they read the buffers my stores target)
     cst_status st = p2p_wait(sc, has_lo ? D->flags + F_DONE_LO : nullptr, e - 1,
                              has_hi ? D->flags + F_DONE_HI : nullptr, e - 1);
-    if (st != CST_OK) return st;
+    if (st != CST_OK) return D->broken = true, st;
     ++extra;
     // boundary planes: local stores + the same values into the neighbours' halos
     double* rlo[CST_MAX_OUT];
@@ -309,27 +310,27 @@ static cst_status dist_sweep_p2p(cst_dist* D, const cst_setting* s, const double
       rhi[a] = has_hi ? D->hi.buf[orole][a] + origin0 - (int64_t)r * pz : nullptr;
     }
     st = cst_launch_range(h, s, cin, cout, 0, r, sc, has_lo ? rlo : nullptr);
-    if (st != CST_OK) return st;
+    if (st != CST_OK) return D->broken = true, st;
     if (G.nz > r) {
       st = cst_launch_range(h, s, cin, cout, G.nz - r, r, sc, has_hi ? rhi : nullptr);
-      if (st != CST_OK) return st;
+      if (st != CST_OK) return D->broken = true, st;
     }
     // my boundary stores are in the neighbours' halos: lower neighbour's BND_HI, upper's BND_LO
     st = p2p_signal(sc, has_lo ? D->lo.flags + F_BND_HI : nullptr,
                     has_hi ? D->hi.flags + F_BND_LO : nullptr, e);
-    if (st != CST_OK) return st;
+    if (st != CST_OK) return D->broken = true, st;
     ++extra;
     if (G.nz > 2 * r) {
       st = cst_launch_range(h, s, cin, cout, r, G.nz - 2 * r, sc);
-      if (st != CST_OK) return st;
+      if (st != CST_OK) return D->broken = true, st;
     }
     st = p2p_signal(sc, has_lo ? D->lo.flags + F_DONE_HI : nullptr,
                     has_hi ? D->hi.flags + F_DONE_LO : nullptr, e);
-    if (st != CST_OK) return st;
+    if (st != CST_OK) return D->broken = true, st;
     // RAW: the neighbours' boundary stores of this step are in my output halo
     st = p2p_wait(sc, has_lo ? D->flags + F_BND_LO : nullptr, e,
                   has_hi ? D->flags + F_BND_HI : nullptr, e);
-    if (st != CST_OK) return st;
+    if (st != CST_OK) return D->broken = true, st;
     extra += 2;
     if (nsteps > 1) {
       for (int a = 0; a < nio; ++a) {
@@ -348,6 +349,7 @@ extern "C" cst_status cst_dist_sweep(cst_dist* D, const cst_setting* s, const do
                                      double* const* out, int32_t nsteps, void* stream) {
   if (!D || !s || !in || !out) return fail(CST_E_INVALID, "null argument");
   if (nsteps < 1) return fail(CST_E_INVALID, "nsteps < 1");
+  if (D->host_only) return fail(CST_E_INVALID, "a cst_dist_create_host handle only tunes");
   cst_stencil* h = D->h;
   const cst_grid& G = h->grid;
   const int r = h->desc.order;
@@ -368,9 +370,9 @@ extern "C" cst_status cst_dist_sweep(cst_dist* D, const cst_setting* s, const do
   if (s->bt > 1)
     return fail(CST_E_UNSUPPORTED, "temporal blocking (bt > 1) needs bt*order halo planes; "
                                    "cst_dist_sweep exchanges order planes per step");
-  if (nsteps > 1)  // boundary condition of every step = in[]'s halo (as cst_sweep); the
-                   // z-halo planes facing a neighbour are the exchange's (never copied: with
-                   // the peer transport the neighbour may already be storing into them)
+  if (nsteps > 1)  // boundary condition of every step = in[]'s halo (as cst_sweep); of
+                   // the z-halo planes facing a neighbour only the x/y ring is copied — their
+                   // interior x/y is the exchange's (the peer may already be storing into it)
     for (int a = 0; a < nio; ++a) {
       st = copy_halo(G, in[a], out[a], sc, D->rank == 0, D->rank == D->nranks - 1);
       if (st != CST_OK) return st;

@@ -393,6 +393,13 @@ static cst_status get_variant(cst_stencil* h, const cst_setting* s, Variant** ou
   return CST_OK;
 }
 
+cst_status cst_resolve_variant(cst_stencil* h, const cst_setting* s, bool remote) {
+  Variant* v = nullptr;
+  cst_status st = get_variant(h, s, &v, false);
+  if (st == CST_OK && remote) st = get_variant(h, s, &v, true);
+  return st;
+}
+
 extern "C" cst_status cst_variant_compile(const cst_stencil* h, const cst_setting* s,
                                           double* compile_s) {
   if (!h || !s || !compile_s) return fail(CST_E_INVALID, "null argument");
@@ -601,10 +608,12 @@ extern "C" cst_status cst_sweep(cst_stencil* h, const cst_setting* s, const doub
   for (int a = 0; a < nin; ++a) cur_in[a] = in[a];
   for (int o = 0; o < nout; ++o) cur_out[o] = out[o];
   if (nsteps > 1) {
-    // boundary condition of every step = in[]'s halo (reading Q23)
-    cst_status st = copy_halo(h->grid, in[0], out[0], (cudaStream_t)stream);
-    if (st != CST_OK) return st;
-    ++h->last_launches;
+    // boundary condition of every step = in[]'s halo (reading Q23), every array
+    for (int a = 0; a < nin; ++a) {
+      cst_status st = copy_halo(h->grid, in[a], out[a], (cudaStream_t)stream);
+      if (st != CST_OK) return st;
+      ++h->last_launches;
+    }
   }
   // temporal blocking: passes of b <= bt fused steps (bt = 1: one launch per step)
   for (int b : pass_schedule(nsteps, s->bt)) {
@@ -612,11 +621,12 @@ extern "C" cst_status cst_sweep(cst_stencil* h, const cst_setting* s, const doub
     sp.bt = b;
     cst_status st = cst_launch_range(h, &sp, cur_in, cur_out, 0, h->grid.nz, (cudaStream_t)stream);
     if (st != CST_OK) return st;
-    if (nsteps > 1) {
-      const double* tmp = cur_in[0];
-      cur_in[0] = cur_out[0];
-      cur_out[0] = const_cast<double*>(tmp);
-    }
+    if (nsteps > 1)
+      for (int a = 0; a < nin; ++a) {  // ping-pong every array (nin == nout here)
+        const double* tmp = cur_in[a];
+        cur_in[a] = cur_out[a];
+        cur_out[a] = const_cast<double*>(tmp);
+      }
   }
   return CST_OK;
 }

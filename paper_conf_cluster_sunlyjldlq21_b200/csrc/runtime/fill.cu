@@ -26,7 +26,9 @@ __global__ void fill_kernel(double* __restrict__ dst, int64_t nx, int64_t ny, in
 }
 
 // one warp per (z, y) row of the logical padded region [-halo, n + halo)^3: halo rows are
-// copied whole, interior rows only their 2*halo x-halo elements
+// copied whole, interior rows only their 2*halo x-halo elements.  A z-halo plane that faces
+// a z-slab neighbour (zlo / zhi = 0) is treated like an interior plane: its x/y ring is
+// copied, its interior x/y is the exchange's (the neighbour's stores or NCCL receive)
 __global__ void copy_halo_kernel(const double* __restrict__ src, double* __restrict__ dst,
                                  int64_t nx, int64_t ny, int64_t nz, int64_t halo,
                                  int64_t lead_x, int64_t pitch_x, int64_t pitch_y, int zlo,
@@ -36,9 +38,9 @@ __global__ void copy_halo_kernel(const double* __restrict__ src, double* __restr
   const int64_t rows_y = ny + 2 * halo;
   if (row >= rows_y * (nz + 2 * halo)) return;
   const int64_t y = row % rows_y - halo, z = row / rows_y - halo;
-  if ((z < 0 && !zlo) || (z >= nz && !zhi)) return;
+  const bool facing = (z < 0 && !zlo) || (z >= nz && !zhi);
   const int64_t base = ((z + halo) * pitch_y + (y + halo)) * pitch_x + lead_x;
-  if (y < 0 || y >= ny || z < 0 || z >= nz) {
+  if (y < 0 || y >= ny || ((z < 0 || z >= nz) && !facing)) {
     for (int64_t x = lane - halo; x < nx + halo; x += 32) dst[base + x] = src[base + x];
   } else if (lane < 2 * halo) {
     const int64_t x = lane < halo ? lane - halo : nx + (lane - halo);
@@ -49,7 +51,9 @@ __global__ void copy_halo_kernel(const double* __restrict__ src, double* __restr
 }  // namespace
 
 namespace cst {
-// Copy the logical halo of one array (the multi-step boundary condition) from src to dst.
+// Copy the logical halo of one array (the multi-step boundary condition) from src to dst;
+// zlo / zhi = false: the z-halo planes on that side face a z-slab neighbour, only their x/y
+// ring is copied.
 cst_status copy_halo(const cst_grid& g, const double* src, double* dst, cudaStream_t stream,
                      bool zlo, bool zhi) {
   const int64_t rows = (g.nz + 2 * (int64_t)g.halo) * (g.ny + 2 * (int64_t)g.halo);

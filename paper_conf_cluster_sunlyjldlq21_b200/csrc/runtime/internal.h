@@ -123,8 +123,8 @@ void Space::for_each(size_t p0, size_t p1, F&& f) const {
 
 // Copy the logical halo of one array (fill.cu).  Multi-step sweeps use in[]'s halo as the
 // boundary condition of every step.
-// zlo / zhi: include the z-halo planes below / above (false where a z-slab neighbour owns
-// them).
+// zlo / zhi: include the z-halo planes below / above whole (false where a z-slab neighbour
+// fills their interior x/y: then only their x/y ring is copied).
 cst_status copy_halo(const cst_grid& g, const double* src, double* dst, cudaStream_t stream,
                      bool zlo = true, bool zhi = true);
 
@@ -185,6 +185,9 @@ std::string nvrtc_description();
 cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* const* in,
                             double* const* out, int64_t z0, int64_t nz, cudaStream_t stream,
                             double* const* rout = nullptr);
+// Resolve (compile, load, check R13) the variant of a setting — and its fused-halo twin if
+// `remote` — without launching anything (so multi-rank protocols fail before they start).
+cst_status cst_resolve_variant(cst_stencil* h, const cst_setting* s, bool remote);
 
 namespace cst {
 

@@ -141,6 +141,16 @@ EVAL_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.POINTER(cst_set
                            ctypes.c_int32, ctypes.POINTER(ctypes.c_double),
                            ctypes.POINTER(ctypes.c_double))
 
+BCAST_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64,
+                            ctypes.c_int32)
+ALLGATHER_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                ctypes.c_int64)
+
+
+class cst_collectives(ctypes.Structure):
+    _fields_ = [("user", ctypes.c_void_p), ("bcast", BCAST_FN), ("allgather", ALLGATHER_FN)]
+
+
 _P = ctypes.c_void_p
 _PP = ctypes.POINTER(ctypes.c_void_p)
 _S = ctypes.c_int  # cst_status
@@ -186,6 +196,10 @@ _decl("cst_tune", _S, _P, ctypes.POINTER(cst_tune_opts), _PP, _PP, EVAL_FN, _P,
 _decl("cst_dist_halo_plan", _S, ctypes.c_int32, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32,
       ctypes.POINTER(cst_halo_xfer), ctypes.POINTER(ctypes.c_int32))
 _decl("cst_dist_create", _S, _P, ctypes.c_int32, ctypes.c_int32, _P, ctypes.POINTER(_P))
+_decl("cst_dist_create_host", _S, _P, ctypes.c_int32, ctypes.c_int32,
+      ctypes.POINTER(cst_collectives), ctypes.POINTER(_P))
+_decl("cst_dist_tune", _S, _P, ctypes.POINTER(cst_tune_opts), _PP, _PP, EVAL_FN, _P,
+      ctypes.POINTER(cst_setting), ctypes.POINTER(cst_tune_report))
 _decl("cst_dist_nccl_unique_id", _S, _P)
 _decl("cst_dist_sweep", _S, _P, ctypes.POINTER(cst_setting), _PP, _PP, ctypes.c_int32, _P)
 _decl("cst_dist_sweep_loopback", _S, _P, ctypes.c_int32, ctypes.POINTER(cst_setting), _PP, _PP,
@@ -349,6 +363,70 @@ def cst_tune_opts_default() -> cst_tune_opts:
     o = cst_tune_opts()
     _lib.cst_tune_opts_default(ctypes.byref(o))
     return o
+
+
+def _eval_cb(eval_fn, nm):
+    if eval_fn is None:
+        return EVAL_FN()
+
+    def _cb(user, settings, n, ms, metrics):
+        try:
+            res = eval_fn([settings[i] for i in range(n)])
+            times, mets = (res if nm > 0 else (res, None))
+            for i in range(n):
+                ms[i] = float(times[i])
+                for k in range(nm):
+                    metrics[i * nm + k] = float(mets[i][k])
+            return 0
+        except Exception:
+            import traceback
+            traceback.print_exc()
+            return 1
+    return EVAL_FN(_cb)
+
+
+def cst_dist_create_host(h, nranks: int, rank: int, bcast, allgather):
+    """Tuning-only cst_dist whose collectives are Python callables:
+    bcast(bytearray-like memoryview, root) in place; allgather(bytes) -> bytes (rank order).
+    Returns (handle, keepalive) — keep the second object alive with the handle."""
+    def _b(user, buf, nbytes, root):
+        try:
+            mv = (ctypes.c_char * nbytes).from_address(buf)
+            out = bcast(bytes(mv), root)
+            ctypes.memmove(buf, out, nbytes)
+            return 0
+        except Exception:
+            import traceback
+            traceback.print_exc()
+            return 1
+
+    def _g(user, send, recv, nbytes):
+        try:
+            data = allgather(ctypes.string_at(send, nbytes))
+            assert len(data) == nbytes * nranks
+            ctypes.memmove(recv, data, len(data))
+            return 0
+        except Exception:
+            import traceback
+            traceback.print_exc()
+            return 1
+
+    coll = cst_collectives(None, BCAST_FN(_b), ALLGATHER_FN(_g))
+    d = ctypes.c_void_p()
+    check(_lib.cst_dist_create_host(h, nranks, rank, ctypes.byref(coll), ctypes.byref(d)))
+    return d, (coll, _b, _g)
+
+
+def cst_dist_tune(d, opts: cst_tune_opts, in_ptrs, scratch_out_ptrs, local_eval=None):
+    """Collective population-parallel cst_tune (include/cst.h).  local_eval: as cst_tune's
+    eval_fn, for this rank's share only (None = built-in GPU timing on in/scratch_out)."""
+    pi, _a = _ptrs(in_ptrs)
+    po, _b = _ptrs(scratch_out_ptrs)
+    best, rep = cst_setting(), cst_tune_report()
+    cb = _eval_cb(local_eval, opts.n_user_metrics)
+    check(_lib.cst_dist_tune(d, ctypes.byref(opts), pi, po, cb, None, ctypes.byref(best),
+                             ctypes.byref(rep)))
+    return best, rep
 
 
 def cst_tune(h, opts: cst_tune_opts, in_ptrs, scratch_out_ptrs, eval_fn=None):

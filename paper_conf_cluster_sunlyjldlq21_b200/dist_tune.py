@@ -1,11 +1,11 @@
-"""Population-parallel evaluation for cst_tune (SURVEY §8(e), P:296 multi-process GA).
+"""Population-parallel cst_tune over torch.distributed ranks.
 
-Rank 0 runs the C++ tuner; every batch of candidates it asks for (the 128-setting dataset,
-then each GA generation of 2 x 16 individuals) is spread round-robin over all ranks, each
-rank evaluates its share on its own GPU (libcst: NVRTC code generation + CUDA-event timing)
-and the fitness vectors are all-gathered through torch.distributed (host coordination,
-8 B per candidate).  The GA itself stays on rank 0 and is deterministic, so the trajectory
-does not depend on the number of evaluating ranks.
+The protocol lives in libcst (`cst_dist_tune`, csrc/dist/dist_tune.cpp): rank 0 runs the
+tuner, every batch of candidates is broadcast, rank k evaluates candidates i with
+i % world == k on its own GPU, and the fitness vectors are all-gathered.  This module only
+supplies the host collectives (torch.distributed object collectives, so gloo and NCCL
+process groups both work) and argument marshalling.  On a NCCL-transport cst_dist the
+library can use its own NCCL communicator instead: call C.cst_dist_tune on that handle.
 """
 from __future__ import annotations
 
@@ -13,60 +13,43 @@ import torch.distributed as dist
 
 from . import cst as C
 
-_STOP = "__cst_tune_stop__"
+
+def _collectives(group):
+    def bcast(data: bytes, root: int) -> bytes:
+        obj = [data]
+        dist.broadcast_object_list(obj, src=root, group=group)
+        return obj[0]
+
+    def allgather(data: bytes) -> bytes:
+        parts = [None] * dist.get_world_size(group)
+        dist.all_gather_object(parts, data, group=group)
+        return b"".join(parts)
+    return bcast, allgather
 
 
-def _share(batch, rank, world):
-    return [(i, t) for i, t in enumerate(batch) if i % world == rank]
-
-
-def _merge(parts, n):
-    out = [None] * n
-    for part in parts:
-        for i, v in part:
-            out[i] = v
-    return out
-
-
-def tune_distributed(h, opts, in_ptrs, out_ptrs, evaluate_local, group=None):
+def tune_distributed(h, opts, in_ptrs, out_ptrs, evaluate_local=None, group=None):
     """Collective over `group`.  evaluate_local(setting_dict) -> ms (or (ms, metrics) when
-    opts.n_user_metrics > 0) runs on every rank for its share of each batch.
-    Returns (best cst_setting, cst_tune_report or None on ranks != 0) on every rank."""
+    opts.n_user_metrics > 0) runs on every rank for its share of each batch; None = libcst's
+    built-in GPU timing on in_ptrs / out_ptrs (this rank's replica of the grid).
+    Returns (best cst_setting, cst_tune_report) on every rank (rank 0's result)."""
     rank = dist.get_rank(group)
     world = dist.get_world_size(group)
-    nm = opts.n_user_metrics
+    bcast, allgather = _collectives(group)
+    d, keep = C.cst_dist_create_host(h, world, rank, bcast, allgather)
+    local = None
+    if evaluate_local is not None:
+        nm = opts.n_user_metrics
 
-    def serve(batch):
-        mine = [(i, evaluate_local(dict(zip(C.FIELDS, t)))) for i, t in _share(batch, rank, world)]
-        parts = [None] * world
-        dist.all_gather_object(parts, mine, group=group)
-        return _merge(parts, len(batch))
-
-    if rank == 0:
-        def cb(settings):
-            batch = [s.as_tuple() for s in settings]
-            dist.broadcast_object_list([batch], src=0, group=group)
-            res = serve(batch)
+        def local(settings):
+            res = [evaluate_local(s.as_dict()) for s in settings]
             if nm > 0:
                 return [r[0] for r in res], [r[1] for r in res]
             return res
-
-        try:
-            best, rep = C.cst_tune(h, opts, in_ptrs, out_ptrs, eval_fn=cb)
-        finally:
-            dist.broadcast_object_list([_STOP], src=0, group=group)
-        obj = [best.as_dict()]
-        dist.broadcast_object_list(obj, src=0, group=group)
-        return best, rep
-    while True:
-        obj = [None]
-        dist.broadcast_object_list(obj, src=0, group=group)
-        if isinstance(obj[0], str) and obj[0] == _STOP:
-            break
-        serve(obj[0])
-    obj = [None]
-    dist.broadcast_object_list(obj, src=0, group=group)
-    return C.cst_setting.from_dict(obj[0]), None
+    try:
+        return C.cst_dist_tune(d, opts, in_ptrs, out_ptrs, local)
+    finally:
+        C.cst_dist_destroy(d)
+        del keep
 
 
 def gpu_evaluator(stencil, ins, outs, warmup=2, reps=5):

@@ -149,3 +149,39 @@ def test_population_parallel_tuning_equals_single_process(tmp_path):
     assert tuple(r0[:-1]) == best.as_tuple()
     rep_d = np.load(tmp_path / "rep.npy")
     assert rep_d[0] == rep.best_ms and int(rep_d[1]) == rep.evaluations
+
+
+def _tune_fail_worker(rank, world, port, outdir):
+    from paper_conf_cluster_sunlyjldlq21_b200 import cst as C
+    from paper_conf_cluster_sunlyjldlq21_b200.dist_tune import tune_distributed
+    import test_tuner as TT
+    _init(rank, world, port)
+    g = C.make_grid(*TT.M, TT.R)
+    h = C.cst_stencil_create(TT.KIND, TT.R, [1.0] * 7, g)
+    o = C.cst_tune_opts_default()
+    o.n_user_metrics = TT.NMET
+    o.time_budget_s = 0
+
+    def ev(d):                     # every candidate fails -> rank 0's tuner fails
+        raise RuntimeError("evaluation failed")
+
+    status = "ok"
+    try:
+        tune_distributed(h, o, [], [], ev)
+    except C.CstError as e:
+        status = f"{e.status}"
+    with open(os.path.join(outdir, f"fail{rank}.txt"), "w") as f:
+        f.write(status)
+    C.cst_stencil_destroy(h)
+    dist.destroy_process_group()
+
+
+def test_population_parallel_tuning_error_reaches_every_rank(tmp_path):
+    """if rank 0's tuner fails, the result message is still broadcast, so every
+    rank returns the error instead of blocking."""
+    world = 2
+    mp.spawn(_tune_fail_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world,
+             join=True)
+    got = [open(tmp_path / f"fail{k}.txt").read() for k in range(world)]
+    assert got[0] == got[1] != "ok", got
+
