@@ -6,11 +6,15 @@ N=1 workload: order-4 25-point star (FD Laplacian, weights /5040), 512^3 FP64 in
 halo 4, the tuned setting from tuned/star25_512.json (cst_tune output, then the A/B-checked
 hill climb of tools/tune.py --refine-all; the default setting if absent).  A step = one sweep (one kernel launch) over inputs resident in HBM; the two
 1.18 GB arrays exceed the 126 MB L2, so no flush is needed between steps.
-N>1 (torchrun, one rank per GPU): weak scaling of the z-slab decomposition — every rank owns
-a 512^3 slab of a (512*N) x 512 x 512 grid and exchanges 4-plane halos with its neighbours
-every step (cst_dist_sweep: by default the boundary kernels store straight into the
-neighbours' halos over peer memory, --halo nccl selects NCCL send/recv overlapped with the
-interior).  value = all ranks' points / max-over-ranks time.
+N>1 (torchrun, one rank per GPU): BASELINE configs[4] — the order-4 star on a z-slab
+decomposed 1024 x 1024 grid with a 4-plane halo exchange per step.  Headline = WEAK scaling,
+256 x 1024 x 1024 per rank (global nz = 256 N), NCCL send/recv overlapped with the interior
+(north_star); value = all ranks' points / max-over-ranks device time.  The same line carries
+"strong" (the 2048 x 1024 x 1024 grid, 2048/N planes per rank), "p2p" (weak scaling with the
+fused peer-memory halo stores) and "population_eval" (configs[4]'s GA part:
+evaluations/s of one 32-candidate generation spread round-robin over the N GPUs, C5c).  At
+N=1 the same three single-GPU baselines appear in other_configs (c5_weak_slab_1gpu,
+c5_strong_1gpu, c5c_population_eval_g1), so E(N) can be formed from either line.
 
 Extra keys: roofline (dominant kernel = the sweep), cpu_baseline (the oracle on a bounded
 sample, rank 0 at N=1), e2e (cst_sweep_host: H2D + sweep + D2H through the C ABI), clocks
@@ -329,6 +333,221 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+# --------------------------------------------------------------------------- configs[4]
+C5_NXY, C5_WEAK_NZ, C5_STRONG_NZ, C5_SEED = 1024, 256, 2048, 5
+
+
+def _gather(dist, world, x):
+    """Every rank's x (all ranks, rank order); [x] on one process."""
+    if world == 1:
+        return [x]
+    out = [None] * world
+    dist.all_gather_object(out, x)
+    return out
+
+
+def c5_setting(C, h):
+    """The tuned star25 setting (tuned/star25_512.json) if valid on this slab, else the
+    library default."""
+    try:
+        s, src = load_setting(C, h)
+        return s, src
+    except C.CstError:
+        return C.cst_setting_default(h), "cst_setting_default"
+
+
+def c5_sweep(C, torch, dist, rank, world, local, nzl, transport, steps, warmup, peak):
+    """One z-slab sweep series of configs[4] (star25, 1024 x 1024 planes, nzl local planes
+    per rank): `warmup` + `steps` single-step cst_dist_sweep calls (cst_sweep at world 1),
+    CUDA events per step on the sweep stream, total time = max over ranks.  Returns the
+    rank-0 view (aggregate GSt/s, per-rank roofline) or None where the transport could
+    not be set up (reason given)."""
+    g = C.make_grid(C5_NXY, C5_NXY, nzl, R)
+    h = C.cst_stencil_create(C.CST_STAR, R, star_coeffs(), g, local)
+    s, s_src = c5_setting(C, h)
+    u = torch.empty(g.numel, dtype=torch.float64, device="cuda")
+    v = torch.empty(g.numel, dtype=torch.float64, device="cuda")
+    stream = torch.cuda.current_stream()
+    for t in (u, v):
+        C.cst_fill_uniform(g, t.data_ptr(), C5_SEED, 0, C5_NXY, C5_NXY, rank * nzl,
+                           float("nan"), stream.cuda_stream)
+    d, why = None, ""
+    if world > 1 and transport == "nccl":
+        uid = C.cst_dist_nccl_unique_id() if rank == 0 else None
+        obj = [uid]
+        dist.broadcast_object_list(obj, src=0)
+        d = C.cst_dist_create(h, world, rank, obj[0])
+    elif world > 1:
+        # every rank must take the same transport: export, all-gather, import, MIN-agree
+        d = C.cst_dist_create(h, world, rank, None)
+        ok, mine = True, None
+        try:
+            mine = C.cst_dist_p2p_export(d, [u.data_ptr()], [v.data_ptr()])
+        except C.CstError as e:
+            ok, why = False, str(e)
+        blobs = [None] * world
+        dist.all_gather_object(blobs, (ok, mine))
+        if ok and all(b[0] for b in blobs):
+            try:
+                for peer in (rank - 1, rank + 1):
+                    if 0 <= peer < world:
+                        C.cst_dist_p2p_import(d, peer, blobs[peer][1])
+            except C.CstError as e:
+                ok, why = False, str(e)
+        else:
+            ok, why = False, why or "a peer could not export"
+        if not all(_gather(dist, world, ok)):
+            C.cst_dist_destroy(d)
+            C.cst_stencil_destroy(h)
+            return {"unavailable": "p2p setup failed: " + (why or "on another rank")[:160]}
+    bufs = [u, v]
+
+    def step(i):
+        a, b = bufs[i % 2], bufs[1 - i % 2]
+        if d is not None:
+            C.cst_dist_sweep(d, s, [a.data_ptr()], [b.data_ptr()], 1, stream.cuda_stream)
+        else:
+            C.cst_sweep(h, s, [a.data_ptr()], [b.data_ptr()], 1, stream.cuda_stream)
+
+    for i in range(max(warmup, 3)):
+        step(i)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(steps + 1)]
+    evs[0].record(stream)
+    launches = 0
+    for i in range(steps):
+        step(i)
+        launches += C.cst_last_launch_count(h)
+        evs[i + 1].record(stream)
+    torch.cuda.synchronize()
+    per = [evs[i].elapsed_time(evs[i + 1]) for i in range(steps)]
+    mine_ms = evs[0].elapsed_time(evs[-1])
+    tot = max(_gather(dist, world, mine_ms))
+    allr = [m / steps for m in _gather(dist, world, mine_ms)]
+    ms = tot / steps
+    pts_rank = C5_NXY * C5_NXY * nzl
+    res = {"grid_global": [C5_NXY, C5_NXY, nzl * world], "planes_per_rank": nzl,
+           "transport": (transport if world > 1 else "none (single GPU)"),
+           "steps": steps, "ms_per_step": ms, "gstencils": pts_rank * world / (ms * 1e-3) / 1e9,
+           "gstencils_per_gpu": pts_rank / (ms * 1e-3) / 1e9,
+           "per_rank_ms_per_step": allr,
+           "per_rank_roofline": [{"achieved_GBs": 16 * pts_rank / (m * 1e-3) / 1e9,
+                                  "frac": 16 * pts_rank / (m * 1e-3) / 1e9 / peak} for m in allr],
+           "rank0_step_ms": {"median": statistics.median(per), "max": max(per)},
+           "launches_per_step": launches / steps, "setting_source": s_src,
+           "halo_bytes_per_side_per_step": (R * g.pitch_x * g.pitch_y * 8 if world > 1 else 0)}
+    if d is not None:
+        C.cst_dist_destroy(d)
+    del u, v, bufs
+    C.cst_stencil_destroy(h)
+    torch.cuda.empty_cache()
+    return res
+
+
+def c5_population_eval(C, torch, dist, rank, world, local, n_cand=32, reps=5):
+    """configs[4]'s GA part: one GA generation (2 x 16 candidates)
+    of star25 settings on the 256 x 1024 x 1024 slab, replayed from a fixed seeded list,
+    spread round-robin over the ranks (the cst_dist_tune protocol): each rank times its
+    share (2 warm-ups + median of `reps`), then the fitness vectors are all-gathered.  Code
+    generation is done before the timed region (warm cubin cache).  evaluations/s = n_cand /
+    max-over-ranks wall time of the round (host wall clock: every evaluation synchronises)."""
+    import random
+    g = C.make_grid(C5_NXY, C5_NXY, C5_WEAK_NZ, R)
+    h = C.cst_stencil_create(C.CST_STAR, R, star_coeffs(), g, local)
+    count = C.cst_space_count(h)
+    rng = random.Random(12345)
+    cands = []
+    while len(cands) < n_cand:        # the same list on every rank; skip R13 rejections
+        s = C.cst_space_at(h, rng.randrange(count))
+        if s.as_dict()["bt"] == 1:
+            cands.append(s)
+    u, v = [torch.empty(g.numel, dtype=torch.float64, device="cuda") for _ in range(2)]
+    C.cst_fill_uniform(g, u.data_ptr(), C5_SEED, 0, C5_NXY, C5_NXY, rank * C5_WEAK_NZ)
+    mine = [i for i in range(n_cand) if i % world == rank]
+    for i in mine:
+        try:
+            C.cst_variant_compile(h, cands[i])
+        except C.CstError:
+            pass
+    stream = torch.cuda.current_stream().cuda_stream
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    ms = {}
+    for i in mine:
+        try:
+            ms[i] = C.cst_time_setting(h, cands[i], [u.data_ptr()], [v.data_ptr()], 2, reps,
+                                       stream)
+        except C.CstError:
+            ms[i] = float("inf")
+    if world > 1:
+        parts = [None] * world
+        dist.all_gather_object(parts, ms)
+        for p in parts:
+            ms.update(p)
+    el = max(_gather(dist, world, time.perf_counter() - t0))
+    valid = [m for m in ms.values() if m < float("inf")]
+    del u, v
+    C.cst_stencil_destroy(h)
+    torch.cuda.empty_cache()
+    return {"candidates": n_cand, "evaluated_by_rank": [len([i for i in range(n_cand)
+                                                            if i % world == k])
+                                                       for k in range(world)],
+            "valid": len(valid), "wall_s_max_over_ranks": el,
+            "evaluations_per_s": n_cand / el, "reps_per_eval": reps, "warmup_per_eval": 2,
+            "best_ms": min(valid) if valid else None,
+            "clock": "host wall clock around the round (evaluations synchronise per candidate)"}
+
+
+def run_multi(args, C, torch, dist, rank, world, local, shared=False):
+    """N > 1: BASELINE configs[4] (see the module docstring).  shared (CST_BENCH_SHARED_GPU,
+    tests only): all ranks on one GPU, where NCCL cannot run — the NCCL lines become p2p."""
+    peak, peak_src = measured_peaks()
+    main_t = "p2p" if shared else "nccl"
+    clocks = ClockSampler(local)
+    clocks.start()
+    weak = c5_sweep(C, torch, dist, rank, world, local, C5_WEAK_NZ, main_t, args.steps,
+                    args.warmup, peak)
+    clk = clocks.stop()
+    strong = c5_sweep(C, torch, dist, rank, world, local, C5_STRONG_NZ // world, main_t,
+                      max(3, args.steps // 2), args.warmup, peak)
+    p2p = c5_sweep(C, torch, dist, rank, world, local, C5_WEAK_NZ, "p2p", args.steps,
+                   args.warmup, peak)
+    pop = c5_population_eval(C, torch, dist, rank, world, local)
+    if rank == 0:
+        pts_rank = C5_NXY * C5_NXY * C5_WEAK_NZ
+        r0 = weak["per_rank_roofline"][0]
+        line = {"metric": METRIC, "value": weak["gstencils"], "unit": UNIT, "n_gpus": world,
+                "steps": args.steps, "warmup": max(args.warmup, 3),
+                "ms_per_step": weak["ms_per_step"], "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic (cstgen splitmix64 U[-1,1), seed 5, global coordinates per "
+                        "slab, device generator)",
+                "config": {"workload": "configs[4]: order-4 25-point star (FD Laplacian /5040) "
+                                       "z-slab decomposed, 256 x 1024 x 1024 per rank (global "
+                                       f"{256 * world} x 1024 x 1024), NCCL halo exchange "
+                                       "overlapped with the interior",
+                           "grid": weak["grid_global"], "halo": R,
+                           "parallelism": f"z-slab x{world}",
+                           "l2": "inputs larger than L2 (2 x 2.3 GB per GPU), no flush"},
+                "roofline": {"bound": "hbm", "achieved": r0["achieved_GBs"], "peak": peak,
+                             "unit": "GB/s", "frac": r0["frac"], "traffic": None,
+                             "peak_source": peak_src,
+                             "alg_bytes_per_launch": 16 * pts_rank,
+                             "kernel": "cst_kernel (star25 slab sweep, rank 0; per-rank "
+                                       "fractions under weak.per_rank_roofline)"},
+                "clocks": clk, "e2e": None, "cpu_baseline": None,
+                "gpu_launches": int(weak["launches_per_step"] * args.steps),
+                "weak": weak, "strong": strong, "p2p": p2p, "population_eval": pop,
+                "nccl_debug": os.environ.get("NCCL_DEBUG", ""),
+                "shared_gpu_test_mode": shared}
+        print(json.dumps(line), flush=True)
+    dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -338,9 +557,6 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-other-configs", action="store_true")
-    ap.add_argument("--halo", default=os.environ.get("CST_BENCH_HALO", "p2p"),
-                    choices=["p2p", "nccl"],
-                    help="N > 1: fused peer-memory halo stores (default) or NCCL send/recv")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -354,9 +570,18 @@ def main():
 
     from paper_conf_cluster_sunlyjldlq21_b200 import cst as C
 
+    shared = os.environ.get("CST_BENCH_SHARED_GPU") == "1"
+    if shared:   # plumbing test on a one-GPU box: every rank on cuda:0, gloo, p2p only
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            os.environ.setdefault("NCCL_DEBUG", "INFO")        # communicator logs on stderr
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        return run_multi(args, C, torch, dist, rank, world, local, shared)
 
     grid = C.make_grid(N, N, N, R)
     h = C.cst_stencil_create(C.CST_STAR, R, star_coeffs(), grid, local)
@@ -364,60 +589,18 @@ def main():
     u = torch.empty(grid.numel, dtype=torch.float64, device="cuda")
     v = torch.empty(grid.numel, dtype=torch.float64, device="cuda")
     stream = torch.cuda.current_stream()
-    z0 = rank * N
-    C.cst_fill_uniform(grid, u.data_ptr(), SEED, 0, N, N, z0, float("nan"), stream.cuda_stream)
-    C.cst_fill_uniform(grid, v.data_ptr(), SEED, 0, N, N, z0, float("nan"), stream.cuda_stream)
-    dist_h = None
-    halo_used = args.halo
-    if world > 1 and args.halo == "p2p":
-        # boundary kernels store straight into the neighbours' halos (NVLink peer stores).
-        # Every rank must take the same transport: export, all-gather (ok, blob), import,
-        # agree by MIN-reduce; any failure anywhere -> all ranks fall back to NCCL.
-        dist_h = C.cst_dist_create(h, world, rank, None)
-        ok, why, mine = True, "", None
-        try:
-            mine = C.cst_dist_p2p_export(dist_h, [u.data_ptr()], [v.data_ptr()])
-        except C.CstError as e:
-            ok, why = False, str(e)
-        blobs = [None] * world
-        dist.all_gather_object(blobs, (ok, mine))
-        if ok and all(b[0] for b in blobs):
-            try:
-                for peer in (rank - 1, rank + 1):
-                    if 0 <= peer < world:
-                        C.cst_dist_p2p_import(dist_h, peer, blobs[peer][1])
-            except C.CstError as e:
-                ok, why = False, str(e)
-        else:
-            ok, why = False, why or "a peer could not export"
-        flag = torch.tensor([1 if ok else 0], device="cuda")
-        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
-        if int(flag.item()) == 0:
-            C.cst_dist_destroy(dist_h)
-            dist_h = None
-            halo_used = "nccl (p2p setup failed: %s)" % (why or "on another rank")[:120]
-    if world > 1 and dist_h is None:
-        uid = C.cst_dist_nccl_unique_id() if rank == 0 else None
-        obj = [uid]
-        dist.broadcast_object_list(obj, src=0)
-        dist_h = C.cst_dist_create(h, world, rank, obj[0])
+    C.cst_fill_uniform(grid, u.data_ptr(), SEED, 0, N, N, 0, float("nan"), stream.cuda_stream)
+    C.cst_fill_uniform(grid, v.data_ptr(), SEED, 0, N, N, 0, float("nan"), stream.cuda_stream)
 
     def step():
-        if dist_h is not None:
-            C.cst_dist_sweep(dist_h, s, [u.data_ptr()], [v.data_ptr()], 1, stream.cuda_stream)
-        else:
-            C.cst_sweep(h, s, [u.data_ptr()], [v.data_ptr()], 1, stream.cuda_stream)
+        C.cst_sweep(h, s, [u.data_ptr()], [v.data_ptr()], 1, stream.cuda_stream)
 
     for _ in range(max(args.warmup, 3)):
         step()
     torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
     clocks = ClockSampler(local)
     evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
     torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
     launches = 0
     clocks.start()
     evs[0].record(stream)
@@ -427,17 +610,11 @@ def main():
         evs[i + 1].record(stream)
     torch.cuda.synchronize()
     clk = clocks.stop()
-    if world > 1:
-        dist.barrier()
     per = [evs[i].elapsed_time(evs[i + 1]) for i in range(args.steps)]
     total_ms = evs[0].elapsed_time(evs[-1])
-    if world > 1:
-        t = torch.tensor([total_ms], device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
     ms_step = total_ms / args.steps
     pts = N * N * N
-    value = pts * world / (ms_step * 1e-3) / 1e9
+    value = pts / (ms_step * 1e-3) / 1e9
 
     peak, peak_src = measured_peaks()
     avg_launch_ms = statistics.mean(per)
@@ -450,7 +627,7 @@ def main():
 
     # ---- e2e: the same metric through cst_sweep_host (pinned host buffers, H2D + D2H)
     e2e = None
-    if rank == 0 and world == 1 and args.e2e_steps > 0:
+    if args.e2e_steps > 0:
         hu = torch.empty(grid.numel, dtype=torch.float64).pin_memory()
         hv = torch.empty(grid.numel, dtype=torch.float64).pin_memory()
         hu.copy_(u.cpu())
@@ -464,7 +641,7 @@ def main():
                "steps": args.e2e_steps, "api": "cst_sweep_host"}
 
     others = None
-    if rank == 0 and world == 1 and not args.no_other_configs:
+    if not args.no_other_configs:
         del u, v
         torch.cuda.empty_cache()
         try:
@@ -474,9 +651,15 @@ def main():
         others = other_configs(C, torch, peak, fp64_peak=fp64_peak)
         others["fp64_peak_TFLOPs_measured"] = fp64_peak
         others["next2_tblock_star7_512_T8"] = tblock_config(C, torch, peak)
+        # configs[4] single-GPU baselines (the N = 1 points of the scaling curves)
+        others["c5_weak_slab_1gpu"] = c5_sweep(C, torch, None, 0, 1, local, C5_WEAK_NZ, "none",
+                                               20, 3, peak)
+        others["c5_strong_1gpu"] = c5_sweep(C, torch, None, 0, 1, local, C5_STRONG_NZ, "none",
+                                            5, 3, peak)
+        others["c5c_population_eval_g1"] = c5_population_eval(C, torch, None, 0, 1, local)
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if not args.no_cpu_baseline:
         cpu = cpu_baseline()
 
     if rank == 0:
@@ -485,16 +668,12 @@ def main():
                 "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
                 "data": "synthetic (cstgen splitmix64 U[-1,1), seed 2, device generator)",
                 "config": {"workload": "star25: order-4 25-point star (FD Laplacian /5040), "
-                                       "512^3 FP64 interior per GPU (BASELINE configs[1])"
-                                       + (("; z-slab weak scaling, halo exchange: "
-                                           + ("fused peer-memory stores" if halo_used == "p2p"
-                                              else "NCCL send/recv" if halo_used == "nccl"
-                                              else halo_used)) if world > 1 else ""),
-                           "grid": [N, N, N * world], "halo": R,
+                                       "512^3 FP64 interior (BASELINE configs[1])",
+                           "grid": [N, N, N], "halo": R,
                            "setting": s.as_dict(), "setting_source": s_src,
                            "l2": "inputs larger than L2 (2 x %.2f GB per GPU), no flush"
                                  % (grid.numel * 8 / 1e9),
-                           "parallelism": f"z-slab x{world}" if world > 1 else "single GPU"},
+                           "parallelism": "single GPU"},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
                 "other_configs": others,
                 "gpu_launches": launches,
@@ -503,11 +682,7 @@ def main():
                                 "slow_steps_gt_1.1x_median":
                                     sum(1 for x in per if x > 1.1 * statistics.median(per))}}
         print(json.dumps(line), flush=True)
-    if dist_h is not None:
-        C.cst_dist_destroy(dist_h)
     C.cst_stencil_destroy(h)
-    if world > 1:
-        dist.destroy_process_group()
 
 
 if __name__ == "__main__":

@@ -1,7 +1,7 @@
 """csTuner tuning-quality experiments on B200 (the csTuner line of
 Figs. 8/9/11/12, P:349-361, P:385-405 — the comparison systems are out of scope).
 
-  python tools/tuning_quality.py --out profiles/r01_tuning_quality.json [--budget 100]
+  python tools/tuning_quality.py --out profiles/r02_tuning_quality.json [--budget 100]
 
 1. Ground truth: exhaustive timing of a restricted sub-space of the star25 512^3 space (TMA
    staging, z streaming, retiming, UF = CM = 1; TB_x, TB_y, BM_x, BM_y, SB, prefetch free).
@@ -101,7 +101,9 @@ def run_cstuner(h, u, v, seed, budget, ratio=0.10, tag="", warm_start=1):
             "wall_s": rep.wall_s, "eval_s": rep.eval_s, "jit_s": rep.jit_s,
             "preproc_s": rep.preproc_s, "sampled_count": rep.sampled_count,
             "space_count": rep.space_count, "trace": j.get("trace", []),
-            "metrics_source": j.get("metrics_source")}
+            "metrics_source": j.get("metrics_source"), "phases": j.get("phases"),
+            "noise": j.get("noise"), "phases_cv_stop": rep.phases_cv_stop,
+            "filter_s": j.get("filter_s")}
 
 
 def run_random(h, u, v, seed, budget, batch=32):
@@ -123,13 +125,18 @@ def run_random(h, u, v, seed, budget, batch=32):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r01_tuning_quality.json"))
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r02_tuning_quality.json"))
     ap.add_argument("--budget", type=float, default=100.0)
     ap.add_argument("--seeds", type=int, default=3)
     args = ap.parse_args()
     g, h, u, v = make()
     res = {"workload": "star25 (order-4 25-point star) 512^3 FP64, B200, inputs resident",
            "space_count": C.cst_space_count(h)}
+    os.makedirs(os.path.dirname(args.out), exist_ok=True)
+
+    def save():                      # after every stage: a cut-off run keeps what it has
+        with open(args.out, "w") as f:
+            json.dump(res, f, indent=1)
     # 1. exhaustive sub-space
     t0 = time.time()
     sub = subspace(h)
@@ -143,11 +150,13 @@ def main():
                                                         [u.data_ptr()], [v.data_ptr()], 2, 5)}
     print(json.dumps({"subspace": {k: res["subspace"][k] for k in ("size", "optimum_ms",
                                                                     "seconds")}}), flush=True)
+    save()
     # 2. iso-time: csTuner vs random search
     res["cstuner"] = [run_cstuner(h, u, v, s + 1, args.budget, tag="iso") for s in range(args.seeds)]
     for r in res["cstuner"]:
         print(json.dumps({k: r[k] for k in ("seed", "best_ms", "evaluations", "wall_s",
                                             "dataset_s")}), flush=True)
+    save()
     # the paper's method as published: the dataset is a pure random sample (no warm start)
     res["cstuner_no_warm_start"] = [run_cstuner(h, u, v, s + 1, args.budget, tag="cold",
                                                 warm_start=0) for s in range(args.seeds)]
@@ -157,15 +166,14 @@ def main():
     res["random_search"] = [run_random(h, u, v, s + 1, args.budget) for s in range(args.seeds)]
     for r in res["random_search"]:
         print(json.dumps({k: r[k] for k in ("seed", "best_ms", "evaluations")}), flush=True)
+    save()
     # 3. sampling ratio sweep
     res["sampling_ratio_sweep"] = [run_cstuner(h, u, v, 1, args.budget, ratio=q, tag="ratio")
                                    for q in (0.05, 0.10, 0.20, 0.50)]
     for r in res["sampling_ratio_sweep"]:
         print(json.dumps({k: r[k] for k in ("sampling_ratio", "best_ms", "preproc_s", "eval_s",
                                             "sampled_count")}), flush=True)
-    os.makedirs(os.path.dirname(args.out), exist_ok=True)
-    with open(args.out, "w") as f:
-        json.dump(res, f, indent=1)
+    save()
     C.cst_stencil_destroy(h)
 
 
