@@ -54,6 +54,7 @@ cst_status driver(const Driver** out) {
               get("cuFuncSetAttribute", (void**)&d.cuFuncSetAttribute) &&
               get("cuFuncGetAttribute", (void**)&d.cuFuncGetAttribute) &&
               get("cuLaunchKernel", (void**)&d.cuLaunchKernel) &&
+              get("cuLaunchKernelEx", (void**)&d.cuLaunchKernelEx) &&
               get("cuTensorMapEncodeTiled", (void**)&d.cuTensorMapEncodeTiled) &&
               get("cuOccupancyMaxActiveBlocksPerMultiprocessor", (void**)&d.cuOccupancy) &&
               get("cuGetErrorString", (void**)&d.cuGetErrorString) &&
@@ -74,10 +75,20 @@ cst_status driver(const Driver** out) {
 struct Geometry {
   unsigned grid_x, grid_y, threads;
   int tiles_a, tiles_b, tiles_c, chunks;
+  int cluster = 1;  // CTAs per cluster along blockIdx.x (streaming: b-stacked tiles)
   int box[3];  // TMA box dims (x, y, z)
 };
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+int cluster_b() {
+  static const int v = [] {
+    const char* e = std::getenv("CST_CLUSTER_B");
+    const int c = e ? std::atoi(e) : 1;
+    return (c == 2 || c == 4 || c == 8) ? c : 1;
+  }();
+  return v;
+}
 
 static Geometry geometry(const StencilInfo& st, const Tuple& t, int64_t nx, int64_t ny,
                          int64_t nz) {
@@ -93,7 +104,8 @@ static Geometry geometry(const StencilInfo& st, const Tuple& t, int64_t nx, int6
     g.tiles_b = (int)cdiv(sz ? ny : nz, sz ? T[1] : T[2]);
     g.chunks = (int)cdiv(sz ? nz : ny, t[F_SB]);
     g.tiles_c = 1;
-    g.grid_x = (unsigned)(g.tiles_a * (int64_t)g.tiles_b);
+    g.cluster = cluster_b();
+    g.grid_x = (unsigned)(g.tiles_a * ((g.tiles_b + g.cluster - 1) / g.cluster * (int64_t)g.cluster));
     g.grid_y = (unsigned)g.chunks;
     g.box[0] = (int)T[0] + 2 * xr;
     if (t[F_BT] > 1) {  // temporally blocked: the input box carries bt halos per side
@@ -536,9 +548,29 @@ cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* 
   P.tiles_c = g.tiles_c;
   P.chunks = g.chunks;
   void* args[] = {&P};
-  st = cu_check(d->cuLaunchKernel(v->fn, g.grid_x, g.grid_y, 1, g.threads, 1, 1,
-                                  (unsigned)v->smem, (CUstream)stream, args, nullptr),
-                "cuLaunchKernel");
+  if (g.cluster > 1) {
+    CUlaunchConfig cfg;
+    std::memset(&cfg, 0, sizeof cfg);
+    cfg.gridDimX = g.grid_x;
+    cfg.gridDimY = g.grid_y;
+    cfg.gridDimZ = 1;
+    cfg.blockDimX = g.threads;
+    cfg.blockDimY = cfg.blockDimZ = 1;
+    cfg.sharedMemBytes = (unsigned)v->smem;
+    cfg.hStream = (CUstream)stream;
+    CUlaunchAttribute at;
+    std::memset(&at, 0, sizeof at);
+    at.id = CU_LAUNCH_ATTRIBUTE_CLUSTER_DIMENSION;
+    at.value.clusterDim.x = (unsigned)g.cluster;
+    at.value.clusterDim.y = at.value.clusterDim.z = 1;
+    cfg.attrs = &at;
+    cfg.numAttrs = 1;
+    st = cu_check(d->cuLaunchKernelEx(&cfg, v->fn, args, nullptr), "cuLaunchKernelEx(cluster)");
+  } else {
+    st = cu_check(d->cuLaunchKernel(v->fn, g.grid_x, g.grid_y, 1, g.threads, 1, 1,
+                                    (unsigned)v->smem, (CUstream)stream, args, nullptr),
+                  "cuLaunchKernel");
+  }
   if (st != CST_OK) return st;
   ++h->last_launches;
   return CST_OK;
