@@ -167,6 +167,26 @@ OTHER = {
                        "320^3 as in Table III — FP64-bound"),
 }
 FLOPS_PER_POINT = {1: None, 2: 53, 3: 358, 4: 666}
+FP64_PEAK_SOURCE = ("cst_fp64_peak: DFMA-chain microbenchmark on this GPU (csrc/runtime/peak.cu); "
+                    "MEASURED_PEAKS.json has no FP64 figure")
+COUNTER_KEY = {"c3_box27_512": "box27", "c4_hypterm_512": "hypterm", "next1_rhs4_320": "rhs4"}
+
+
+def fp64_from_counters(key, pts, ms, fp64_peak):
+    """FP64 fraction from ncu instruction counts: executed FP64 FLOPs per point
+    = 2 DFMA + DADD + DMUL from profiles/r02_fp64_counts.json (one ncu launch of the same
+    tuned setting), times the points, over this run's CUDA-event time."""
+    p = os.path.join(ROOT, "profiles", "r02_fp64_counts.json")
+    if not key or not fp64_peak or not os.path.exists(p):
+        return {}
+    try:
+        d = json.load(open(p))[key]
+    except (KeyError, ValueError):
+        return {}
+    ex = d["executed_fp64_flops_per_point"]
+    tf = pts * ex / (ms * 1e-3) / 1e12
+    return {"fp64_executed_flops_per_point_ncu": ex, "achieved_TFLOPs_executed": tf,
+            "fp64_frac_counters": tf / fp64_peak, "fp64_counts_source": "profiles/r02_fp64_counts.json"}
 
 
 def other_coeffs(kind, r):
@@ -218,7 +238,9 @@ def other_configs(C, torch, peak, steps=10, fp64_peak=None):
         if fpp and fp64_peak:
             tf = pts * fpp / (ms * 1e-3) / 1e12
             res[name].update({"flops_per_point_as_written": fpp, "achieved_TFLOPs": tf,
-                              "fp64_frac_measured": tf / fp64_peak})
+                              "fp64_frac_measured": tf / fp64_peak,
+                              "fp64_peak_source": FP64_PEAK_SOURCE})
+        res[name].update(fp64_from_counters(COUNTER_KEY.get(name), pts, ms, fp64_peak))
         del ins, outs
         C.cst_stencil_destroy(h)
         torch.cuda.empty_cache()
@@ -624,6 +646,12 @@ def main():
             "frac": achieved / peak, "traffic": ncu_traffic(), "peak_source": peak_src,
             "alg_bytes_per_launch": alg_bytes, "kernel": "cst_kernel (star25 sweep)",
             "avg_launch_ms": avg_launch_ms, "frac_of_nominal_8TBs": achieved / 8000.0}
+    try:
+        fp64_peak_h, _ = C.cst_fp64_peak(local)
+        roof["fp64"] = dict(fp64_from_counters("star25", pts, avg_launch_ms, fp64_peak_h),
+                            fp64_peak_TFLOPs=fp64_peak_h, fp64_peak_source=FP64_PEAK_SOURCE)
+    except Exception:
+        pass
 
     # ---- e2e: the same metric through cst_sweep_host (pinned host buffers, H2D + D2H)
     e2e = None
