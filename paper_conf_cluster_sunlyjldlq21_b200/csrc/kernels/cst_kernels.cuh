@@ -447,7 +447,7 @@ struct SGeo {
 // (consecutive blockIdx.x) are CLB consecutive b-tiles of one a-column, clusters a-major.
 // tb >= tiles_b marks a padding CTA (the grid is rounded up to whole clusters).
 __device__ __forceinline__ void stream_tile(const cst_kparams& P, int* ta, int* tb) {
-  const int tile = blockIdx.x;
+  const int tile = blockIdx.x + P.tile0;
   if constexpr (CLB > 1) {
     const int c = tile / CLB;
     *ta = c % P.tiles_a;
@@ -469,7 +469,7 @@ __device__ __forceinline__ SGeo stream_geo(const cst_kparams& P) {
   stream_tile(P, &ta, &tb);
   g.a0 = ta * TA;
   g.b0 = tb * TB;
-  g.s_start = blockIdx.y * SB;
+  g.s_start = (blockIdx.y + P.chunk0) * SB;
   g.s_end = min(g.n_s, g.s_start + SB);
   return g;
 }

@@ -81,6 +81,14 @@ struct Geometry {
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
+int launch_group() {
+  static const int v = [] {
+    const char* e = std::getenv("CST_LAUNCH_GROUP");
+    return e ? std::max(0, std::atoi(e)) : 0;
+  }();
+  return v;
+}
+
 int cluster_b() {
   static const int v = [] {
     const char* e = std::getenv("CST_CLUSTER_B");
@@ -548,6 +556,25 @@ cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* 
   P.tiles_c = g.tiles_c;
   P.chunks = g.chunks;
   void* args[] = {&P};
+  // experiment hook ($CST_LAUNCH_GROUP = n): a streaming sweep is issued as launches of at
+  // most n tiles (per chunk), so every launch is one wave whose CTAs start together and
+  // stream the planes in near lockstep (neighbours' halo rows then hit in L2)
+  const int lg = launch_group();
+  if (lg > 0 && t[F_STREAM] == 2 && g.cluster == 1) {
+    const unsigned ntile = g.grid_x;
+    for (unsigned c = 0; c < g.grid_y; ++c)
+      for (unsigned t0 = 0; t0 < ntile; t0 += (unsigned)lg) {
+        P.tile0 = (int)t0;
+        P.chunk0 = (int)c;
+        const unsigned n = std::min<unsigned>((unsigned)lg, ntile - t0);
+        st = cu_check(d->cuLaunchKernel(v->fn, n, 1, 1, g.threads, 1, 1, (unsigned)v->smem,
+                                        (CUstream)stream, args, nullptr),
+                      "cuLaunchKernel(group)");
+        if (st != CST_OK) return st;
+        ++h->last_launches;
+      }
+    return CST_OK;
+  }
   if (g.cluster > 1) {
     CUlaunchConfig cfg;
     std::memset(&cfg, 0, sizeof cfg);

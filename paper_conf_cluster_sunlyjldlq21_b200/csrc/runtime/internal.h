@@ -178,6 +178,8 @@ cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
 uint64_t jit_compile_count();
 // streaming tiles per thread-block cluster along b (experiment hook: $CST_CLUSTER_B, 1 = off)
 int cluster_b();
+// tiles per launch of a streaming sweep (experiment hook: $CST_LAUNCH_GROUP, 0 = one launch)
+int launch_group();
 std::string nvrtc_description();
 
 }  // namespace cst
