@@ -128,14 +128,18 @@ def _tune_worker(rank, world, port, outdir):
     dist.destroy_process_group()
 
 
-def test_population_parallel_tuning_equals_single_process(tmp_path):
+@pytest.mark.parametrize("world", [2, 4])
+def test_population_parallel_tuning_equals_single_process(tmp_path, world):
+    """Same seed -> the same result and report for 1, 2 and 4 evaluating ranks (SURVEY
+    8(c) GA pin: the trajectory does not depend on the number of evaluators)."""
     import test_tuner as TT
     from paper_conf_cluster_sunlyjldlq21_b200 import cst as C
-    world = 2
     mp.spawn(_tune_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
-    r0, r1 = np.load(tmp_path / "tune0.npy"), np.load(tmp_path / "tune1.npy")
-    assert np.array_equal(r0[:-1], r1[:-1])                 # every rank knows the best setting
-    assert r0[-1] > 0 and r1[-1] > 0                          # both ranks evaluated candidates
+    rs = [np.load(tmp_path / f"tune{k}.npy") for k in range(world)]
+    r0 = rs[0]
+    for r in rs[1:]:
+        assert np.array_equal(r0[:-1], r[:-1])              # every rank knows the best setting
+    assert all(r[-1] > 0 for r in rs)                         # every rank evaluated candidates
     g = C.make_grid(*TT.M, TT.R)
     h = C.cst_stencil_create(TT.KIND, TT.R, [1.0] * 7, g)
     o = C.cst_tune_opts_default()
