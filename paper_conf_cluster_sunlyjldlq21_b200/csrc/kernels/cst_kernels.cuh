@@ -34,6 +34,9 @@
 #ifndef CST_HYP_ROWS
 #define CST_HYP_ROWS 1  // TMEM hypterm: in-plane terms by row streaming
 #endif
+#ifndef CST_LGRP
+#define CST_LGRP 0  // 1: launched in groups of tiles (P.tile0 / P.chunk0 offsets; experiment)
+#endif
 #ifndef CST_CLB
 #define CST_CLB 1  // streaming tiles per thread-block cluster, stacked along b (co-scheduled
                    // b-neighbours share their halo rows in L2 while they are hot)
@@ -447,7 +450,7 @@ struct SGeo {
 // (consecutive blockIdx.x) are CLB consecutive b-tiles of one a-column, clusters a-major.
 // tb >= tiles_b marks a padding CTA (the grid is rounded up to whole clusters).
 __device__ __forceinline__ void stream_tile(const cst_kparams& P, int* ta, int* tb) {
-  const int tile = blockIdx.x + P.tile0;
+  const int tile = blockIdx.x + (CST_LGRP ? P.tile0 : 0);
   if constexpr (CLB > 1) {
     const int c = tile / CLB;
     *ta = c % P.tiles_a;
@@ -469,7 +472,7 @@ __device__ __forceinline__ SGeo stream_geo(const cst_kparams& P) {
   stream_tile(P, &ta, &tb);
   g.a0 = ta * TA;
   g.b0 = tb * TB;
-  g.s_start = (blockIdx.y + P.chunk0) * SB;
+  g.s_start = (blockIdx.y + (CST_LGRP ? P.chunk0 : 0)) * SB;
   g.s_end = min(g.n_s, g.s_start + SB);
   return g;
 }
