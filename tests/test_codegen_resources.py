@@ -48,6 +48,22 @@ CASES = [
 ]
 
 
+def _tuned(name):
+    with open(os.path.join(ROOT, "tuned", name)) as f:
+        return json.load(f)["setting"]
+
+
+# the settings bench.py times (tuned/*.json), and the fused-halo twin of the star25 one on
+# bench's configs[4] slab (its p2p line)
+CASES += [
+    (1, 4, (512, 512, 512), _tuned("star25_512.json"), False),
+    (1, 4, (1024, 1024, 256), _tuned("star25_512.json"), True),
+    (2, 1, (512, 512, 512), _tuned("box27_512.json"), False),
+    (3, 4, (512, 512, 512), _tuned("hypterm_512.json"), False),
+    (4, 2, (320, 320, 320), _tuned("rhs4_320.json"), False),
+]
+
+
 @pytest.mark.skipif(shutil.which("cuobjdump") is None, reason="cuobjdump not found")
 def test_default_and_bench_variants_have_no_stack_or_local(tmp_path):
     env = dict(os.environ, CST_CACHE_DIR=str(tmp_path))
