@@ -39,6 +39,15 @@ def main():
     ap.add_argument("--rounds", type=int, default=6)
     ap.add_argument("--heat-ms", type=float, default=1500.0)
     ap.add_argument("--burst", type=int, default=10)
+    ap.add_argument("--isolated", action="store_true",
+                    help="each setting alone: cool down --cool-s, then --heat-ms of back-to-back "
+                         "sweeps; burst = the first --burst launches, steady = launches after "
+                         "--settle-ms")
+    ap.add_argument("--cool-s", type=float, default=3.0)
+    ap.add_argument("--settle-ms", type=float, default=400.0)
+    ap.add_argument("--burst-ab", type=int, default=0,
+                    help="burst A/B: this many rounds of (0.5 s idle, 30 launches) per setting, "
+                         "settings interleaved; reports the median of the per-round medians")
     a = ap.parse_args()
     kind, r, coeffs, n, seed = tune.config(a.config)
     g = C.make_grid(*n, r)
@@ -87,6 +96,63 @@ def main():
         torch.cuda.synchronize()
         return [ev[i].elapsed_time(ev[i + 1]) for i in range(k)]
 
+    if a.burst_ab > 0:
+        pts = n[0] * n[1] * n[2]
+        bpp = 8 * (C.N_IN[kind] + C.N_OUT[kind])
+        per = {json.dumps(ov): [] for ov, _ in settings}
+        for _ in range(a.burst_ab):
+            for ov, s in settings:
+                time.sleep(0.5)
+                per[json.dumps(ov)].append(statistics.median(run(s, 30)))
+        out = {"config": a.config, "grid": list(n), "mode": "burst_ab", "rounds": a.burst_ab,
+               "base": base, "results": []}
+        for k, v in per.items():
+            m = statistics.median(v)
+            out["results"].append({"override": json.loads(k), "round_medians_ms": v,
+                                   "median_ms": m, "gstencils": pts / (m * 1e-3) / 1e9,
+                                   "alg_GBs": pts * bpp / (m * 1e-3) / 1e9})
+        print(json.dumps(out), flush=True)
+        C.cst_stencil_destroy(h)
+        return
+    if a.isolated:
+        th = threading.Thread(target=poll, daemon=True)
+        th.start()
+        t_start = time.time()
+        pts = n[0] * n[1] * n[2]
+        bpp = 8 * (C.N_IN[kind] + C.N_OUT[kind])
+        out = {"config": a.config, "grid": list(n), "mode": "isolated", "heat_ms": a.heat_ms,
+               "settle_ms": a.settle_ms, "cool_s": a.cool_s, "base": base, "results": []}
+        for ov, s in settings:
+            time.sleep(a.cool_s)
+            t0 = time.time() - t_start
+            ms, el = [], 0.0
+            while el < a.heat_ms:
+                b = run(s, 20)
+                ms += b
+                el += sum(b)
+            t1 = time.time() - t_start
+            cum, steady = 0.0, []
+            for m in ms:
+                cum += m
+                if cum >= a.settle_ms:
+                    steady.append(m)
+            t_settle = t0 + (t1 - t0) * (a.settle_ms / max(el, 1e-9))
+            cl = [c for (t, c, pw) in samples if t_settle <= t <= t1]
+            pw = [q for (t, c, q) in samples if t_settle <= t <= t1]
+            sm = statistics.mean(steady) if steady else float("nan")
+            out["results"].append({
+                "override": ov, "launches": len(ms),
+                "burst_median_ms": statistics.median(ms[:a.burst]),
+                "steady_mean_ms": sm, "steady_gstencils": pts / (sm * 1e-3) / 1e9,
+                "steady_alg_GBs": pts * bpp / (sm * 1e-3) / 1e9,
+                "steady_sm_clock_median": statistics.median(cl) if cl else None,
+                "steady_power_median_W": statistics.median(pw) if pw else None,
+                "series_ms_every_20th": [round(m, 4) for m in ms[::20]]})
+        stop.set()
+        th.join()
+        print(json.dumps(out), flush=True)
+        C.cst_stencil_destroy(h)
+        return
     res = {ov_s: {"burst": [], "sustained": [], "clock": [], "power": []}
            for ov_s in (json.dumps(ov) for ov, _ in settings)}
     th = threading.Thread(target=poll, daemon=True)
