@@ -34,13 +34,6 @@
 #ifndef CST_HYP_ROWS
 #define CST_HYP_ROWS 1  // TMEM hypterm: in-plane terms by row streaming
 #endif
-#ifndef CST_LGRP
-#define CST_LGRP 0  // 1: launched in groups of tiles (P.tile0 / P.chunk0 offsets; experiment)
-#endif
-#ifndef CST_CLB
-#define CST_CLB 1  // streaming tiles per thread-block cluster, stacked along b (co-scheduled
-                   // b-neighbours share their halo rows in L2 while they are hot)
-#endif
 
 // ------------------------------------------------------------------ configuration
 constexpr int KIND = CST_KIND;  // 1 star, 2 box, 3 hypterm, 4 rhs4center-like
@@ -57,7 +50,6 @@ constexpr int BMX = CST_BMX, BMY = CST_BMY, BMZ = CST_BMZ;
 constexpr bool RETIME = CST_RET == 2;
 constexpr int PF = CST_PF;  // pipeline stages (1 = no prefetch)
 constexpr bool QTM = CST_QSTORE == 2;
-constexpr int CLB = CST_CLB;
 
 constexpr int NIN = KIND == 3 ? 8 : (KIND == 4 ? 5 : 1);
 constexpr int NOUT = KIND == 3 ? 5 : (KIND == 4 ? 3 : 1);
@@ -446,21 +438,6 @@ struct SGeo {
   int a0, b0, s_start, s_end;
 };
 
-// tile of this CTA: a-major over (tiles_a, tiles_b); with CLB > 1 the CLB CTAs of a cluster
-// (consecutive blockIdx.x) are CLB consecutive b-tiles of one a-column, clusters a-major.
-// tb >= tiles_b marks a padding CTA (the grid is rounded up to whole clusters).
-__device__ __forceinline__ void stream_tile(const cst_kparams& P, int* ta, int* tb) {
-  const int tile = blockIdx.x + (CST_LGRP ? P.tile0 : 0);
-  if constexpr (CLB > 1) {
-    const int c = tile / CLB;
-    *ta = c % P.tiles_a;
-    *tb = (c / P.tiles_a) * CLB + tile % CLB;
-  } else {
-    *ta = tile % P.tiles_a;
-    *tb = tile / P.tiles_a;
-  }
-}
-
 __device__ __forceinline__ SGeo stream_geo(const cst_kparams& P) {
   SGeo g;
   g.n_a = P.nx;
@@ -468,11 +445,10 @@ __device__ __forceinline__ SGeo stream_geo(const cst_kparams& P) {
   g.n_s = SZ ? P.nz : P.ny;
   g.st_b = SZ ? P.py : P.pz;
   g.st_s = SZ ? P.pz : P.py;
-  int ta, tb;
-  stream_tile(P, &ta, &tb);
-  g.a0 = ta * TA;
-  g.b0 = tb * TB;
-  g.s_start = (blockIdx.y + (CST_LGRP ? P.chunk0 : 0)) * SB;
+  const int tile = blockIdx.x;
+  g.a0 = (tile % P.tiles_a) * TA;
+  g.b0 = (tile / P.tiles_a) * TB;
+  g.s_start = blockIdx.y * SB;
   g.s_end = min(g.n_s, g.s_start + SB);
   return g;
 }
@@ -2396,11 +2372,6 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 #endif
 extern "C" __global__ void CST_LB cst_kernel(const __grid_constant__ cst_kparams P) {
   extern __shared__ __align__(128) double cst_smem[];
-  if constexpr (STREAM && CLB > 1) {  // padding CTA of the last cluster row: nothing to do
-    int ta, tb;
-    stream_tile(P, &ta, &tb);
-    if (tb >= P.tiles_b) return;
-  }
   if constexpr (BT > 1) {
     kernel_tblock<0>(P, cst_smem);
   } else if constexpr (!STREAM) {

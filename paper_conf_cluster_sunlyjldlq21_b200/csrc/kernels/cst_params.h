@@ -26,7 +26,6 @@ struct __attribute__((aligned(64))) cst_kparams {
   int tiles_a, tiles_b;              // CTA tiles over the two non-streamed dims (or x,y)
   int tiles_c;                       // third tile dim (non-streaming z tiles)
   int chunks;                        // streaming chunks (SB)
-  int tile0, chunk0;                 // streaming: offsets of blockIdx.x / .y (launch groups)
   int remote;                        // 1: every store also goes to rout[q] + same offset
   double* rout[CST_MAX_OUT];         // peer-mapped neighbour halo (fused z-slab exchange)
 };

@@ -54,7 +54,6 @@ cst_status driver(const Driver** out) {
               get("cuFuncSetAttribute", (void**)&d.cuFuncSetAttribute) &&
               get("cuFuncGetAttribute", (void**)&d.cuFuncGetAttribute) &&
               get("cuLaunchKernel", (void**)&d.cuLaunchKernel) &&
-              get("cuLaunchKernelEx", (void**)&d.cuLaunchKernelEx) &&
               get("cuTensorMapEncodeTiled", (void**)&d.cuTensorMapEncodeTiled) &&
               get("cuOccupancyMaxActiveBlocksPerMultiprocessor", (void**)&d.cuOccupancy) &&
               get("cuGetErrorString", (void**)&d.cuGetErrorString) &&
@@ -75,28 +74,10 @@ cst_status driver(const Driver** out) {
 struct Geometry {
   unsigned grid_x, grid_y, threads;
   int tiles_a, tiles_b, tiles_c, chunks;
-  int cluster = 1;  // CTAs per cluster along blockIdx.x (streaming: b-stacked tiles)
   int box[3];  // TMA box dims (x, y, z)
 };
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
-
-int launch_group() {
-  static const int v = [] {
-    const char* e = std::getenv("CST_LAUNCH_GROUP");
-    return e ? std::max(0, std::atoi(e)) : 0;
-  }();
-  return v;
-}
-
-int cluster_b() {
-  static const int v = [] {
-    const char* e = std::getenv("CST_CLUSTER_B");
-    const int c = e ? std::atoi(e) : 1;
-    return (c == 2 || c == 4 || c == 8) ? c : 1;
-  }();
-  return v;
-}
 
 static Geometry geometry(const StencilInfo& st, const Tuple& t, int64_t nx, int64_t ny,
                          int64_t nz) {
@@ -112,8 +93,7 @@ static Geometry geometry(const StencilInfo& st, const Tuple& t, int64_t nx, int6
     g.tiles_b = (int)cdiv(sz ? ny : nz, sz ? T[1] : T[2]);
     g.chunks = (int)cdiv(sz ? nz : ny, t[F_SB]);
     g.tiles_c = 1;
-    g.cluster = cluster_b();
-    g.grid_x = (unsigned)(g.tiles_a * ((g.tiles_b + g.cluster - 1) / g.cluster * (int64_t)g.cluster));
+    g.grid_x = (unsigned)(g.tiles_a * (int64_t)g.tiles_b);
     g.grid_y = (unsigned)g.chunks;
     g.box[0] = (int)T[0] + 2 * xr;
     if (t[F_BT] > 1) {  // temporally blocked: the input box carries bt halos per side
@@ -556,48 +536,9 @@ cst_status cst_launch_range(cst_stencil* h, const cst_setting* s, const double* 
   P.tiles_c = g.tiles_c;
   P.chunks = g.chunks;
   void* args[] = {&P};
-  // experiment hook ($CST_LAUNCH_GROUP = n): a streaming sweep is issued as launches of at
-  // most n tiles (per chunk), so every launch is one wave whose CTAs start together and
-  // stream the planes in near lockstep (neighbours' halo rows then hit in L2)
-  const int lg = launch_group();
-  if (lg > 0 && t[F_STREAM] == 2 && g.cluster == 1) {
-    const unsigned ntile = g.grid_x;
-    for (unsigned c = 0; c < g.grid_y; ++c)
-      for (unsigned t0 = 0; t0 < ntile; t0 += (unsigned)lg) {
-        P.tile0 = (int)t0;
-        P.chunk0 = (int)c;
-        const unsigned n = std::min<unsigned>((unsigned)lg, ntile - t0);
-        st = cu_check(d->cuLaunchKernel(v->fn, n, 1, 1, g.threads, 1, 1, (unsigned)v->smem,
-                                        (CUstream)stream, args, nullptr),
-                      "cuLaunchKernel(group)");
-        if (st != CST_OK) return st;
-        ++h->last_launches;
-      }
-    return CST_OK;
-  }
-  if (g.cluster > 1) {
-    CUlaunchConfig cfg;
-    std::memset(&cfg, 0, sizeof cfg);
-    cfg.gridDimX = g.grid_x;
-    cfg.gridDimY = g.grid_y;
-    cfg.gridDimZ = 1;
-    cfg.blockDimX = g.threads;
-    cfg.blockDimY = cfg.blockDimZ = 1;
-    cfg.sharedMemBytes = (unsigned)v->smem;
-    cfg.hStream = (CUstream)stream;
-    CUlaunchAttribute at;
-    std::memset(&at, 0, sizeof at);
-    at.id = CU_LAUNCH_ATTRIBUTE_CLUSTER_DIMENSION;
-    at.value.clusterDim.x = (unsigned)g.cluster;
-    at.value.clusterDim.y = at.value.clusterDim.z = 1;
-    cfg.attrs = &at;
-    cfg.numAttrs = 1;
-    st = cu_check(d->cuLaunchKernelEx(&cfg, v->fn, args, nullptr), "cuLaunchKernelEx(cluster)");
-  } else {
-    st = cu_check(d->cuLaunchKernel(v->fn, g.grid_x, g.grid_y, 1, g.threads, 1, 1,
-                                    (unsigned)v->smem, (CUstream)stream, args, nullptr),
-                  "cuLaunchKernel");
-  }
+  st = cu_check(d->cuLaunchKernel(v->fn, g.grid_x, g.grid_y, 1, g.threads, 1, 1,
+                                  (unsigned)v->smem, (CUstream)stream, args, nullptr),
+                "cuLaunchKernel");
   if (st != CST_OK) return st;
   ++h->last_launches;
   return CST_OK;

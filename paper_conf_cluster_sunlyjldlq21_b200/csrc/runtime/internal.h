@@ -149,7 +149,6 @@ struct Driver {
   PFN_cuFuncSetAttribute_v9000 cuFuncSetAttribute = nullptr;
   PFN_cuFuncGetAttribute_v2020 cuFuncGetAttribute = nullptr;
   PFN_cuLaunchKernel_v4000 cuLaunchKernel = nullptr;
-  PFN_cuLaunchKernelEx_v11060 cuLaunchKernelEx = nullptr;
   PFN_cuTensorMapEncodeTiled_v12000 cuTensorMapEncodeTiled = nullptr;
   PFN_cuOccupancyMaxActiveBlocksPerMultiprocessor_v6050 cuOccupancy = nullptr;
   PFN_cuGetErrorString_v6000 cuGetErrorString = nullptr;
@@ -176,10 +175,6 @@ cst_status jit_cubin(const StencilInfo& st, const Tuple& t, std::string* cubin,
                      double* compile_s,
                      bool remote = false);
 uint64_t jit_compile_count();
-// streaming tiles per thread-block cluster along b (experiment hook: $CST_CLUSTER_B, 1 = off)
-int cluster_b();
-// tiles per launch of a streaming sweep (experiment hook: $CST_LAUNCH_GROUP, 0 = one launch)
-int launch_group();
 std::string nvrtc_description();
 
 }  // namespace cst

@@ -121,8 +121,6 @@ static std::string prefix_for(const StencilInfo& st, const Tuple& t, bool remote
   std::ostringstream o;
   o << "#define CST_KIND " << st.kind << "\n#define CST_R " << st.r << "\n";
   if (remote) o << "#define CST_REMOTE 1\n";
-  if (t[F_STREAM] == 2 && cluster_b() > 1) o << "#define CST_CLB " << cluster_b() << "\n";
-  if (t[F_STREAM] == 2 && launch_group() > 0) o << "#define CST_LGRP 1\n";
   static const char* names[F_COUNT] = {"TBX", "TBY", "TBZ", "STAGING", "CONST", "STREAM",
                                        "SD",  "SB",  "UFX", "UFY",     "UFZ",   "CMX",
                                        "CMY", "CMZ", "BMX", "BMY",     "BMZ",   "RET",
