@@ -579,6 +579,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-other-configs", action="store_true")
+    ap.add_argument("--sustained-s", type=float, default=1.5,
+                    help="seconds of extra sweeps after the timed region for the steady-state "
+                         "(power-capped) line; 0 = skip")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -653,6 +656,37 @@ def main():
     except Exception:
         pass
 
+    # ---- steady state: after the timed region, keep sweeping for ~1.5 s and time the
+    # launches after the first 0.5 s — the board's 1000 W power cap has then lowered the SM
+    # clock (burst vs power-capped regimes); reported beside the headline
+    sustained = None
+    if args.sustained_s > 0:
+        cs = ClockSampler(local)
+        cs.start()
+        blk, times, t_el = 50, [], 0.0
+        while t_el < args.sustained_s * 1e3:
+            ev2 = [torch.cuda.Event(enable_timing=True) for _ in range(blk + 1)]
+            ev2[0].record(stream)
+            for i in range(blk):
+                step()
+                ev2[i + 1].record(stream)
+            torch.cuda.synchronize()
+            b = [ev2[i].elapsed_time(ev2[i + 1]) for i in range(blk)]
+            times += b
+            t_el += sum(b)
+        ck = cs.stop()
+        cum, steady = 0.0, []
+        for m in times:
+            cum += m
+            if cum >= args.sustained_s * 1e3 / 3:
+                steady.append(m)
+        sm = statistics.mean(steady)
+        sustained = {"ms_per_step": sm, "value": pts / (sm * 1e-3) / 1e9, "unit": UNIT,
+                     "hbm_frac": alg_bytes / (sm * 1e-3) / 1e9 / peak, "launches": len(times),
+                     "window": f"launches after the first {args.sustained_s / 3:.2f} s of "
+                               f"{args.sustained_s:.1f} s of back-to-back sweeps",
+                     "clocks": ck}
+
     # ---- e2e: the same metric through cst_sweep_host (pinned host buffers, H2D + D2H)
     e2e = None
     if args.e2e_steps > 0:
@@ -703,6 +737,7 @@ def main():
                                  % (grid.numel * 8 / 1e9),
                            "parallelism": "single GPU"},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
+                "sustained": sustained,
                 "other_configs": others,
                 "gpu_launches": launches,
                 "per_step_ms": {"min": min(per), "median": statistics.median(per), "max": max(per),
