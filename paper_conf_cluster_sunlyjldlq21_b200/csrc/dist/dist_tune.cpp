@@ -58,6 +58,7 @@ struct Comm {
     return CST_OK;
   }
   cst_status bcast(void* buf, int64_t bytes) {
+    if (D->nranks == 1) return CST_OK;
     if (D->has_coll) {
       if (D->coll.bcast(D->coll.user, buf, bytes, 0) != 0)
         return fail(CST_E_INTERNAL, "cst_dist_tune: broadcast callback failed");
@@ -78,6 +79,10 @@ struct Comm {
 #endif
   }
   cst_status allgather(const void* send, void* recv, int64_t bytes) {
+    if (D->nranks == 1) {
+      std::memcpy(recv, send, (size_t)bytes);
+      return CST_OK;
+    }
     if (D->has_coll) {
       if (D->coll.allgather(D->coll.user, send, recv, bytes) != 0)
         return fail(CST_E_INTERNAL, "cst_dist_tune: all-gather callback failed");
@@ -240,10 +245,10 @@ extern "C" cst_status cst_dist_tune(cst_dist* D, const cst_tune_opts* o, const d
   if (D->nranks > 1 && !D->has_coll && !have_nccl)
     return fail(CST_E_UNSUPPORTED, "cst_dist_tune needs the NCCL transport (a handle created "
                                    "with an nccl_unique_id) or cst_dist_create_host collectives");
+  if (!D->has_coll || !local_eval) CST_CUDA(cudaSetDevice(D->h->device));  // NCCL staging / timing
   Comm comm{D};
   Server srv{D, &comm, o, in, scratch_out, local_eval, local_user};
   if (!local_eval) {
-    CST_CUDA(cudaSetDevice(D->h->device));
     CST_CUDA(cudaStreamCreateWithFlags(&srv.stream, cudaStreamNonBlocking));
   }
   struct StreamGuard {

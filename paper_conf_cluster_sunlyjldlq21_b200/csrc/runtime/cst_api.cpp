@@ -692,7 +692,9 @@ extern "C" cst_status cst_sweep_host(cst_stencil* h, const cst_setting* s,
       CST_CUDA(cudaStreamCreateWithFlags(&h->host_in_stream, cudaStreamNonBlocking));
       CST_CUDA(cudaStreamCreateWithFlags(&h->host_out_stream, cudaStreamNonBlocking));
     }
-    const int64_t nc = std::max<int64_t>(1, std::min<int64_t>(8, G.nz / std::max(16, 4 * h->info.r)));
+    int64_t ncmax = 8;
+    if (const char* e = std::getenv("CST_HOST_CHUNKS")) ncmax = std::max(1, std::atoi(e));  // tmp
+    const int64_t nc = std::max<int64_t>(1, std::min<int64_t>(ncmax, G.nz / std::max(16, 4 * h->info.r)));
     std::vector<cudaEvent_t> evs;
     auto event = [&](cudaStream_t st_) -> cudaEvent_t {
       cudaEvent_t e;
