@@ -692,9 +692,9 @@ extern "C" cst_status cst_sweep_host(cst_stencil* h, const cst_setting* s,
       CST_CUDA(cudaStreamCreateWithFlags(&h->host_in_stream, cudaStreamNonBlocking));
       CST_CUDA(cudaStreamCreateWithFlags(&h->host_out_stream, cudaStreamNonBlocking));
     }
-    int64_t ncmax = 8;
-    if (const char* e = std::getenv("CST_HOST_CHUNKS")) ncmax = std::max(1, std::atoi(e));  // tmp
-    const int64_t nc = std::max<int64_t>(1, std::min<int64_t>(ncmax, G.nz / std::max(16, 4 * h->info.r)));
+    // 16 chunks: 28 ms for star25 512^3 vs 30 ms with 8 on B200 (PCIe ~55 GB/s per
+    // direction, ~45 GB/s each when both run; tools/e2e_probe.py)
+    const int64_t nc = std::max<int64_t>(1, std::min<int64_t>(16, G.nz / std::max(16, 4 * h->info.r)));
     std::vector<cudaEvent_t> evs;
     auto event = [&](cudaStream_t st_) -> cudaEvent_t {
       cudaEvent_t e;
