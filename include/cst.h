@@ -245,6 +245,10 @@ typedef struct {
                                 cv_threshold as given                                */
   int32_t filter_threads;    /* host threads streaming the whole valid space through
                                 the PMNF threshold filter (0 = all cores)             */
+  int32_t cool_ms;           /* 30: idle ms before each built-in timing, so every
+                                candidate is timed in the same (boost-clock) power
+                                state instead of later ones under the board's power
+                                cap                                   */
 } cst_tune_opts;
 
 typedef struct {

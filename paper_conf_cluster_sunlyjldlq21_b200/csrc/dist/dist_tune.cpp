@@ -13,6 +13,7 @@
 //   gather   per rank n x double ms (NaN = not mine) + n x n_user_metrics doubles
 //   result   Result (status, best setting, report, error text)
 #include <atomic>
+#include <chrono>
 #include <cmath>
 #include <cstring>
 #include <thread>
@@ -152,6 +153,7 @@ struct Server {
       for (size_t i = 0; i < sub.size(); ++i) {
         if (check_rules(h->info, to_tuple(sub[i])) != nullptr) continue;
         double m = INFINITY;
+        if (o->cool_ms > 0) std::this_thread::sleep_for(std::chrono::milliseconds(o->cool_ms));
         if (cst_time_setting(h, &sub[i], in, out, 1, o->warmup, std::max(1, o->reps), stream,
                              &m) == CST_OK)
           sms[i] = m;

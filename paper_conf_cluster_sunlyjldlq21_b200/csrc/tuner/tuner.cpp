@@ -397,6 +397,7 @@ extern "C" void cst_tune_opts_default(cst_tune_opts* o) {
   o->nsteps = 1;
   o->noise_reps = 8;
   o->filter_threads = 0;
+  o->cool_ms = 30;
 }
 
 namespace {
@@ -442,6 +443,20 @@ struct Evaluator {
     return t;
   }
 
+  // idle before a built-in timing so every candidate starts from the same power state:
+  // max(cool_ms, the previous timing's wall time), i.e. a duty cycle of at most 1/2
+  mutable std::chrono::steady_clock::time_point t_cool{};
+  void cool() const {
+    if (o->cool_ms <= 0) return;
+    const auto now = std::chrono::steady_clock::now();
+    double busy_ms = 0;
+    if (t_cool.time_since_epoch().count() != 0)
+      busy_ms = std::chrono::duration<double, std::milli>(now - t_cool).count();
+    const double ms = std::max<double>(o->cool_ms, std::min(busy_ms, 100.0));
+    std::this_thread::sleep_for(std::chrono::microseconds((int64_t)(ms * 1e3)));
+    t_cool = std::chrono::steady_clock::now();
+  }
+
   // timing noise (Q18): n independent re-evaluations of one setting, bypassing
   // the memo; returns their fitness values
   cst_status repeat(const Tuple& t0, int n, std::vector<double>* fit) {
@@ -460,6 +475,7 @@ struct Evaluator {
       if (o->nsteps > 1) return CST_OK;  // multi-step timing copies its input: skip
       for (int i = 0; i < n; ++i) {
         double m = INFINITY;
+        cool();
         const cst_status st = cst_time_setting(h, &ss[i], in, out, 1, o->warmup,
                                                std::max(1, o->reps), stream, &m);
         if (st == CST_E_CUDA) return st;
@@ -522,6 +538,7 @@ struct Evaluator {
         for (size_t i = 0; i < ss.size(); ++i) {
           double m = INFINITY;
           cst_status st;
+          cool();
           if (nsteps > 1) {
             // fresh copy of the input for every candidate (values stay bounded)
             CST_CUDA(cudaMemcpyAsync(tin, in[0], numel * 8, cudaMemcpyDeviceToDevice, stream));

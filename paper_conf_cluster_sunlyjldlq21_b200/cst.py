@@ -119,7 +119,7 @@ class cst_tune_opts(ctypes.Structure):
                 ("n_user_metrics", ctypes.c_int32), ("quantile_sample", ctypes.c_int32),
                 ("warm_start", ctypes.c_int32), ("metrics_mode", ctypes.c_int32),
                 ("nsteps", ctypes.c_int32), ("noise_reps", ctypes.c_int32),
-                ("filter_threads", ctypes.c_int32)]
+                ("filter_threads", ctypes.c_int32), ("cool_ms", ctypes.c_int32)]
 
 
 class cst_tune_report(ctypes.Structure):
