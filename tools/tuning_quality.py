@@ -60,13 +60,15 @@ def subspace(h):
     return out
 
 
-def time_all(h, settings, u, v, reps=5):
-    """Parallel NVRTC code generation, then serial CUDA-event timing (like cst_tune)."""
+def time_all(h, settings, u, v, reps=5, cool_ms=30):
+    """Parallel NVRTC code generation, then serial CUDA-event timing with the tuner's idle
+    before each timing (cst_tune_opts.cool_ms: every setting timed in the same power state)."""
     with cf.ThreadPoolExecutor(16) as ex:
         list(ex.map(lambda s: _compile(h, s), settings))
     res = []
     stream = torch.cuda.current_stream().cuda_stream
     for s in settings:
+        time.sleep(cool_ms / 1e3)
         try:
             ms = C.cst_time_setting(h, s, [u.data_ptr()], [v.data_ptr()], 2, reps, stream)
         except C.CstError:
