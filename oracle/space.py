@@ -39,7 +39,8 @@ BM_x, BM_y <= 2, every UF = 1 (reading Q23); R15 qstore = 2 only 
 TMEM path: star or hypterm (hypterm: one point along x, BM_b <= 2 along the other in-plane
 dim, no cyclic merging), streaming with T_SD = 1, TMA staging, retimed, bt = 1, and
 ceil(threads/128) * points per thread * (4r star, 20r hypterm) <= 512 TMEM columns;
-R16 rhs4: use_retiming = 1 (its kernels have one summation form).  R6/R9/R16 keep every
+R16 rhs4: use_retiming = 2 only for the retimed column walk (r4ret_path: streaming with
+T_SD = 1, TMA, bt = 1, qstore 1, CM = 1, BM_b = 1, BM_x <= 2).  R6/R9/R16 keep every
 field a kernel path does not read at its canonical value (round 2; tools/knob_audit.py).
 """
 from __future__ import annotations
@@ -101,6 +102,22 @@ def tb_blocks_per_thread(r: int, s: dict, level: int) -> int:
     return -(-((ex // s["bm_x"]) * (ey // s["bm_y"])) // nthr)
 
 
+def r4ret_path(kind: int, s: dict) -> bool:
+    """R16: the setting selects rhs4's retimed column walk (use_retiming = 2): streaming with
+    T_SD = 1, TMA staging, bt = 1, registers (qstore 1), no cyclic merging, one point along
+    the in-plane non-x dim b, BM_x <= 2."""
+    if kind != RHS4 or s["use_retiming"] != 2:
+        return False
+    if not (s["use_streaming"] == 2 and s["staging"] == 3 and s["bt"] == 1
+            and s["qstore"] == 1):
+        return False
+    sd = "xyz"[s["sd"] - 1]
+    b = "y" if sd == "z" else "z"
+    if any(s["cm_" + d] != 1 for d in "xyz"):
+        return False
+    return s["tb_" + sd] == 1 and s["bm_" + sd] == 1 and s["bm_" + b] == 1 and s["bm_x"] <= 2
+
+
 def plane_geometry(kind: int, r: int, s: dict):
     """(in-plane elements P, ring planes NP) of the smem staging for a streaming setting;
     (box elements, 1) for a non-streaming one."""
@@ -111,7 +128,9 @@ def plane_geometry(kind: int, r: int, s: dict):
     a, b = [d for d in range(3) if d != sd]
     P = (T[a] + 2 * r) * (T[b] + 2 * r)
     D = s["prefetch"]
-    if T[sd] == 1:
+    if T[sd] == 1 and r4ret_path(kind, s):
+        NP = D + 2 * r          # planes c-2 .. c+2 + prefetch (+ 6 product planes, smem_bytes)
+    elif T[sd] == 1:
         NP = D + (0 if s["use_retiming"] == 2 else retention(kind, r))
     else:
         NP = D * T[sd] + 2 * r
@@ -129,7 +148,7 @@ def smem_bytes(kind: int, r: int, s: dict) -> int:
         return s["prefetch"] * rnd(e0[0] * e0[1]) + (s["bt"] - 1) * 2 * rnd(e1[0] * e1[1])
     P, NP = plane_geometry(kind, r, s)
     plane = -(-(P * 8) // 128) * 128
-    return n_arrays(kind) * NP * plane
+    return (n_arrays(kind) * NP + (6 if r4ret_path(kind, s) else 0)) * plane
 
 
 def points_per_thread(s: dict) -> int:
@@ -171,6 +190,10 @@ def est_regs(kind: int, r: int, s: dict) -> int:
     if s["qstore"] == 2:
         # in-plane part + centre per point, one point's ring, the block's column windows
         return 32 + 2 * (2 * points_per_thread(s) + (r + 1) + 2 * r)
+    if r4ret_path(kind, s):
+        # s-window queue (5 arrays x 5 planes; 3 arrays when BM_x = 2), 5 x 3 pending
+        # outputs, ~20 operands in flight, per point
+        return 32 + 2 * s["bm_x"] * (60 if s["bm_x"] == 1 else 50)
     if s["bt"] > 1:
         # 2r+1 rotating accumulators per point of every level + one operand window
         pts = sum(tb_blocks_per_thread(r, s, lv) for lv in range(1, s["bt"] + 1))
@@ -205,6 +228,8 @@ def uf_trip(kind: int, s: dict, d: int) -> int:
     if s["use_streaming"] == 1:
         return bmcm
     sd = s["sd"] - 1
+    if r4ret_path(kind, s):
+        return 1        # rhs4 retimed: the x pair runs in lockstep, the plane loop stays rolled
     if not (kind in (STAR, BOX, HYPTERM) and tiles(s)[sd] == 1):
         return bmcm
     if d != sd:
@@ -262,7 +287,7 @@ def check(kind: int, r: int, M, s: dict):
         return "R14"
     if s["qstore"] == 2 and not qs_path_ok(kind, r, s):
         return "R15"
-    if kind == RHS4 and s["use_retiming"] != 1:
+    if kind == RHS4 and s["use_retiming"] == 2 and not r4ret_path(kind, s):
         return "R16"
     if smem_bytes(kind, r, s) > SMEM_LIMIT:
         return "R10"

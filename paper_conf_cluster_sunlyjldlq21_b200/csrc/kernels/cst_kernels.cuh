@@ -1497,6 +1497,268 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
 }
 
 // =============================================================================
+// rhs4center-like, retimed column walk (NEXT-1; use_retiming = 2 with T_SD = 1, TMA,
+// CM = 1, BM_b = 1, BM_a <= 2).  Retiming applied to the operator of
+// reading O7: every mixed term D_o[c D_n f] is split by where its two derivatives point.
+//   outer along s (D_s[mu D_a u_s], D_s[mu D_b u_s], D_s[la D_a u_a], D_s[la D_b u_b]):
+//     the inner product P = c D_n f is formed once per plane at the point's own column (its
+//     operands are the in-plane windows the V terms load anyway) and scattered into the
+//     pending outputs c-2, c-1, c+1, c+2 with the outer weights (-1, 8, -8, 1);
+//   inner along s (D_a[la D_s u_s], D_b[la D_s u_s], D_a[mu D_s u_a], D_b[mu D_s u_b]):
+//     the products Q = c D_s f of plane c are formed once per column from the s-window and
+//     staged as three product planes in shared memory (own columns by their threads, the
+//     cross-shaped halo columns from the ring), then differenced along a / b;
+//   both derivatives in-plane: gathered from the ring plane as in the generic path.
+// The s-window of the own column (u1..u3, mu, lambda at planes c-2..c+2) is a register
+// queue (2.5-D blocking).  At step c the newest plane is c+2; output c-2 completes.
+// =============================================================================
+constexpr bool R4RET = KIND == 4 && STREAM && TS == 1 && RETIME;
+constexpr int R4NP = PF + 2 * R;                 // ring: planes c-2 .. c+2 + PF-1 ahead
+constexpr int R4NH = 2 * TB + 4 * (TA / 2);      // halo column pairs of the product planes
+// the two x-adjacent points of a BM_a = 2 thread in lockstep (every smem operand one 16-B
+// load for both); mu / lambda s-windows then come from the ring instead of registers
+#ifndef CST_R4Q
+#define CST_R4Q (BMA == 1 ? 3 : 0)
+#endif
+constexpr int R4Q = CST_R4Q;  // arrays of the s-window kept in the register queue
+
+template <class T>
+__device__ __forceinline__ T r4_row(const double* row, int da) {
+  if constexpr (sizeof(T) == 8) {
+    return row[da];
+  } else {
+    if ((da & 1) == 0) {
+      const double2 v = *reinterpret_cast<const double2*>(row + da);
+      return T{v.x, v.y};
+    }
+    const double2 lo = *reinterpret_cast<const double2*>(row + da - 1);
+    const double2 hi = *reinterpret_cast<const double2*>(row + da + 1);
+    return T{lo.y, hi.x};
+  }
+}
+template <class T>
+__device__ __forceinline__ void r4_put_row(double* row, T v) {
+  if constexpr (sizeof(T) == 8) row[0] = v;
+  else *reinterpret_cast<double2*>(row) = make_double2(v.x, v.y);
+}
+__device__ __forceinline__ double r4_lane(double v, int) { return v; }
+__device__ __forceinline__ double r4_lane(dpair v, int h) { return h ? v.y : v.x; }
+
+// V_d[a](f) of reading O7, unscaled (the 1/6 and s_d^2 are in coefficient 3 + d)
+template <class T, class A, class F>
+__device__ __forceinline__ T r4_v(const A& a, const F& f) {
+  const T am2 = a(-2), am1 = a(-1), a0 = a(0), ap1 = a(1), ap2 = a(2);
+  const T m1 = fma(-0.75, a0 + am2, am1);
+  const T m2 = fma(3.0, a0 + am1, am2 + ap1);
+  const T m3 = fma(3.0, ap1 + a0, am1 + ap2);
+  const T m4 = fma(-0.75, a0 + ap2, ap1);
+  const T f0 = f(0);
+  T v = m1 * (f(-2) - f0);
+  v = fma(m2, f(-1) - f0, v);
+  v = fma(m3, f(1) - f0, v);
+  v = fma(m4, f(2) - f0, v);
+  return v;
+}
+// unscaled D'[f] = 8 (f(+1) - f(-1)) + (f(-2) - f(+2))  (the 1/12 factors are folded)
+template <class T, class F>
+__device__ __forceinline__ T r4_d(const F& f) {
+  return fma(8.0, f(1) - f(-1), f(-2) - f(2));
+}
+
+template <int DUMMY>
+__device__ __forceinline__ void kernel_rhs4_ret(const cst_kparams& P, double* smem) {
+  using T = typename Cond<BMA == 2, dpair, double>::type;
+  static_assert(STAGING == 3 && BMA <= 2 && NCB == 1 && CMA == 1, "R16: rhs4 retimed path");
+  Ctx C{P};
+  constexpr int NP = R4NP;
+  constexpr int QN = 5;  // s-window / pending outputs: planes c-2 .. c+2
+  const SGeo g = stream_geo(P);
+  const int tid = threadIdx.x;
+  const int la = thread_x() * BMA;
+  const int lb = SZ ? thread_y() : thread_z();
+  const int n_out = g.s_end - g.s_start;
+  const int n_planes = n_out + 2 * R;
+  double* qbuf = smem + NP * RSLOT;  // 2 buffers x {la*D_s u_s, mu*D_s u_a, mu*D_s u_b}
+  u64* bars = (u64*)(qbuf + 6 * SLOT);
+  const int own = (lb + R) * PA + la + XR;  // the point's element in a plane slot
+  auto slot = [&](int j) { return smem + (j % NP) * RSLOT; };
+  const double kv[3] = {C.coef(3), C.coef(4), C.coef(5)};
+  auto wp = [&](int d, int i) { return C.coef(6 + d + i - 1); };  // s_d s_i / 144, d != i
+
+  if (tid == 0) {
+    for (int s = 0; s < NP; ++s) mbar_init(&bars[s], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (tid == 0) {
+    for (int j = 0; j < NP && j < n_planes; ++j) {
+      mbar_arrive_expect_tx(&bars[j], TX_BYTES);
+      tma_plane(P, g, slot(j), &bars[j], g.s_start - R + j);
+    }
+  }
+
+  // queue q[arr][phys]: logical k (plane c-2+k) at phys (k + u) % 5 in phase u = c % 5
+  constexpr int NQA = R4Q;
+  T q[NQA > 0 ? NQA : 1][QN];
+  T acc[3][QN];  // pending outputs, same rotation; index = physical output direction
+#pragma unroll
+  for (int m = 0; m < QN; ++m) {
+#pragma unroll
+    for (int i = 0; i < 3; ++i) acc[i][m] = T{};
+#pragma unroll
+    for (int a = 0; a < NQA; ++a) q[a][m] = T{};
+  }
+  // prologue: planes 0 and 1 are logical 2 and 3 of step 0
+  for (int j = 0; j < 2 && j < n_planes; ++j) {
+    mbar_wait(&bars[j], 0u);
+#pragma unroll
+    for (int a = 0; a < NQA; ++a) q[a][2 + j] = r4_row<T>(slot(j) + a * SLOT + own, 0);
+  }
+
+  const long long col = (long long)(g.a0 + la) + (long long)(g.b0 + lb) * g.st_b;
+  const bool in_b = g.b0 + lb < g.n_b;
+  const bool in_a0 = g.a0 + la < g.n_a, in_a1 = BMA == 2 && g.a0 + la + 1 < g.n_a;
+
+  for (int j0 = 0; j0 < n_planes; j0 += QN) {
+    static_for<0, QN>([&](auto UU) {
+      constexpr int u = decltype(UU)::value;
+      auto ph = [](int k) { return (k + u) % QN; };
+      const int c = j0 + u;  // centre plane (sequence index)
+      if (c >= n_planes) return;  // CTA-uniform
+      const bool real = c >= R && c < R + n_out;
+      // ---- newest plane c+2 -> queue
+      if (c + 2 < n_planes) {
+        mbar_wait(&bars[(c + 2) % NP], (u32)(((c + 2) / NP) & 1));
+#pragma unroll
+        for (int a = 0; a < NQA; ++a) q[a][ph(4)] = r4_row<T>(slot(c + 2) + a * SLOT + own, 0);
+      }
+      // s-window of array a at the own column, offset k in -2..2
+      auto sw = [&](int a, int k) -> T {
+        if (a < NQA) return q[a][ph(2 + k)];
+        return r4_row<T>(slot(c + k) + a * SLOT + own, 0);
+      };
+      double* qb = qbuf + (c & 1) * 3 * SLOT;
+      if (real) {
+        // ---- V_s and the inner-s products of the own column
+        const T mu0 = sw(3, 0), la0 = sw(4, 0);
+#pragma unroll
+        for (int i = 0; i < 3; ++i) {
+          const T v = r4_v<T>(
+              [&](int k) { return i == DS ? fma(2.0, sw(3, k), sw(4, k)) : sw(3, k); },
+              [&](int k) { return sw(i, k); });
+          acc[i][ph(2)] = fma(kv[DS], v, acc[i][ph(2)]);
+        }
+        r4_put_row<T>(qb + 0 * SLOT + own, la0 * r4_d<T>([&](int k) { return sw(DS, k); }));
+        r4_put_row<T>(qb + 1 * SLOT + own, mu0 * r4_d<T>([&](int k) { return sw(DA, k); }));
+        r4_put_row<T>(qb + 2 * SLOT + own, mu0 * r4_d<T>([&](int k) { return sw(DB, k); }));
+        // ---- halo columns of the product planes (pairs of x-adjacent columns):
+        // a-strips (la*D_s u_s, mu*D_s u_a), b-strips (la*D_s u_s, mu*D_s u_b)
+        for (int e = tid; e < R4NH; e += NTHR) {
+          int ha, hb, fa;
+          if (e < 2 * TB) {
+            ha = (e & 1) ? TA : -2;
+            hb = e >> 1;
+            fa = DA;
+          } else {
+            const int f = e - 2 * TB;
+            ha = 2 * (f % (TA / 2));
+            const int rr = f / (TA / 2);  // 0..3 -> rows -2, -1, TB, TB+1
+            hb = rr < 2 ? rr - 2 : TB + rr - 2;
+            fa = DB;
+          }
+          const int ho = (hb + R) * PA + ha + XR;
+          auto hw = [&](int a, int k) { return r4_row<dpair>(slot(c + k) + a * SLOT + ho, 0); };
+          const dpair hmu = hw(3, 0), hla = hw(4, 0);
+          r4_put_row<dpair>(qb + ho, hla * r4_d<dpair>([&](int k) { return hw(DS, k); }));
+          const dpair pf = hmu * r4_d<dpair>([&](int k) { return hw(fa, k); });
+          r4_put_row<dpair>(qb + (fa == DA ? 1 : 2) * SLOT + ho, pf);
+        }
+      }
+      __syncthreads();
+      // ---- the slot of plane c-2 is free: refill it with plane c-2+NP
+      if (tid == 0 && c >= 2 && c - 2 + NP < n_planes) {
+        const int jn = c - 2 + NP;
+        fence_proxy_async();
+        mbar_arrive_expect_tx(&bars[jn % NP], TX_BYTES);
+        tma_plane(P, g, slot(jn), &bars[jn % NP], g.s_start - R + jn);
+      }
+      // ---- plane c, in-plane operands
+      const double* pl = slot(c) + own;
+      auto L = [&](int a, int da, int db) { return r4_row<T>(pl + a * SLOT + db * PA, da); };
+      auto Ld = [&](int a, int dir, int k) {  // along physical direction a (x) or b
+        return dir == DA ? L(a, k, 0) : L(a, 0, k);
+      };
+      // per in-plane direction d: the outer-s products P = c * D'_d f, scattered to outputs
+      // c-2, c-1, c+1, c+2, and V_d of every output (real outputs only).  (Compiler fences
+      // between these phases cut the pair variant from 228 to 168 registers but cost 10-30 %:
+      // the hoisted loads are the latency hiding.)
+      auto scat = [&](int i, double w, T p) {
+        acc[i][ph(0)] = fma(-w, p, acc[i][ph(0)]);
+        acc[i][ph(1)] = fma(8.0 * w, p, acc[i][ph(1)]);
+        acc[i][ph(3)] = fma(-8.0 * w, p, acc[i][ph(3)]);
+        acc[i][ph(4)] = fma(w, p, acc[i][ph(4)]);
+      };
+#pragma unroll
+      for (int dd = 0; dd < 2; ++dd) {
+        const int d = dd == 0 ? DA : DB;
+        const T mu0 = L(3, 0, 0), la0 = L(4, 0, 0);
+        // mu D_d u_s -> r_d ; la D_d u_d -> r_s
+        scat(d, wp(d, DS), mu0 * r4_d<T>([&](int k) { return Ld(DS, d, k); }));
+        scat(DS, wp(d, DS), la0 * r4_d<T>([&](int k) { return Ld(d, d, k); }));
+        if (real) {
+#pragma unroll
+          for (int i = 0; i < 3; ++i) {
+            const T v = r4_v<T>(
+                [&](int k) { return i == d ? fma(2.0, Ld(3, d, k), Ld(4, d, k)) : Ld(3, d, k); },
+                [&](int k) { return Ld(i, d, k); });
+            acc[i][ph(2)] = fma(kv[d], v, acc[i][ph(2)]);
+          }
+        }
+      }
+      if (real) {
+        // in-plane mixed terms: D_o[c D_n f] with o, n in {a, b}
+        auto mixed = [&](int o, int n, int ca, int fa) {
+          auto inner = [&](int ko) {
+            auto f = [&](int kn) {
+              return L(fa, (o == DA ? ko : 0) + (n == DA ? kn : 0),
+                       (o == DB ? ko : 0) + (n == DB ? kn : 0));
+            };
+            return L(ca, o == DA ? ko : 0, o == DB ? ko : 0) * r4_d<T>(f);
+          };
+          return r4_d<T>(inner);
+        };
+        const double wab = wp(DA, DB);
+        acc[DA][ph(2)] = fma(wab, mixed(DB, DA, 3, DB) + mixed(DA, DB, 4, DB), acc[DA][ph(2)]);
+        acc[DB][ph(2)] = fma(wab, mixed(DA, DB, 3, DA) + mixed(DB, DA, 4, DA), acc[DB][ph(2)]);
+        // inner-s terms: outer differences of the product planes
+        const double* qp = qb + own;
+        auto Q = [&](int qi, int dir, int k) {
+          const double* row = qp + qi * SLOT + (dir == DB ? k * PA : 0);
+          return r4_row<T>(row, dir == DA ? k : 0);
+        };
+        const double was = wp(DA, DS), wbs = wp(DB, DS);
+        acc[DA][ph(2)] = fma(was, r4_d<T>([&](int k) { return Q(0, DA, k); }), acc[DA][ph(2)]);
+        acc[DB][ph(2)] = fma(wbs, r4_d<T>([&](int k) { return Q(0, DB, k); }), acc[DB][ph(2)]);
+        acc[DS][ph(2)] = fma(was, r4_d<T>([&](int k) { return Q(1, DA, k); }), acc[DS][ph(2)]);
+        acc[DS][ph(2)] = fma(wbs, r4_d<T>([&](int k) { return Q(2, DB, k); }), acc[DS][ph(2)]);
+      }
+      // ---- output c-2 is complete
+      const int co = c - 2;
+      if (co >= R && co < R + n_out && in_b) {
+        const long long off = col + (long long)(g.s_start + co - R) * g.st_s;
+#pragma unroll
+        for (int i = 0; i < 3; ++i) {
+          if (in_a0) put(P, i, off, r4_lane(acc[i][ph(0)], 0));
+          if (in_a1) put(P, i, off + 1, r4_lane(acc[i][ph(0)], 1));
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < 3; ++i) acc[i][ph(0)] = T{};
+    });
+  }
+}
+
+// =============================================================================
 // temporal blocking, bt > 1 (B200 extension):
 // BT sweeps of a star / box stencil fused into one pass over HBM.
 //   level 0   input planes, TMA ring, extent (TA + 2 BT XR) x (TB + 2 BT R)
@@ -2365,6 +2627,13 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 #endif
 #if CST_QSTORE == 2
 #define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ, CST_TM_MINB)
+#elif CST_KIND == 4 && CST_RET == 2 && CST_BMX == 1
+// rhs4 retimed, one point per thread: cap at ~168 registers (3 CTAs of 128 threads: 1.05 vs
+// 1.22 ms at 216 registers / 2 CTAs, 320^3); the queue then holds u1..u3
+#ifndef CST_R4MINB
+#define CST_R4MINB (65536 / (CST_TBX * CST_TBY * CST_TBZ * 168) > 0 ? 65536 / (CST_TBX * CST_TBY * CST_TBZ * 168) : 1)
+#endif
+#define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ, CST_R4MINB)
 #elif defined(CST_MINB)  // experiment hook (CST_NVRTC_DEFINES="-DCST_MINB=n")
 #define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ, CST_MINB)
 #else
@@ -2384,6 +2653,8 @@ extern "C" __global__ void CST_LB cst_kernel(const __grid_constant__ cst_kparams
     kernel_stream1(P, cst_smem);
   } else if constexpr (KIND == 3 && TS == 1) {
     kernel_hyp_stream1(P, cst_smem);
+  } else if constexpr (R4RET) {
+    kernel_rhs4_ret<0>(P, cst_smem);
   } else {
     kernel_stream_generic(P, cst_smem);
   }

@@ -51,6 +51,8 @@ const char* check_rules(const StencilInfo& st, const Tuple& t);
 int64_t model_smem_bytes(int kind, int r, const Tuple& t);
 int64_t model_regs(int kind, int r, const Tuple& t);
 int64_t uf_trip(int kind, const Tuple& t, int d);
+// R16: the setting selects rhs4's retimed column-walk kernel (kernel_rhs4_ret)
+bool r4ret_path(int kind, const Tuple& t);
 // TMEM columns one CTA of the qstore = 2 path allocates (power of two >= 32)
 int tmem_cols_alloc(int kind, int r, const Tuple& t);
 // Dynamic shared memory the kernel variant actually uses (<= model for fast paths).

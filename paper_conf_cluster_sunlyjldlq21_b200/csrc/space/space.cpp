@@ -127,6 +127,18 @@ static bool qs_path_ok(int kind, int r, const Tuple& t) {
   return tmem_cols_kind(kind, r, t) <= 512;
 }
 
+// R16: rhs4's retimed kernel (kernel_rhs4_ret in csrc/kernels/cst_kernels.cuh): streaming
+// with T_SD = 1, TMA, bt = 1, registers, no cyclic merging, one point along b, BM_a <= 2
+bool r4ret_path(int kind, const Tuple& t) {
+  if (kind != CST_RHS4 || t[F_RET] != 2) return false;
+  if (t[F_STREAM] != 2 || t[F_STAGING] != 3 || t[F_BT] != 1 || t[F_QS] != 1) return false;
+  const int sd = t[F_SD] - 1;
+  const int b = sd == 2 ? 1 : 2;
+  for (int d = 0; d < 3; ++d)
+    if (t[F_CMX + d] != 1) return false;
+  return t[F_TBX + sd] == 1 && t[F_BMX + sd] == 1 && t[F_BMX + b] == 1 && t[F_BMX] <= 2;
+}
+
 static bool tb_path_ok(int kind, const Tuple& t) {
   return (kind == CST_STAR || kind == CST_BOX) && t[F_STREAM] == 2 && t[F_SD] == 3 &&
          t[F_STAGING] == 3 && t[F_RET] == 2 && t[F_TBZ] == 1 && t[F_BMZ] == 1 &&
@@ -149,7 +161,9 @@ static void plane_geometry(int kind, int r, const Tuple& t, int64_t* P, int64_t*
     if (d != sd) (a < 0 ? a : b) = d;
   *P = (T[a] + 2 * r) * (T[b] + 2 * r);
   const int64_t D = t[F_PF];
-  if (T[sd] == 1)
+  if (T[sd] == 1 && r4ret_path(kind, t))
+    *NP = D + 2 * r;  // + the 6 product planes (model_smem_bytes)
+  else if (T[sd] == 1)
     *NP = D + (t[F_RET] == 2 ? 0 : retention(kind, r));
   else
     *NP = D * T[sd] + 2 * r;
@@ -161,7 +175,7 @@ int64_t model_smem_bytes(int kind, int r, const Tuple& t) {
   int64_t P, NP;
   plane_geometry(kind, r, t, &P, &NP);
   const int64_t plane = (P * 8 + 127) / 128 * 128;
-  return n_arrays(kind) * NP * plane;
+  return (n_arrays(kind) * NP + (r4ret_path(kind, t) ? 6 : 0)) * plane;
 }
 
 // Per-array halos of the hypterm TMA fast path (HTRIM in csrc/kernels/cst_kernels.cuh):
@@ -202,13 +216,17 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
     const int b = sd == 2 ? 1 : 2;
     plane_elems = (T[0] + 2 * XR) * (T[b] + 2 * r);
     const int64_t D = t[F_PF];
-    if (T[sd] == 1 && kind != CST_RHS4)  // fast streaming paths
+    if (r4ret_path(kind, t))              // rhs4 retimed: planes c-2 .. c+2 + prefetch
+      NP = D + 2 * r;
+    else if (T[sd] == 1 && kind != CST_RHS4)  // fast streaming paths
       NP = D + (t[F_RET] == 2 ? 0 : retention(kind, r));
     else                                 // generic ring
       NP = D * T[sd] + 2 * r;
   }
   const int64_t plane = (plane_elems * 8 + 127) / 128 * 128;
   const int64_t bars = t[F_STAGING] == 3 ? 2 * NP * 8 : 0;  // full (+ optional empty) mbarriers
+  if (t[F_STREAM] == 2 && r4ret_path(kind, t))  // + 2 buffers x 3 product planes
+    return (n_arrays(kind) * NP + 6) * plane + bars;
   if (t[F_STREAM] == 2 && hyp_trimmed(kind, t)) {
     int64_t slot = 0;
     for (int a = 0; a < n_arrays(kind); ++a) {
@@ -233,6 +251,11 @@ int64_t model_regs(int kind, int r, const Tuple& t) {
     int64_t ppt = 1;
     for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
     return 32 + 2 * (2 * ppt + (r + 1) + 2 * r);
+  }
+  if (r4ret_path(kind, t)) {
+    // per point: s-window queue (5 arrays x 5 planes; 3 arrays when BM_a = 2, mu / lambda
+    // then from the ring), 5 x 3 pending outputs, ~20 operands in flight
+    return 32 + 2 * t[F_BMX] * (t[F_BMX] == 1 ? 60 : 50);
   }
   if (t[F_BT] > 1) {
     int64_t pts = 0;
@@ -283,6 +306,7 @@ int64_t uf_trip(int kind, const Tuple& t, int d) {
   const int64_t bmcm = (int64_t)t[F_BMX + d] * t[F_CMX + d];
   if (t[F_STREAM] != 2) return bmcm;
   const int sd = t[F_SD] - 1;
+  if (r4ret_path(kind, t)) return 1;  // rhs4 retimed: the pair is lockstep, the plane loop rolled
   const bool fast = (kind == CST_STAR || kind == CST_BOX || kind == CST_HYPTERM) &&
                     (int64_t)t[F_TBX + sd] * t[F_BMX + sd] * t[F_CMX + sd] == 1;
   if (!fast) return bmcm;
@@ -338,7 +362,7 @@ const char* check_rules(const StencilInfo& st, const Tuple& t) {
   if (t[F_PF] > 1 && (!stream || t[F_STAGING] == 1)) return "R9";
   if (t[F_BT] > 1 && !tb_path_ok(st.kind, t)) return "R14";
   if (t[F_QS] == 2 && !qs_path_ok(st.kind, st.r, t)) return "R15";
-  if (st.kind == CST_RHS4 && t[F_RET] != 1) return "R16";
+  if (st.kind == CST_RHS4 && t[F_RET] == 2 && !r4ret_path(st.kind, t)) return "R16";
   if (model_smem_bytes(st.kind, st.r, t) > SMEM_LIMIT) return "R10";
   if (model_regs(st.kind, st.r, t) > REG_LIMIT) return "R11";
   if (t[F_STAGING] == 3 && !tma_ok(st.r, t)) return "R12";

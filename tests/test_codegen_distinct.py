@@ -18,7 +18,7 @@ import pytest
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 SUBSET = {"star4_tma_ret", "star4_ldst", "star4_tmem", "star4_generic", "star4_tile3d",
-          "star1_tblock", "hyp_tmem", "hyp_reg", "rhs4_bmz2", "box_l1"}
+          "star1_tblock", "hyp_tmem", "hyp_reg", "rhs4_bmz2", "box_l1", "rhs4_ret"}
 
 
 @pytest.mark.skipif(shutil.which("cuobjdump") is None, reason="cuobjdump not found")

@@ -160,6 +160,33 @@ def test_rhs4_paired_points_ragged(name, kw):
         H.assert_halo_untouched(L, got[o], np.full(L.numel, np.nan))
 
 
+RHS4_RETIMED = [("ret-pair-z", dict(tb_x=8, tb_y=8, bm_x=2)),
+                ("ret-scalar-z", dict(tb_x=16, tb_y=8, bm_x=1)),
+                ("ret-scalar-z-pf1", dict(tb_x=16, tb_y=8, bm_x=1, prefetch=1)),
+                ("ret-pair-z-pf3-sb4", dict(tb_x=8, tb_y=4, bm_x=2, prefetch=3, sb=4)),
+                ("ret-pair-y", dict(tb_x=16, tb_y=1, tb_z=8, sd=2, bm_x=2, prefetch=1)),
+                ("ret-scalar-y-sb16", dict(tb_x=32, tb_y=1, tb_z=2, sd=2, bm_x=1, sb=16)),
+                ("ret-pair-const", dict(tb_x=16, tb_y=2, bm_x=2, use_constant=2, prefetch=4))]
+
+
+@pytest.mark.parametrize("name,kw", RHS4_RETIMED, ids=[p[0] for p in RHS4_RETIMED])
+def test_rhs4_retimed_ragged(name, kw):
+    """rhs4's retimed column walk (R16): outer-s products scattered to the
+    pending outputs, inner-s product planes with their halo columns, s-window queue; ragged
+    grid (odd nx: the last pair of a row half outside; SB chunks with a ragged tail),
+    poisoned far halo, NaN-filled outputs."""
+    kind, r = 4, 2
+    L = H.layout((37, 22, 19), r + 1)
+    c = H.coeffs(kind, r, "random", seed=11)
+    ins = H.inputs(kind, L, seed=17, poison_beyond=r)
+    _, want = H.oracle_outputs(kind, r, c, L, ins)
+    kw = dict(kw)
+    _, got = run_gpu(kind, r, c, L, ins, S(**dict(dict(sb=8), **kw)))
+    for o in range(ost.N_OUT[kind]):
+        H.assert_parity(L, got[o], want[o], f"{name} out{o}")
+        H.assert_halo_untouched(L, got[o], np.full(L.numel, np.nan))
+
+
 def test_integer_polynomial_bit_exact():
     """Integer weights and integer data: FMA is exact, so GPU == oracle bit-for-bit."""
     r = 4

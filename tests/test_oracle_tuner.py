@@ -167,11 +167,19 @@ def test_space_rules_spot_checks():
     assert S.check(1, 4, M, dict(base, tb_y=2, tb_z=2, bm_z=2, uf_z=2)) is None
     assert S.check(1, 4, M, dict(base, use_streaming=1, sd=1, sb=1, prefetch=1, bm_y=2,
                                  uf_y=2)) is None
-    # R9: no staging -> nothing to prefetch; R16: rhs4 has one summation form
+    # R9: no staging -> nothing to prefetch; R16: rhs4's retimed form only on its column
+    # walk (T_SD = 1, TMA, bt 1, registers, CM 1, BM_b 1, BM_x <= 2)
     assert S.check(1, 4, M, dict(base, staging=1)) == "R9"
     assert S.check(1, 4, M, dict(base, staging=1, prefetch=1)) is None
-    assert S.check(4, 2, M, dict(base, tb_x=16, tb_y=8)) == "R16"
+    assert S.check(4, 2, M, dict(base, tb_x=16, tb_y=8)) is None
+    assert S.check(4, 2, M, dict(base, tb_x=8, tb_y=8, bm_x=2)) is None
     assert S.check(4, 2, M, dict(base, tb_x=16, tb_y=8, use_retiming=1)) is None
+    assert S.check(4, 2, M, dict(base, tb_x=16, tb_y=4, bm_y=2)) == "R16"
+    assert S.check(4, 2, M, dict(base, tb_x=8, tb_y=8, bm_x=4)) == "R16"
+    assert S.check(4, 2, M, dict(base, tb_x=16, tb_y=8, staging=2)) == "R16"
+    assert S.check(4, 2, M, dict(base, tb_x=16, tb_y=4, tb_z=2)) == "R16"
+    assert S.check(4, 2, M, dict(base, tb_x=8, tb_y=8, cm_x=2)) == "R16"
+    assert S.check(4, 2, M, dict(base, tb_x=16, tb_y=8, uf_x=2)) == "R6"
     assert S.check(1, 4, M, dict(base, bm_y=8, cm_y=4)) == "R7"
     assert S.check(1, 4, M, dict(base, sd=1)) == "R8"
     assert S.check(1, 4, M, dict(base, use_streaming=1, sd=1, sb=1, prefetch=2)) == "R9"

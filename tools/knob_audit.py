@@ -55,6 +55,8 @@ BASES = [
     ("rhs4_bmz2", 4, 2, dict(tb_x=16, tb_y=8, bm_x=1, bm_y=1, bm_z=2, uf_z=2, prefetch=2,
                                    use_retiming=1)),
     ("box_ldst", 2, 1, dict(staging=2, prefetch=1)),
+    ("rhs4_ret", 4, 2, dict(tb_x=16, tb_y=8, bm_x=1, bm_y=1, prefetch=2, use_retiming=2)),
+    ("rhs4_ret_pair", 4, 2, dict(tb_x=8, tb_y=8, bm_x=2, bm_y=1, prefetch=2, use_retiming=2)),
     ("star2_tma_ret", 1, 2, {}),
 ]
 
