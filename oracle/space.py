@@ -40,7 +40,8 @@ TMEM path: star or hypterm (hypterm: one point along x, BM_b <= 2 along the othe
 dim, no cyclic merging), streaming with T_SD = 1, TMA staging, retimed, bt = 1, and
 ceil(threads/128) * points per thread * (4r star, 20r hypterm) <= 512 TMEM columns;
 R16 rhs4: use_retiming = 2 only for the retimed column walk (r4ret_path: streaming with
-T_SD = 1, TMA, bt = 1, qstore 1, CM = 1, BM_b = 1, BM_x <= 2).  R6/R9/R16 keep every
+T_SD = 1, TMA, bt = 1, CM = 1, BM_b = 1, BM_x <= 2; qstore 2 puts its s-window queue in TMEM,
+R15: ceil(threads/128) * points * 10(2r+1) <= 512 columns).  R6/R9/R16 keep every
 field a kernel path does not read at its canonical value (round 2; tools/knob_audit.py).
 """
 from __future__ import annotations
@@ -104,12 +105,11 @@ def tb_blocks_per_thread(r: int, s: dict, level: int) -> int:
 
 def r4ret_path(kind: int, s: dict) -> bool:
     """R16: the setting selects rhs4's retimed column walk (use_retiming = 2): streaming with
-    T_SD = 1, TMA staging, bt = 1, registers (qstore 1), no cyclic merging, one point along
-    the in-plane non-x dim b, BM_x <= 2."""
+    T_SD = 1, TMA staging, bt = 1, no cyclic merging, one point along the in-plane non-x dim
+    b, BM_x <= 2; its s-window queue in registers / shared memory (qstore 1) or TMEM (2)."""
     if kind != RHS4 or s["use_retiming"] != 2:
         return False
-    if not (s["use_streaming"] == 2 and s["staging"] == 3 and s["bt"] == 1
-            and s["qstore"] == 1):
+    if not (s["use_streaming"] == 2 and s["staging"] == 3 and s["bt"] == 1):
         return False
     sd = "xyz"[s["sd"] - 1]
     b = "y" if sd == "z" else "z"
@@ -163,12 +163,18 @@ def tmem_columns(r: int, s: dict, kind: int = STAR) -> int:
     quarters (ceil(threads/128) share one), each thread keeps 4r columns per point (star:
     r (value, partial) pairs) or 20r (hypterm: r slots of 5 products + r of 5 partials)."""
     nthr = s["tb_x"] * s["tb_y"] * s["tb_z"]
-    per = 20 if kind == HYPTERM else 4
-    return (nthr // 32 + 3) // 4 * points_per_thread(s) * per * r
+    if kind == RHS4:      # rhs4 retimed: 5 arrays x (2r+1) planes of the s-window, 2 columns each
+        per = 10 * (2 * r + 1)
+    else:
+        per = (20 if kind == HYPTERM else 4) * r
+    return (nthr // 32 + 3) // 4 * points_per_thread(s) * per
 
 
 def qs_path_ok(kind: int, r: int, s: dict) -> bool:
-    """R15: the TMEM streamed-state path's structural and capacity requirements."""
+    """R15: the TMEM streamed-state path's structural and capacity requirements (rhs4: the
+    retimed column walk with its s-window queue in TMEM)."""
+    if kind == RHS4:
+        return r4ret_path(kind, s) and tmem_columns(r, s, kind) <= 512
     if not (kind in (STAR, HYPTERM) and s["use_streaming"] == 2 and s["staging"] == 3
             and s["use_retiming"] == 2 and s["bt"] == 1):
         return False
@@ -184,16 +190,16 @@ def qs_path_ok(kind: int, r: int, s: dict) -> bool:
 
 
 def est_regs(kind: int, r: int, s: dict) -> int:
+    if r4ret_path(kind, s):
+        # s-window queue (5 arrays x 5 planes; 3 arrays when BM_x = 2), 5 x 3 pending
+        # outputs, ~20 operands in flight, per point
+        return 32 + 2 * s["bm_x"] * (60 if s["bm_x"] == 1 else 50)
     if s["qstore"] == 2 and kind == HYPTERM:
         # products, partial fluxes, the ring of one point, the in-plane row values
         return 32 + 2 * (5 * (r + 1) + 10 * points_per_thread(s) + 30)
     if s["qstore"] == 2:
         # in-plane part + centre per point, one point's ring, the block's column windows
         return 32 + 2 * (2 * points_per_thread(s) + (r + 1) + 2 * r)
-    if r4ret_path(kind, s):
-        # s-window queue (5 arrays x 5 planes; 3 arrays when BM_x = 2), 5 x 3 pending
-        # outputs, ~20 operands in flight, per point
-        return 32 + 2 * s["bm_x"] * (60 if s["bm_x"] == 1 else 50)
     if s["bt"] > 1:
         # 2r+1 rotating accumulators per point of every level + one operand window
         pts = sum(tb_blocks_per_thread(r, s, lv) for lv in range(1, s["bt"] + 1))

@@ -1520,7 +1520,42 @@ constexpr int R4NH = 2 * TB + 4 * (TA / 2);      // halo column pairs of the pro
 #ifndef CST_R4Q
 #define CST_R4Q (BMA == 1 ? 3 : 0)
 #endif
-constexpr int R4Q = CST_R4Q;  // arrays of the s-window kept in the register queue
+constexpr int R4Q = QTM ? 0 : CST_R4Q;  // arrays of the s-window in the register queue
+// qstore = 2: the whole s-window queue (5 arrays x 5 planes) lives in tensor memory, one lane
+// per thread (R15): R4TC columns per value, R4TPT per thread (array-major, 5 slots each)
+constexpr int R4TC = BMA == 2 ? 4 : 2, R4TPT = 25 * R4TC;
+constexpr int R4TUSED = ((NTHR / 32 + 3) / 4) * R4TPT;
+constexpr int R4TCOLS = R4TUSED <= 32 ? 32 : R4TUSED <= 64 ? 64 : R4TUSED <= 128 ? 128
+                       : R4TUSED <= 256 ? 256 : 512;
+// one value T of the queue (array-major layout: column of array a, slot p =
+// tq + (a * 5 + p) * R4TC): store / load into raw 32-bit words / unpack
+template <class T>
+__device__ __forceinline__ void r4_tm_st1(u32 a, T v) {
+  if constexpr (sizeof(T) == 8) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1, %2};" ::"r"(a),
+                 "r"((u32)__double2loint(v)), "r"((u32)__double2hiint(v)));
+  } else {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a),
+                 "r"((u32)__double2loint(v.x)), "r"((u32)__double2hiint(v.x)),
+                 "r"((u32)__double2loint(v.y)), "r"((u32)__double2hiint(v.y)));
+  }
+}
+__device__ __forceinline__ void tmem_ld_x4(u32 a, u32* r) {
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+               : "r"(a)
+               : "memory");
+}
+template <class T>
+__device__ __forceinline__ void r4_tm_ld1(u32 a, u32* r) {
+  if constexpr (sizeof(T) == 8) tmem_ld_x2(a, r);
+  else tmem_ld_x4(a, r);
+}
+template <class T>
+__device__ __forceinline__ T r4_tm_v1(const u32* r) {
+  if constexpr (sizeof(T) == 8) return tmem_d(r[0], r[1]);
+  else return T{tmem_d(r[0], r[1]), tmem_d(r[2], r[3])};
+}
 
 template <class T>
 __device__ __forceinline__ T r4_row(const double* row, int da) {
@@ -1559,6 +1594,24 @@ __device__ __forceinline__ T r4_v(const A& a, const F& f) {
   v = fma(m4, f(2) - f0, v);
   return v;
 }
+// the same split in two: the weights m1..m4 of a field a, then the sum over f
+template <class T, class A>
+__device__ __forceinline__ void r4_m(const A& a, T (&m)[4]) {
+  const T am2 = a(-2), am1 = a(-1), a0 = a(0), ap1 = a(1), ap2 = a(2);
+  m[0] = fma(-0.75, a0 + am2, am1);
+  m[1] = fma(3.0, a0 + am1, am2 + ap1);
+  m[2] = fma(3.0, ap1 + a0, am1 + ap2);
+  m[3] = fma(-0.75, a0 + ap2, ap1);
+}
+template <class T, class F>
+__device__ __forceinline__ T r4_vm(const T (&m)[4], const F& f) {
+  const T f0 = f(0);
+  T v = m[0] * (f(-2) - f0);
+  v = fma(m[1], f(-1) - f0, v);
+  v = fma(m[2], f(1) - f0, v);
+  v = fma(m[3], f(2) - f0, v);
+  return v;
+}
 // unscaled D'[f] = 8 (f(+1) - f(-1)) + (f(-2) - f(+2))  (the 1/12 factors are folded)
 template <class T, class F>
 __device__ __forceinline__ T r4_d(const F& f) {
@@ -1585,11 +1638,20 @@ __device__ __forceinline__ void kernel_rhs4_ret(const cst_kparams& P, double* sm
   const double kv[3] = {C.coef(3), C.coef(4), C.coef(5)};
   auto wp = [&](int d, int i) { return C.coef(6 + d + i - 1); };  // s_d s_i / 144, d != i
 
+  u32* tslot = (u32*)(bars + NP);  // spare mbarrier words (kernel_smem_bytes reserves 2 NP)
+  const int warp = tid >> 5;
+  if constexpr (QTM) {
+    if (warp == 0) tmem_alloc(tslot, R4TCOLS);
+  }
   if (tid == 0) {
     for (int s = 0; s < NP; ++s) mbar_init(&bars[s], 1);
     fence_mbar_init();
   }
+  if constexpr (QTM) tmem_fence_before_sync();
   __syncthreads();
+  if constexpr (QTM) tmem_fence_after_sync();
+  // the thread's TMEM queue: lane quarter of its warp, column block of its warp in the quarter
+  const u32 tq = QTM ? *tslot + ((u32)((warp & 3) * 32) << 16) + (u32)((warp >> 2) * R4TPT) : 0u;
   if (tid == 0) {
     for (int j = 0; j < NP && j < n_planes; ++j) {
       mbar_arrive_expect_tx(&bars[j], TX_BYTES);
@@ -1613,7 +1675,13 @@ __device__ __forceinline__ void kernel_rhs4_ret(const cst_kparams& P, double* sm
     mbar_wait(&bars[j], 0u);
 #pragma unroll
     for (int a = 0; a < NQA; ++a) q[a][2 + j] = r4_row<T>(slot(j) + a * SLOT + own, 0);
+    if constexpr (QTM) {
+#pragma unroll
+      for (int a = 0; a < 5; ++a)
+        r4_tm_st1<T>(tq + (u32)((a * QN + 2 + j) * R4TC), r4_row<T>(slot(j) + a * SLOT + own, 0));
+    }
   }
+  if constexpr (QTM) tmem_wait_st();
 
   const long long col = (long long)(g.a0 + la) + (long long)(g.b0 + lb) * g.st_b;
   const bool in_b = g.b0 + lb < g.n_b;
@@ -1627,10 +1695,18 @@ __device__ __forceinline__ void kernel_rhs4_ret(const cst_kparams& P, double* sm
       if (c >= n_planes) return;  // CTA-uniform
       const bool real = c >= R && c < R + n_out;
       // ---- newest plane c+2 -> queue
+      T nw[QTM ? 5 : 1];
       if (c + 2 < n_planes) {
         mbar_wait(&bars[(c + 2) % NP], (u32)(((c + 2) / NP) & 1));
 #pragma unroll
         for (int a = 0; a < NQA; ++a) q[a][ph(4)] = r4_row<T>(slot(c + 2) + a * SLOT + own, 0);
+        if constexpr (QTM) {
+#pragma unroll
+          for (int a = 0; a < 5; ++a) {
+            nw[a] = r4_row<T>(slot(c + 2) + a * SLOT + own, 0);
+            r4_tm_st1<T>(tq + (u32)((a * QN + ph(4)) * R4TC), nw[a]);
+          }
+        }
       }
       // s-window of array a at the own column, offset k in -2..2
       auto sw = [&](int a, int k) -> T {
@@ -1638,7 +1714,51 @@ __device__ __forceinline__ void kernel_rhs4_ret(const cst_kparams& P, double* sm
         return r4_row<T>(slot(c + k) + a * SLOT + own, 0);
       };
       double* qb = qbuf + (c & 1) * 3 * SLOT;
-      if (real) {
+      if (QTM && real) {
+        // ---- V_s and the inner-s products from the TMEM queue, in stages (mu, lambda and
+        // u_s; then u_a; then u_b — each load issued one stage ahead) so that only one
+        // array's window is live beside the V weights
+        auto tcol = [&](int a, int k) { return tq + (u32)((a * QN + ph(2 + k)) * R4TC); };
+        u32 wm[4][R4TC], wl[4][R4TC], wu[3][4][R4TC];
+        auto issue_u = [&](int ii, int a) {
+#pragma unroll
+          for (int k = 0; k < 4; ++k) r4_tm_ld1<T>(tcol(a, k - 2), wu[ii][k]);
+        };
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          r4_tm_ld1<T>(tcol(3, k - 2), wm[k]);
+          r4_tm_ld1<T>(tcol(4, k - 2), wl[k]);
+        }
+        issue_u(0, DS);
+        tmem_wait_ld();
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          tmem_pin(wm[k]);
+          tmem_pin(wl[k]);
+          tmem_pin(wu[0][k]);
+        }
+        auto mu = [&](int k) { return k == 2 ? nw[3] : r4_tm_v1<T>(wm[k + 2]); };
+        auto lam = [&](int k) { return k == 2 ? nw[4] : r4_tm_v1<T>(wl[k + 2]); };
+        const T mu0 = mu(0), la0 = lam(0);
+        // V weights for a = mu (outputs i != s) and a = 2 mu + lambda (output s)
+        T mm[4], mk[4];
+        r4_m<T>([&](int k) { return mu(k); }, mm);
+        r4_m<T>([&](int k) { return fma(2.0, mu(k), lam(k)); }, mk);
+#pragma unroll
+        for (int ii = 0; ii < 3; ++ii) {
+          const int i = ii == 0 ? DS : (ii == 1 ? DA : DB);
+          if (ii < 2) issue_u(ii + 1, ii == 0 ? DA : DB);
+          auto f = [&](int k) { return k == 2 ? nw[i] : r4_tm_v1<T>(wu[ii][k + 2]); };
+          acc[i][ph(2)] = fma(kv[DS], r4_vm<T>(ii == 0 ? mk : mm, f), acc[i][ph(2)]);
+          r4_put_row<T>(qb + ii * SLOT + own, (ii == 0 ? la0 : mu0) * r4_d<T>(f));
+          if (ii < 2) {
+            tmem_wait_ld();
+#pragma unroll
+            for (int k = 0; k < 4; ++k) tmem_pin(wu[ii + 1][k]);
+          }
+        }
+      }
+      if (!QTM && real) {
         // ---- V_s and the inner-s products of the own column
         const T mu0 = sw(3, 0), la0 = sw(4, 0);
 #pragma unroll
@@ -1651,6 +1771,8 @@ __device__ __forceinline__ void kernel_rhs4_ret(const cst_kparams& P, double* sm
         r4_put_row<T>(qb + 0 * SLOT + own, la0 * r4_d<T>([&](int k) { return sw(DS, k); }));
         r4_put_row<T>(qb + 1 * SLOT + own, mu0 * r4_d<T>([&](int k) { return sw(DA, k); }));
         r4_put_row<T>(qb + 2 * SLOT + own, mu0 * r4_d<T>([&](int k) { return sw(DB, k); }));
+      }
+      if (real) {
         // ---- halo columns of the product planes (pairs of x-adjacent columns):
         // a-strips (la*D_s u_s, mu*D_s u_a), b-strips (la*D_s u_s, mu*D_s u_b)
         for (int e = tid; e < R4NH; e += NTHR) {
@@ -1754,7 +1876,14 @@ __device__ __forceinline__ void kernel_rhs4_ret(const cst_kparams& P, double* sm
       }
 #pragma unroll
       for (int i = 0; i < 3; ++i) acc[i][ph(0)] = T{};
+      if constexpr (QTM) tmem_wait_st();  // the next plane reads the slot written here
     });
+  }
+  if constexpr (QTM) {
+    tmem_fence_before_sync();
+    __syncthreads();
+    tmem_fence_after_sync();
+    if (warp == 0) tmem_dealloc(*tslot, R4TCOLS);
   }
 }
 
@@ -2625,7 +2754,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 #ifndef CST_TM_MINB
 #define CST_TM_MINB (65536 / (CST_TM_NTHR * CST_TM_REGS) > 0 ? 65536 / (CST_TM_NTHR * CST_TM_REGS) : 1)
 #endif
-#if CST_QSTORE == 2
+#if CST_QSTORE == 2 && CST_KIND != 4
 #define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ, CST_TM_MINB)
 #elif CST_KIND == 4 && CST_RET == 2 && CST_BMX == 1
 // rhs4 retimed, one point per thread: cap at ~168 registers (3 CTAs of 128 threads: 1.05 vs
@@ -2645,6 +2774,8 @@ extern "C" __global__ void CST_LB cst_kernel(const __grid_constant__ cst_kparams
     kernel_tblock<0>(P, cst_smem);
   } else if constexpr (!STREAM) {
     kernel_tile3d(P, cst_smem);
+  } else if constexpr (R4RET) {
+    kernel_rhs4_ret<0>(P, cst_smem);
   } else if constexpr (QTM && KIND == 3) {
     kernel_hyp_tmem<0>(P, cst_smem);
   } else if constexpr (QTM) {
@@ -2653,8 +2784,6 @@ extern "C" __global__ void CST_LB cst_kernel(const __grid_constant__ cst_kparams
     kernel_stream1(P, cst_smem);
   } else if constexpr (KIND == 3 && TS == 1) {
     kernel_hyp_stream1(P, cst_smem);
-  } else if constexpr (R4RET) {
-    kernel_rhs4_ret<0>(P, cst_smem);
   } else {
     kernel_stream_generic(P, cst_smem);
   }

@@ -249,29 +249,31 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
   const int64_t* M = h->info.M;
   // measured-good starting points on B200, shrunk to fit small grids:
   // streaming along z, TMA staging, retimed accumulators; star/box 64x8 tiles of 2x2
-  // register blocks; rhs4 16x8 tiles, one point per thread (128-plane blocks, 2-deep TMA
-  // ring — 24.5 vs 23.4 GSt/s at 320^3 over pf 1); hypterm 32x4 threads with two points
+  // register blocks; rhs4 the retimed column walk, 8x16 threads with two x-adjacent points
+  // each, 64-plane blocks, 1-deep prefetch, coefficients in __constant__ (0.965 vs 1.095 ms
+  // for the generic path at 320^3); hypterm 32x4 threads with two points
   // stacked along y each, streamed state in TMEM, 3-deep ring, coefficients in __constant__
   // (3.16-3.19 ms vs 3.53 ms for the best register-path setting at 512^3).
   const bool hyp = h->info.kind == CST_HYPTERM || h->info.kind == CST_RHS4;
   const bool hyp_tm = h->info.kind == CST_HYPTERM;
+  const bool r4 = h->info.kind == CST_RHS4;
   cst_setting c{};
-  c.tb[0] = hyp && !hyp_tm ? 16 : 32;
-  c.tb[1] = hyp && !hyp_tm ? 8 : 4;
+  c.tb[0] = r4 ? 8 : 32;
+  c.tb[1] = r4 ? 16 : 4;
   c.tb[2] = 1;
   c.staging = 3;
   c.use_constant = 1;
   c.use_streaming = 2;
   c.sd = 3;
-  c.sb = p2floor(M[2], h->info.kind == CST_HYPTERM ? 256 : 128);
+  c.sb = p2floor(M[2], h->info.kind == CST_HYPTERM ? 256 : (r4 ? 64 : 128));
   for (int d = 0; d < 3; ++d) c.uf[d] = c.cm[d] = c.bm[d] = 1;
-  c.bm[0] = hyp ? 1 : 2;
-  c.bm[1] = hyp && !hyp_tm ? 1 : 2;
-  c.use_retiming = h->info.kind == CST_RHS4 ? 1 : 2;  // R16: rhs4 has one summation form
+  c.bm[0] = hyp && !r4 ? 1 : 2;
+  c.bm[1] = r4 ? 1 : 2;
+  c.use_retiming = 2;
   c.bt = 1;
   c.qstore = hyp_tm ? 2 : 1;
-  if (hyp_tm) c.use_constant = 2;
-  c.prefetch = (h->info.kind == CST_BOX || h->info.kind == CST_RHS4) ? 2 : 3;
+  if (hyp) c.use_constant = 2;
+  c.prefetch = h->info.kind == CST_BOX ? 2 : (r4 ? 1 : 3);
   for (int tries = 0; tries < 12 && check_rules(h->info, to_tuple(c)); ++tries) {
     if (c.qstore == 2 && c.staging != 3) { c.qstore = 1; continue; }  // R15 needs TMA
     // shrink the tile until it fits the grid (coverage) and the thread floor
@@ -281,6 +283,7 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
     else if (c.tb[1] > 1 && c.tb[1] > M[1]) { c.tb[1] /= 2; }
     else if (c.tb[0] * c.bm[0] % 2) { c.staging = 2; }
     else if (c.qstore == 2) { c.qstore = 1; }
+    else if (r4 && c.use_retiming == 2) { c.use_retiming = 1; }  // R16 needs TMA staging
     else break;
   }
   if (!check_rules(h->info, to_tuple(c))) {

@@ -103,7 +103,9 @@ static int64_t tmem_cols_kind(int kind, int r, const Tuple& t) {
   int64_t ppt = 1;
   for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
   const int64_t nthr = (int64_t)t[F_TBX] * t[F_TBY] * t[F_TBZ];
-  return (nthr / 32 + 3) / 4 * ppt * (kind == CST_HYPTERM ? 20 : 4) * r;
+  // rhs4 retimed: the s-window queue, 5 arrays x (2r + 1) planes x 2 columns per point
+  const int64_t per = kind == CST_HYPTERM ? 20 * r : (kind == CST_RHS4 ? 10 * (2 * r + 1) : 4 * r);
+  return (nthr / 32 + 3) / 4 * ppt * per;
 }
 
 int tmem_cols_alloc(int kind, int r, const Tuple& t) {
@@ -113,7 +115,10 @@ int tmem_cols_alloc(int kind, int r, const Tuple& t) {
   return c;
 }
 
+bool r4ret_path(int kind, const Tuple& t);
+
 static bool qs_path_ok(int kind, int r, const Tuple& t) {
+  if (kind == CST_RHS4) return r4ret_path(kind, t) && tmem_cols_kind(kind, r, t) <= 512;
   if ((kind != CST_STAR && kind != CST_HYPTERM) || t[F_STREAM] != 2 || t[F_STAGING] != 3 ||
       t[F_RET] != 2 || t[F_BT] != 1)
     return false;
@@ -128,10 +133,11 @@ static bool qs_path_ok(int kind, int r, const Tuple& t) {
 }
 
 // R16: rhs4's retimed kernel (kernel_rhs4_ret in csrc/kernels/cst_kernels.cuh): streaming
-// with T_SD = 1, TMA, bt = 1, registers, no cyclic merging, one point along b, BM_a <= 2
+// with T_SD = 1, TMA, bt = 1, no cyclic merging, one point along b, BM_a <= 2; the s-window
+// queue in registers / shared memory (qstore 1) or tensor memory (qstore 2, R15 columns)
 bool r4ret_path(int kind, const Tuple& t) {
   if (kind != CST_RHS4 || t[F_RET] != 2) return false;
-  if (t[F_STREAM] != 2 || t[F_STAGING] != 3 || t[F_BT] != 1 || t[F_QS] != 1) return false;
+  if (t[F_STREAM] != 2 || t[F_STAGING] != 3 || t[F_BT] != 1) return false;
   const int sd = t[F_SD] - 1;
   const int b = sd == 2 ? 1 : 2;
   for (int d = 0; d < 3; ++d)
@@ -240,6 +246,11 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
 }
 
 int64_t model_regs(int kind, int r, const Tuple& t) {
+  if (r4ret_path(kind, t)) {
+    // per point: s-window queue (5 arrays x 5 planes; 3 arrays when BM_a = 2, mu / lambda
+    // then from the ring), 5 x 3 pending outputs, ~20 operands in flight
+    return 32 + 2 * t[F_BMX] * (t[F_BMX] == 1 ? 60 : 50);
+  }
   if (t[F_QS] == 2 && kind == CST_HYPTERM) {  // products, partial fluxes, ring, row values
     int64_t ppt = 1;
     for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
@@ -251,11 +262,6 @@ int64_t model_regs(int kind, int r, const Tuple& t) {
     int64_t ppt = 1;
     for (int d = 0; d < 3; ++d) ppt *= (int64_t)t[F_BMX + d] * t[F_CMX + d];
     return 32 + 2 * (2 * ppt + (r + 1) + 2 * r);
-  }
-  if (r4ret_path(kind, t)) {
-    // per point: s-window queue (5 arrays x 5 planes; 3 arrays when BM_a = 2, mu / lambda
-    // then from the ring), 5 x 3 pending outputs, ~20 operands in flight
-    return 32 + 2 * t[F_BMX] * (t[F_BMX] == 1 ? 60 : 50);
   }
   if (t[F_BT] > 1) {
     int64_t pts = 0;

@@ -29,7 +29,7 @@ CHILD = textwrap.dedent("""
         before = set(os.listdir(os.environ["CST_CACHE_DIR"]))
         C.cst_variant_compile(h, s)
         new = sorted(set(os.listdir(os.environ["CST_CACHE_DIR"])) - before)
-        out.append(new)
+        out.append([json.dumps([kind, r, n, s.as_dict(), remote]), new])
         C.cst_stencil_destroy(h)
     print(json.dumps(out))
 """)
@@ -71,8 +71,12 @@ def test_default_and_bench_variants_have_no_stack_or_local(tmp_path):
                          env=env, capture_output=True, text=True, timeout=900)
     assert res.returncode == 0, res.stderr[-2000:]
     files = json.loads(res.stdout.strip().splitlines()[-1])
-    for case, new in zip(CASES, files):
+    seen = {}
+    for case, (key, new) in zip(CASES, files):
+        if not new and key in seen:   # same variant as an earlier case (e.g. default == tuned)
+            new = seen[key]
         assert len(new) == 1, (case, new)
+        seen[key] = new
         usage = subprocess.run(["cuobjdump", "--dump-resource-usage", str(tmp_path / new[0])],
                                capture_output=True, text=True, check=True).stdout
         m = re.search(r"REG:(\d+) STACK:(\d+) SHARED:\d+ LOCAL:(\d+)", usage)

@@ -166,7 +166,12 @@ RHS4_RETIMED = [("ret-pair-z", dict(tb_x=8, tb_y=8, bm_x=2)),
                 ("ret-pair-z-pf3-sb4", dict(tb_x=8, tb_y=4, bm_x=2, prefetch=3, sb=4)),
                 ("ret-pair-y", dict(tb_x=16, tb_y=1, tb_z=8, sd=2, bm_x=2, prefetch=1)),
                 ("ret-scalar-y-sb16", dict(tb_x=32, tb_y=1, tb_z=2, sd=2, bm_x=1, sb=16)),
-                ("ret-pair-const", dict(tb_x=16, tb_y=2, bm_x=2, use_constant=2, prefetch=4))]
+                ("ret-pair-const", dict(tb_x=16, tb_y=2, bm_x=2, use_constant=2, prefetch=4)),
+                # qstore 2: the s-window queue in tensor memory (R15)
+                ("ret-pair-tmem", dict(tb_x=8, tb_y=16, bm_x=2, qstore=2, prefetch=1)),
+                ("ret-pair-tmem-256thr", dict(tb_x=16, tb_y=16, bm_x=2, qstore=2, prefetch=1)),
+                ("ret-scalar-tmem-y", dict(tb_x=32, tb_y=1, tb_z=4, sd=2, bm_x=1, qstore=2,
+                                           prefetch=2, sb=4))]
 
 
 @pytest.mark.parametrize("name,kw", RHS4_RETIMED, ids=[p[0] for p in RHS4_RETIMED])

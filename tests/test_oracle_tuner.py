@@ -224,7 +224,11 @@ def test_space_rules_spot_checks():
     assert S.est_regs(3, 4, hq) == 32 + 2 * (25 + 10 + 30)
     assert S.check(3, 4, M, dict(hq, bm_x=2, tb_x=16)) == "R15"   # blocked: not this path
     assert S.check(3, 4, M, dict(hq, tb_y=32)) == "R15"            # 640 columns
-    assert S.check(4, 2, M, dict(hq)) == "R15"                     # rhs4: no TMEM path
+    # rhs4: the retimed column walk's s-window queue, 10 (2r + 1) = 50 columns per point
+    assert S.tmem_columns(2, hq, 4) == 50 and S.check(4, 2, M, hq) is None
+    assert S.check(4, 2, M, dict(hq, tb_x=16, bm_x=2)) is None     # 100 columns
+    assert S.check(4, 2, M, dict(hq, tb_y=32, bm_x=2)) == "R15"    # 8 warps/quarter: 800
+    assert S.check(4, 2, M, dict(hq, use_retiming=1)) == "R15"     # generic path: no TMEM
     assert S.check(1, 4, M, dict(q, staging=2)) == "R15"
     assert S.check(1, 4, M, dict(q, use_retiming=1)) == "R15"
     assert S.check(1, 4, M, dict(q, tb_z=2, tb_y=2)) == "R15"  # T_SD = 2
