@@ -7,8 +7,8 @@ compute-sanitizer:
 
 Paths: star / box fast streaming with TMA ring (retimed, gather), ld/st and no staging;
 y-streaming; generic (T_SD > 1) ring; 3-D tiles; TMEM streamed state (star, hypterm with
-two points along b); hypterm register path; rhs4 generic; temporal blocking (bt = 2, 4
-steps); multi-step ping-pong.  The two-process peer-memory twin (CST_REMOTE) runs under
+two points along b); hypterm register path; rhs4 generic and retimed (ring, register queue,
+TMEM queue); temporal blocking (bt = 2, 4 steps); multi-step ping-pong.  The two-process peer-memory twin (CST_REMOTE) runs under
 --target-processes all through tests/test_gpu_p2p.py.
 """
 import os
@@ -50,6 +50,13 @@ CASES = [
                                               use_retiming=1), 1),
     ("rhs4-paired", 4, 2, (37, 22, 19), dict(tb_x=8, tb_y=8, bm_x=2, bm_y=1,
                                              use_retiming=1), 1),
+    # rhs4 retimed column walk (round 2): product planes + one barrier per plane, ring of
+    # 2r + PF planes; s-window from the ring (pair), register queue (scalar), TMEM (qstore 2)
+    ("rhs4-ret-pair", 4, 2, (37, 22, 19), dict(tb_x=8, tb_y=16, bm_x=2, bm_y=1, prefetch=1,
+                                               use_constant=2), 1),
+    ("rhs4-ret-scalar", 4, 2, (37, 22, 19), dict(tb_x=16, tb_y=8, bm_x=1, bm_y=1), 1),
+    ("rhs4-ret-tmem-256", 4, 2, (37, 22, 19), dict(tb_x=16, tb_y=16, bm_x=2, bm_y=1,
+                                                   prefetch=1, qstore=2), 1),
 ]
 
 
