@@ -2722,7 +2722,8 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 #if !CST_HYP_ROWS
 #error "CST_HYP_ROWS = 0 (window path) was removed from the TMEM hypterm kernel"
 #endif
-    tmem_wait_st();  // the next plane reads these slots
+    tmem_wait_st();  // the next plane reads these slots (waiting at the next plane's ring
+                     // fetch instead measured the same: 3.171 vs 3.170 ms, g25)
     __syncthreads();
     if (tid == 0 && j + D < n_planes) {
       const int sl = (j + D) % NP;
