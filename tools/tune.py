@@ -75,6 +75,9 @@ def main():
     ap.add_argument("--start", default=None,
                     help="tuned JSON to refine from: skips cst_tune and hill-climbs from its "
                          "setting (implies --refine)")
+    ap.add_argument("--no-warm-start", action="store_true",
+                    help="do not add cst_setting_default() to the dataset (cst_tune_opts."
+                         "warm_start = 0): the paper's pipeline from seeded samples only")
     ap.add_argument("--fix", action="append", default=[],
                     help="field=value: tune the sub-space with this field fixed (e.g. "
                          "staging=1); other candidates get fitness 0 through the evaluation "
@@ -92,8 +95,10 @@ def main():
     o.seed = args.seed
     o.time_budget_s = args.budget
     o.reps = args.reps
+    if args.no_warm_start:
+        o.warm_start = 0
     os.makedirs(os.path.join(ROOT, "tuned", "logs"), exist_ok=True)
-    tag = "".join(f"_{kv.replace('=', '')}" for kv in args.fix)
+    tag = "".join(f"_{kv.replace('=', '')}" for kv in args.fix) + ("_nows" if args.no_warm_start else "")
     log = os.path.join(ROOT, "tuned", "logs", f"{args.config}{tag}_seed{args.seed}.json")
     o.log_path = log.encode()
     fixed = {kv.split("=")[0]: int(kv.split("=")[1]) for kv in args.fix}
