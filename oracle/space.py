@@ -148,7 +148,18 @@ def smem_bytes(kind: int, r: int, s: dict) -> int:
         return s["prefetch"] * rnd(e0[0] * e0[1]) + (s["bt"] - 1) * 2 * rnd(e1[0] * e1[1])
     P, NP = plane_geometry(kind, r, s)
     plane = -(-(P * 8) // 128) * 128
-    return (n_arrays(kind) * NP + (6 if r4ret_path(kind, s) else 0)) * plane
+    return ((n_arrays(kind) * NP + (6 if r4ret_path(kind, s) else 0)) * plane
+            + hyp_xprod_bytes(kind, r, s))
+
+
+def hyp_xprod_bytes(kind: int, r: int, s: dict) -> int:
+    """x-product planes of the TMEM hypterm kernel (round 2): two buffers of the 5 products
+    E^x_f over the tile and its (even) x-halo."""
+    if kind != HYPTERM or s["qstore"] != 2 or s["use_streaming"] != 2:
+        return 0
+    T = tiles(s)
+    b = 1 if s["sd"] == 3 else 2
+    return 2 * 5 * (-(-((T[0] + 2 * xr(r)) * T[b] * 8) // 128) * 128)
 
 
 def points_per_thread(s: dict) -> int:

@@ -2373,12 +2373,14 @@ __device__ __forceinline__ void kernel_star_tmem(const cst_kparams& P, double* s
 // Every in-plane derivative contributes  sum_{k=-R..R, k!=0} wd[k] E^d_f(p + k e_d)  to flux f,
 // wd[k] = -sign(k) dxinv_d a_|k| (the bank's ws tables, one per direction), E^d_f the
 // pointwise products of direction d.  Instead of loading a window per array and point, the
-// lanes walk the union of their windows one position at a time (six loads, five products,
-// five FMAs per position; few live registers):
-//  * along a (x): lanes 2i, 2i+1 share each 16-B chunk of the 2R+2 positions starting at the
-//    even element la - XR - (la & 1); a lane's weight at position j is wd[j - XR - (la & 1)],
-//    chosen by a select between two uniform constants;
-//  * along b each lane walks its own 2R rows.  (CST_HYP_HPAIR = 1, experiment: when a warp
+// lanes walk the union of their windows one position at a time:
+//  * along a (x): the products E^a_f are formed once per column into shared-memory product
+//    planes (hyp_prod_a, round 2; round 1 walked six inputs per position and formed the
+//    products per lane); lanes 2i, 2i+1 share each 16-B chunk of the 2R+2 positions starting
+//    at the even element la - XR - (la & 1); a lane's weight at position j is
+//    wd[j - XR - (la & 1)], chosen by a select between two uniform constants;
+//  * along b each lane walks its own 2R rows (six loads, five products, five FMAs per row;
+//    with two points stacked along b, the union of their rows).  (CST_HYP_HPAIR = 1, experiment: when a warp
 //    holds two b-rows (T_a = 16) both half-warps read the same row at a time, 2R+2 rows per
 //    pair, the weight selected by the row parity — measured slower: 3.85 vs 3.53 ms at
 //    512^3; the shared 8-byte loads of the two half-warps are not merged into one wavefront.)
@@ -2460,48 +2462,6 @@ constexpr int hyp_wx_slot(int j) {  // index into HypWx::w of walk position j, -
   return (k0 != 0 && k0 >= -R && k0 <= R && k1 != 0 && k1 >= -R && k1 <= R) ? n : -1;
 }
 
-// x-direction terms into A; the point's own cons1..4 and q4 into cen
-template <class LD>
-__device__ __forceinline__ void hyp_rows_a(const Ctx& C, const LD* ld, int la, int lb,
-                                           double (&A)[5], double (&cen)[5],
-                                           const HypWx* wx = nullptr) {
-  static_assert(XR == R, "even order");
-  const bool odd = la & 1;
-  const int e0 = la - XR - (int)odd;
-  static_for<0, R + 1>([&](auto CC) {
-    constexpr int c = decltype(CC)::value;
-    double2 v2[6];
-#pragma unroll
-    for (int m = 0; m < 4; ++m) v2[m] = ld[m].at2(e0 + 2 * c, lb);
-    v2[4] = ld[Q_A].at2(e0 + 2 * c, lb);
-    v2[5] = ld[7].at2(e0 + 2 * c, lb);
-    static_for<0, 2>([&](auto HH) {
-      constexpr int h = decltype(HH)::value, j = 2 * c + h;
-      double v[6];
-#pragma unroll
-      for (int m = 0; m < 6; ++m) v[m] = h ? v2[m].y : v2[m].x;
-      if constexpr (j == XR) {
-#pragma unroll
-        for (int m = 0; m < 4; ++m) cen[m] = v[m];
-        cen[4] = v[5];
-      } else if constexpr (j == XR + 1) {
-#pragma unroll
-        for (int m = 0; m < 4; ++m) cen[m] = odd ? v[m] : cen[m];
-        cen[4] = odd ? v[5] : cen[4];
-      }
-      double E[5];
-      hyp_e<DA>(v, E);
-      constexpr int ws_i = hyp_wx_slot(j);
-      if (ws_i >= 0 && wx != nullptr) {
-#pragma unroll
-        for (int f = 0; f < 5; ++f) A[f] = fma(wx->w[ws_i < 0 ? 0 : ws_i], E[f], A[f]);
-      } else {
-        hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A);
-      }
-    });
-  });
-}
-
 // b-direction terms into A
 template <class LD>
 __device__ __forceinline__ void hyp_rows_b(const Ctx& C, const LD* ld, int la, int lb,
@@ -2574,6 +2534,46 @@ __device__ __forceinline__ void hyp_rows_bn(const Ctx& C, const LD* ld, int la, 
 // terms T are computed from shared memory.  Slot of plane j = j mod R, rotated at run time.
 // Layout per point (20R columns): E slot s at 10 s, A slot s at 10 (R + s); 5 doubles each.
 // =============================================================================
+// x-direction product planes (the TMEM hypterm path, round 2): E^a_f of every column of the
+// tile and its x-halo is formed once per plane (own columns by their threads, the 2 XR halo
+// columns by spare threads) into a double-buffered shared-memory plane; the x-derivative then
+// reads 5 products per position instead of forming them from 6 inputs (the x-walk of
+// round-1 x row walk formed each product 2R times, once per point whose window holds it): 3.19 vs
+// 3.27 ms at 512^3 (4 interleaved rounds, profiles/r02/g34), 2 prefetch stages (the planes
+// take the smem of the third).
+constexpr bool XPROD = KIND == 3 && QTM;
+constexpr int XP_PITCH = TA + 2 * XR;                 // row pitch of a product plane
+constexpr int XP_SLOT = round_slot(XP_PITCH * TB);    // one product plane (elements)
+constexpr int XP_BUF = XPROD ? 2 * 5 * XP_SLOT : 0;  // two buffers of 5 products
+// D_a of the 5 fluxes from the product planes at (la, lb) into A (same weights and walk
+// as the round-1 x row walk: lanes 2i, 2i+1 share each 16-B chunk of the 2R+2 positions)
+__device__ __forceinline__ void hyp_prod_a(const Ctx& C, const double* pb, int la, int lb,
+                                           double (&A)[5], const HypWx* wx) {
+  const bool odd = la & 1;
+  const int e0 = la - XR - (int)odd;  // tile-local x of the first walk position
+  const double* row = pb + lb * XP_PITCH + XR + e0;
+  static_for<0, R + 1>([&](auto CC) {
+    constexpr int c = decltype(CC)::value;
+    double2 v2[5];
+#pragma unroll
+    for (int f = 0; f < 5; ++f)
+      v2[f] = *reinterpret_cast<const double2*>(row + f * XP_SLOT + 2 * c);
+    static_for<0, 2>([&](auto HH) {
+      constexpr int h = decltype(HH)::value, j = 2 * c + h;
+      double E[5];
+#pragma unroll
+      for (int f = 0; f < 5; ++f) E[f] = h ? v2[f].y : v2[f].x;
+      constexpr int ws_i = hyp_wx_slot(j);
+      if (ws_i >= 0 && wx != nullptr) {
+#pragma unroll
+        for (int f = 0; f < 5; ++f) A[f] = fma(wx->w[ws_i < 0 ? 0 : ws_i], E[f], A[f]);
+      } else {
+        hyp_acc<DA, j - XR, j - XR - 1>(C, odd, E, A);
+      }
+    });
+  });
+}
+
 template <int DUMMY>
 __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* smem) {
   static_assert(DUMMY != 0 || (KIND == 3 && STAGING == 3 && TS == 1 && NCA == 1 && CMB == 1 &&
@@ -2587,7 +2587,8 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
   const int tb = SZ ? thread_y() : thread_z();
   const int tid = threadIdx.x, warp = tid / 32;
   const int n_planes = (g.s_end - g.s_start) + 2 * R;
-  u64* bars = (u64*)(smem + NP * RSLOT);
+  double* pbuf = smem + NP * RSLOT;  // x-product planes (XPROD), 2 x 5 x XP_SLOT
+  u64* bars = (u64*)(smem + NP * RSLOT + XP_BUF);
   u32* tslot = (u32*)(bars + NP);  // spare mbarrier words (kernel_smem_bytes reserves 2 NP)
 
   int la[NCA], lb[NCB];
@@ -2653,38 +2654,67 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
         for (int ib = 0; ib < NCB; ++ib) issue_ring(ib);
       }
       {
+        static_assert(XPROD, "TMEM hypterm: x-product planes");
+        // own columns: centres and E^a into the product planes of this plane's buffer; the
+        // x-halo columns' E^a by the first 2 XR * TB threads; the b-terms; E^s.  Then the CTA
+        // barrier (products visible, ring slot read), the refill, and D_a from the products.
+        double* pb = pbuf + (j & 1) * 5 * XP_SLOT;
         double cen[NCB][5];
+        double Ab[NCB][5];
+#pragma unroll
+        for (int ib = 0; ib < NCB; ++ib) {
+#pragma unroll
+          for (int m = 0; m < 4; ++m) cen[ib][m] = ld[m].at(la[0], lb[ib]);
+          cen[ib][4] = ld[7].at(la[0], lb[ib]);
+          const double qs = ld[4 + DS].at(la[0], lb[ib]);
+          if (need_a) {
+            const double v[6] = {cen[ib][0], cen[ib][1], cen[ib][2], cen[ib][3],
+                                 ld[Q_A].at(la[0], lb[ib]), cen[ib][4]};
+            double Ea[5];
+            hyp_e<DA>(v, Ea);
+#pragma unroll
+            for (int f = 0; f < 5; ++f) pb[f * XP_SLOT + lb[ib] * XP_PITCH + XR + la[0]] = Ea[f];
+          }
+          const double vs[6] = {cen[ib][0], cen[ib][1], cen[ib][2], cen[ib][3], qs, cen[ib][4]};
+          hyp_e<DS>(vs, E[ib]);
+        }
         if (need_a) {
-          // separate x and b partial sums: two independent FMA chains per flux
-          double Ab[NCB][5];
+          for (int e = tid; e < 2 * XR * TB; e += NTHR) {
+            const int hc = e % (2 * XR), hr = e / (2 * XR);
+            const int hx = hc < XR ? hc - XR : TA + hc - XR;  // tile-local x of the column
+            double v[6];
+#pragma unroll
+            for (int m = 0; m < 4; ++m) v[m] = ld[m].at(hx, hr);
+            v[4] = ld[Q_A].at(hx, hr);
+            v[5] = ld[7].at(hx, hr);
+            double Ea[5];
+            hyp_e<DA>(v, Ea);
+#pragma unroll
+            for (int f = 0; f < 5; ++f) pb[f * XP_SLOT + hr * XP_PITCH + XR + hx] = Ea[f];
+          }
 #pragma unroll
           for (int ib = 0; ib < NCB; ++ib)
 #pragma unroll
             for (int f = 0; f < 5; ++f) A[ib][f] = Ab[ib][f] = 0.0;
-#pragma unroll
-          for (int ib = 0; ib < NCB; ++ib)
-            hyp_rows_a(C, ld, la[0], lb[ib], A[ib], cen[ib], CST_HYP_WXPRE ? &wxl : nullptr);
           if constexpr (NCB == 1 && HPAIR)
             hyp_rows_b(C, ld, la[0], lb[0], Ab[0]);
           else
             hyp_rows_bn<NCB>(C, ld, la[0], lb[0], Ab);
-#pragma unroll
-          for (int ib = 0; ib < NCB; ++ib)
-#pragma unroll
-            for (int f = 0; f < 5; ++f) A[ib][f] += Ab[ib][f];
-        } else {
+        }
+        __syncthreads();
+        if (tid == 0 && j + D < n_planes) {
+          const int sl = (j + D) % NP;
+          fence_proxy_async();
+          mbar_arrive_expect_tx(&bars[sl], TX_BYTES);
+          tma_plane(P, g, smem + sl * RSLOT, &bars[sl], p + D);
+        }
+        if (need_a) {
 #pragma unroll
           for (int ib = 0; ib < NCB; ++ib) {
+            hyp_prod_a(C, pb, la[0], lb[ib], A[ib], CST_HYP_WXPRE ? &wxl : nullptr);
 #pragma unroll
-            for (int m = 0; m < 4; ++m) cen[ib][m] = ld[m].at(la[0], lb[ib]);
-            cen[ib][4] = ld[7].at(la[0], lb[ib]);
+            for (int f = 0; f < 5; ++f) A[ib][f] += Ab[ib][f];
           }
-        }
-#pragma unroll
-        for (int ib = 0; ib < NCB; ++ib) {
-          const double v[6] = {cen[ib][0], cen[ib][1], cen[ib][2], cen[ib][3],
-                               ld[4 + DS].at(la[0], lb[ib]), cen[ib][4]};
-          hyp_e<DS>(v, E[ib]);
         }
       }
       // streamed-direction state, one point at a time (ring loaded after the in-plane terms)
@@ -2730,13 +2760,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 #endif
     tmem_wait_st();  // the next plane reads these slots (waiting at the next plane's ring
                      // fetch instead measured the same: 3.171 vs 3.170 ms, g25)
-    __syncthreads();
-    if (tid == 0 && j + D < n_planes) {
-      const int sl = (j + D) % NP;
-      fence_proxy_async();
-      mbar_arrive_expect_tx(&bars[sl], TX_BYTES);
-      tma_plane(P, g, smem + sl * RSLOT, &bars[sl], p + D);
-    }
+    // (the plane's CTA barrier and ring refill are mid-plane, after the product planes)
   }
   tmem_fence_before_sync();
   __syncthreads();

@@ -252,8 +252,8 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
   // register blocks; rhs4 the retimed column walk, 8x16 threads with two x-adjacent points
   // each, 64-plane blocks, 1-deep prefetch, coefficients in __constant__ (0.965 vs 1.095 ms
   // for the generic path at 320^3); hypterm 32x4 threads with two points
-  // stacked along y each, streamed state in TMEM, 3-deep ring, coefficients in __constant__
-  // (3.16-3.19 ms vs 3.53 ms for the best register-path setting at 512^3).
+  // stacked along y each, streamed state in TMEM, x-product planes with a 2-deep ring,
+  // coefficients in __constant__.
   const bool hyp = h->info.kind == CST_HYPTERM || h->info.kind == CST_RHS4;
   const bool hyp_tm = h->info.kind == CST_HYPTERM;
   const bool r4 = h->info.kind == CST_RHS4;
@@ -273,7 +273,7 @@ extern "C" cst_status cst_setting_default(const cst_stencil* h, cst_setting* s) 
   c.bt = 1;
   c.qstore = hyp_tm ? 2 : 1;
   if (hyp) c.use_constant = 2;
-  c.prefetch = h->info.kind == CST_BOX ? 2 : (r4 ? 1 : 3);
+  c.prefetch = (h->info.kind == CST_BOX || hyp_tm) ? 2 : (r4 ? 1 : 3);
   for (int tries = 0; tries < 12 && check_rules(h->info, to_tuple(c)); ++tries) {
     if (c.qstore == 2 && c.staging != 3) { c.qstore = 1; continue; }  // R15 needs TMA
     // shrink the tile until it fits the grid (coverage) and the thread floor

@@ -175,13 +175,24 @@ static void plane_geometry(int kind, int r, const Tuple& t, int64_t* P, int64_t*
     *NP = D * T[sd] + 2 * r;
 }
 
+// x-product planes of the TMEM hypterm kernel (hyp_prod_a in csrc/kernels/cst_kernels.cuh):
+// two buffers of 5 products over the tile and its x-halo
+static int64_t hyp_xprod_bytes(int kind, int r, const Tuple& t) {
+  if (kind != CST_HYPTERM || t[F_QS] != 2 || t[F_STREAM] != 2) return 0;
+  int64_t T[3];
+  tiles(t, T);
+  const int b = (t[F_SD] - 1) == 2 ? 1 : 2;
+  return 2 * 5 * rnd128((T[0] + 2 * xr_of(r)) * T[b] * 8);
+}
+
 int64_t model_smem_bytes(int kind, int r, const Tuple& t) {
   if (t[F_STAGING] == 1) return 0;
   if (t[F_BT] > 1) return tb_smem_bytes(r, t);
   int64_t P, NP;
   plane_geometry(kind, r, t, &P, &NP);
   const int64_t plane = (P * 8 + 127) / 128 * 128;
-  return (n_arrays(kind) * NP + (r4ret_path(kind, t) ? 6 : 0)) * plane;
+  return (n_arrays(kind) * NP + (r4ret_path(kind, t) ? 6 : 0)) * plane +
+         hyp_xprod_bytes(kind, r, t);
 }
 
 // Per-array halos of the hypterm TMA fast path (HTRIM in csrc/kernels/cst_kernels.cuh):
@@ -240,7 +251,7 @@ int64_t kernel_smem_bytes(int kind, int r, const Tuple& t) {
       stream_array_box(kind, r, t, a, &wa, &wb);
       slot += rnd128(wa * wb * 8);
     }
-    return NP * slot + bars;
+    return NP * slot + hyp_xprod_bytes(kind, r, t) + bars;
   }
   return n_arrays(kind) * NP * plane + bars;
 }
