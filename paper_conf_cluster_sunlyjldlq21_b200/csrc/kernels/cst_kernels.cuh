@@ -2679,6 +2679,8 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
           hyp_e<DS>(vs, E[ib]);
         }
         if (need_a) {
+          // x-halo columns of the product planes, one thread per column (splitting each
+          // column's products over two threads measured slower: 3.146 vs 3.105 ms, g38)
           for (int e = tid; e < 2 * XR * TB; e += NTHR) {
             const int hc = e % (2 * XR), hr = e / (2 * XR);
             const int hx = hc < XR ? hc - XR : TA + hc - XR;  // tile-local x of the column
