@@ -192,6 +192,27 @@ def test_rhs4_retimed_ragged(name, kw):
         H.assert_halo_untouched(L, got[o], np.full(L.numel, np.nan))
 
 
+@pytest.mark.parametrize("n,kw", [((20, 18, 3), dict(tb_x=8, tb_y=8, bm_x=2, sb=1, prefetch=1)),
+                                  ((20, 18, 5), dict(tb_x=8, tb_y=8, bm_x=2, sb=2, prefetch=4)),
+                                  ((21, 6, 17), dict(tb_x=16, tb_y=1, tb_z=8, sd=2, bm_x=1,
+                                                     sb=2, prefetch=2)),
+                                  ((17, 17, 9), dict(tb_x=8, tb_y=16, bm_x=2, sb=1, qstore=2,
+                                                   prefetch=1))],
+                         ids=["sb1-nz3", "sb2-pf4", "y-sb2-ragged", "tmem-sb1-ragged"])
+def test_rhs4_retimed_short_chunks(n, kw):
+    """Retimed rhs4 edge cases: chunks of 1-2 planes (every step is warm-up or drain but
+    one), a 3-plane grid, a ragged y-streamed grid, the TMEM queue at SB 1."""
+    kind, r = 4, 2
+    L = H.layout(n, r + 1)
+    c = H.coeffs(kind, r, "random", seed=21)
+    ins = H.inputs(kind, L, seed=23, poison_beyond=r)
+    _, want = H.oracle_outputs(kind, r, c, L, ins)
+    _, got = run_gpu(kind, r, c, L, ins, S(**kw))
+    for o in range(3):
+        H.assert_parity(L, got[o], want[o], f"{kw} out{o}")
+        H.assert_halo_untouched(L, got[o], np.full(L.numel, np.nan))
+
+
 def test_integer_polynomial_bit_exact():
     """Integer weights and integer data: FMA is exact, so GPU == oracle bit-for-bit."""
     r = 4
