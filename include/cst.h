@@ -95,7 +95,11 @@ typedef struct {
   int32_t uf[3];          /* loop unrolling factors */
   int32_t cm[3];          /* cyclic merging (points at stride TB_d*BM_d) */
   int32_t bm[3];          /* block merging (adjacent points) */
-  int32_t use_retiming;   /* 1 gather form, 2 retimed scatter accumulation */
+  int32_t use_retiming;   /* 1 gather form, 2 retimed scatter accumulation
+                           * Rule R16 (rhs4): 2 selects the retimed column walk (outer-s
+                           * products scattered to pending outputs, inner-s product planes;
+                           * DESIGN.md §4.5) and needs streaming with T_SD = 1, TMA staging,
+                           * bt = 1, CM = 1, BM_b = 1, BM_x <= 2. */
   int32_t prefetch;       /* 1 off, 2..4 pipeline stages in flight */
   int32_t bt;             /* temporal blocking degree {1,2,4}: sweeps fused per kernel
                            * pass (B200 extension, "more
@@ -109,7 +113,9 @@ typedef struct {
                            * R15: qstore = 2 needs the star or hypterm (hypterm: one point
                            * along x, BM_b <= 2, CM = 1), streaming with T_SD = 1, TMA
                            * staging, retiming, bt = 1, and ceil(threads/128) * points per
-                           * thread * (4r star, 20r hypterm) <= 512 TMEM columns. */
+                           * thread * (4r star, 20r hypterm) <= 512 TMEM columns; or rhs4's
+                           * retimed walk (R16), whose s-window queue then takes 10 (2r + 1)
+                           * columns per point. */
 } cst_setting;
 
 typedef struct cst_stencil cst_stencil;     /* opaque: JIT modules, TMA descriptors, space */
@@ -120,7 +126,7 @@ cst_status cst_stencil_create(const cst_stencil_desc* desc, const cst_grid* grid
                               cst_stencil** out);
 void cst_stencil_destroy(cst_stencil* h);
 
-/* Rules R1-R12, R14, R15 (explicit, implicit analytic resource rules, P:149-151,
+/* Rules R1-R12, R14-R16 (explicit, implicit analytic resource rules, P:149-151,
  * and the structural rules of the B200 extensions).
  * CST_OK if valid, else CST_E_CONSTRAINT with the rule in cst_last_error(). */
 cst_status cst_setting_check(const cst_stencil* h, const cst_setting* s);

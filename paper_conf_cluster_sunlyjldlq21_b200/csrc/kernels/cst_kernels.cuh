@@ -1509,14 +1509,18 @@ __device__ __forceinline__ void kernel_stream_generic(const cst_kparams& P, doub
 //     staged as three product planes in shared memory (own columns by their threads, the
 //     cross-shaped halo columns from the ring), then differenced along a / b;
 //   both derivatives in-plane: gathered from the ring plane as in the generic path.
-// The s-window of the own column (u1..u3, mu, lambda at planes c-2..c+2) is a register
-// queue (2.5-D blocking).  At step c the newest plane is c+2; output c-2 completes.
+// The s-window of the own column (u1..u3, mu, lambda at planes c-2..c+2): a register queue
+// of u1..u3 with mu / lambda from the ring (one point per thread; 2.5-D blocking), read
+// from the ring (two x-adjacent points per thread), or a tensor-memory queue (qstore = 2).
+// At step c the newest plane is c+2; output c-2 completes.
 // =============================================================================
 constexpr bool R4RET = KIND == 4 && STREAM && TS == 1 && RETIME;
 constexpr int R4NP = PF + 2 * R;                 // ring: planes c-2 .. c+2 + PF-1 ahead
 constexpr int R4NH = 2 * TB + 4 * (TA / 2);      // halo column pairs of the product planes
 // the two x-adjacent points of a BM_a = 2 thread in lockstep (every smem operand one 16-B
-// load for both); mu / lambda s-windows then come from the ring instead of registers
+// load for both); their s-windows come from the ring (a register queue spills them: 255
+// registers + 200 B of stack); one point per thread keeps u1..u3 in registers (166 registers,
+// 3 CTAs/SM; all five: 216 registers, 2 CTAs, 15 % slower).  Experiment hook: CST_R4Q.
 #ifndef CST_R4Q
 #define CST_R4Q (BMA == 1 ? 3 : 0)
 #endif
