@@ -2535,16 +2535,18 @@ __device__ __forceinline__ void hyp_rows_bn(const Ctx& C, const LD* ld, int la, 
 //   A_f(q)      = -T_a,f(q) - T_b,f(q) + sum_{k=-R..-1} ws[k] E_f(q+k)
 //   flux_f(q-R) = A_f(q-R) + sum_{k=1..R-1} ws[k] E_f(q-R+k) + ws[R] E_f(q)
 // Both sums read the same ring slots (planes q-R .. q-1), fetched while the in-plane
-// terms T are computed from shared memory.  Slot of plane j = j mod R, rotated at run time.
+// terms T are computed from shared memory (T_a from the x-product planes below, T_b by the
+// b row walk).  Slot of plane j = j mod R, rotated at run time.
 // Layout per point (20R columns): E slot s at 10 s, A slot s at 10 (R + s); 5 doubles each.
 // =============================================================================
 // x-direction product planes (the TMEM hypterm path, round 2): E^a_f of every column of the
 // tile and its x-halo is formed once per plane (own columns by their threads, the 2 XR halo
 // columns by spare threads) into a double-buffered shared-memory plane; the x-derivative then
-// reads 5 products per position instead of forming them from 6 inputs (the x-walk of
-// round-1 x row walk formed each product 2R times, once per point whose window holds it): 3.19 vs
-// 3.27 ms at 512^3 (4 interleaved rounds, profiles/r02/g34), 2 prefetch stages (the planes
-// take the smem of the third).
+// reads 5 products per position instead of forming them from 6 inputs (the round-1 x row
+// walk formed each product 2R times, once per point whose window holds it): 3.19 vs 3.27 ms
+// at 512^3 (4 interleaved rounds, profiles/r02/g34), 2 prefetch stages (the planes take the
+// smem of the third).  Per plane: own loads, E^x and E^s, halo E^x, b-walk -> CTA barrier
+// (products visible, ring slot read) -> TMA refill -> D_x from the planes -> TMEM ring.
 constexpr bool XPROD = KIND == 3 && QTM;
 constexpr int XP_PITCH = TA + 2 * XR;                 // row pitch of a product plane
 constexpr int XP_SLOT = round_slot(XP_PITCH * TB);    // one product plane (elements)
