@@ -711,7 +711,12 @@ def main():
         for _ in range(args.e2e_steps):
             C.cst_sweep_host(h, s, [hu.data_ptr()], [hv.data_ptr()], 1)
         el = (time.perf_counter() - t0) / args.e2e_steps
-        e2e = {"value": pts / el / 1e9, "unit": UNIT, "h2d_bytes_per_step": grid.numel * 8,
+        # cst_sweep_host uploads every padded plane and row but, per row, only the columns a
+        # kernel can read (interior + even x-halo), and reads back the interior
+        xh = min(grid.lead_x, grid.halo + (grid.halo & 1))
+        xw = min(grid.pitch_x - (grid.lead_x - xh), grid.nx + 2 * xh)
+        h2d = (grid.nz + 2 * grid.halo) * grid.pitch_y * xw * 8
+        e2e = {"value": pts / el / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": pts * 8, "ms_per_step": el * 1e3,
                "steps": args.e2e_steps, "api": "cst_sweep_host"}
 

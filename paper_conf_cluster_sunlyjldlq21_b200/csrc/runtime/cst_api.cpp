@@ -695,9 +695,11 @@ extern "C" cst_status cst_sweep_host(cst_stencil* h, const cst_setting* s,
       CST_CUDA(cudaStreamCreateWithFlags(&h->host_in_stream, cudaStreamNonBlocking));
       CST_CUDA(cudaStreamCreateWithFlags(&h->host_out_stream, cudaStreamNonBlocking));
     }
-    // 16 chunks: 28 ms for star25 512^3 vs 30 ms with 8 on B200 (PCIe ~55 GB/s per
-    // direction, ~45 GB/s each when both run; tools/e2e_probe.py)
-    const int64_t nc = std::max<int64_t>(1, std::min<int64_t>(16, G.nz / std::max(16, 4 * h->info.r)));
+    // up to 32 chunks of >= max(8, 4r) planes: star25 512^3 25.5 ms vs 26.5 ms with 16 and
+    // 30 ms with 8 on B200 (PCIe ~55 GB/s per direction, ~45 GB/s each when both run;
+    // tools/e2e_probe.py, profiles/r02/g51_host_chunks.txt)
+    const int64_t nc = std::max<int64_t>(
+        1, std::min<int64_t>(32, G.nz / std::max<int64_t>(8, 4 * h->info.r)));
     std::vector<cudaEvent_t> evs;
     auto event = [&](cudaStream_t st_) -> cudaEvent_t {
       cudaEvent_t e;
@@ -708,15 +710,29 @@ extern "C" cst_status cst_sweep_host(cst_stencil* h, const cst_setting* s,
     };
     int64_t copied = 0;  // padded planes already on the device
     const int64_t planes = G.nz + 2 * (int64_t)G.halo;
+    // per row only the columns a kernel can read: the interior and an x-halo of halo rounded
+    // up to even (the kernels' 16-B aligned TMA boxes), not the row padding (4.4 % of a
+    // star25 512^3 row: 520 of 544 doubles)
+    const int64_t xh = std::min<int64_t>(G.lead_x, G.halo + (G.halo & 1));
+    const int64_t xw = std::min<int64_t>(G.pitch_x - (G.lead_x - xh), G.nx + 2 * xh);
+    auto copy_in = [&](const double* hsrc, double* ddst, int64_t p0, int64_t p1) -> cst_status {
+      cudaMemcpy3DParms q = {};
+      const int64_t first = p0 * plane + (G.lead_x - xh);
+      q.srcPtr = make_cudaPitchedPtr((void*)(hsrc + first), G.pitch_x * 8, xw * 8, G.pitch_y);
+      q.dstPtr = make_cudaPitchedPtr((void*)(ddst + first), G.pitch_x * 8, xw * 8, G.pitch_y);
+      q.extent = make_cudaExtent(xw * 8, G.pitch_y, p1 - p0);
+      q.kind = cudaMemcpyHostToDevice;
+      CST_CUDA(cudaMemcpy3DAsync(&q, h->host_in_stream));
+      return CST_OK;
+    };
     h->last_launches = 0;
     st = CST_OK;
     for (int64_t k = 0; k < nc && st == CST_OK; ++k) {
       const int64_t z0 = k * G.nz / nc, z1 = (k + 1) * G.nz / nc;
       const int64_t need = k == nc - 1 ? planes : std::min(planes, z1 + G.halo + h->info.r);
-      for (int a = 0; a < nin && need > copied; ++a)
-        CST_CUDA(cudaMemcpyAsync(h->dev_bufs[a] + copied * plane, in[a] + copied * plane,
-                                 (size_t)(need - copied) * plane * 8, cudaMemcpyHostToDevice,
-                                 h->host_in_stream));
+      for (int a = 0; a < nin && need > copied && st == CST_OK; ++a)
+        st = copy_in(in[a], h->dev_bufs[a], copied, need);
+      if (st != CST_OK) break;
       copied = std::max(copied, need);
       CST_CUDA(cudaStreamWaitEvent(sm, event(h->host_in_stream), 0));
       st = cst_launch_range(h, &s1, din, dout, z0, z1 - z0, sm);

@@ -276,6 +276,34 @@ def test_host_path_matches_device_path():
     H.assert_halo_untouched(L, got, np.full(L.numel, np.nan))
 
 
+@pytest.mark.parametrize("kind,r,n", [(3, 4, (40, 24, 36)), (4, 2, (37, 22, 40)), (1, 3, (45, 30, 50))],
+                         ids=["hypterm", "rhs4", "star-r3"])
+def test_host_path_multi_input_poisoned_padding(kind, r, n):
+    """cst_sweep_host uploads per row only the columns a kernel can read (interior + even
+    x-halo), not the row padding: NaN in everything beyond the radius (the outer halo ring
+    and the row padding) of the host inputs cannot reach an output; multi-input kinds, and an
+    odd radius (x-halo rounded up to even)."""
+    L = H.layout(n, r + 1)
+    c = H.coeffs(kind, r, "random", seed=kind + 40)
+    ins = H.inputs(kind, L, seed=41, poison_beyond=r)
+    for b in ins:  # poison the row padding too
+        v = b.reshape(L.nz + 2 * L.halo, L.ny + 2 * L.halo, L.pitch_x)
+        v[:, :, :L.lead_x - L.halo] = np.nan
+        v[:, :, L.lead_x + L.nx + L.halo:] = np.nan
+    _, want = H.oracle_outputs(kind, r, c, L, ins)
+    g = C.cst_grid(L.nx, L.ny, L.nz, L.halo, L.lead_x, L.pitch_x, L.pitch_y)
+    h = C.cst_stencil_create(kind, r, list(c), g)
+    s = C.cst_setting_default(h)
+    hin = [torch.from_numpy(b.copy()).pin_memory() for b in ins]
+    hout = [torch.full((L.numel,), float("nan"), dtype=torch.float64).pin_memory()
+            for _ in range(ost.N_OUT[kind])]
+    C.cst_sweep_host(h, s, [t.data_ptr() for t in hin], [t.data_ptr() for t in hout], 1)
+    C.cst_stencil_destroy(h)
+    for o in range(ost.N_OUT[kind]):
+        H.assert_parity(L, hout[o].numpy(), want[o], f"host out{o}")
+        H.assert_halo_untouched(L, hout[o].numpy(), np.full(L.numel, np.nan))
+
+
 def test_invalid_arguments_on_gpu():
     L = H.layout((16, 16, 16), 2)
     g = C.cst_grid(L.nx, L.ny, L.nz, L.halo, L.lead_x, L.pitch_x, L.pitch_y)

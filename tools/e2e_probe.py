@@ -1,6 +1,6 @@
 """Host-path probe: pinned H2D / D2H bandwidth alone and concurrent (torch copies), then
 cst_sweep_host of the star25 512^3 bench workload (one step; profiles/r02/g08_e2e_probe.jsonl
-has the chunk-count sweep that set cst_sweep_host's 16 pipeline chunks)."""
+and g51_host_chunks.txt have the chunk-count sweeps that set cst_sweep_host's 32 pipeline chunks)."""
 import json, os, sys, time
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
