@@ -2660,7 +2660,7 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
         for (int ib = 0; ib < NCB; ++ib) issue_ring(ib);
       }
       {
-        static_assert(XPROD, "TMEM hypterm: x-product planes");
+        static_assert(DUMMY != 0 || XPROD, "TMEM hypterm: x-product planes");
         // own columns: centres and E^a into the product planes of this plane's buffer; the
         // x-halo columns' E^a by the first 2 XR * TB threads; the b-terms; E^s.  Then the CTA
         // barrier (products visible, ring slot read), the refill, and D_a from the products.
