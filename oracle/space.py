@@ -32,7 +32,8 @@ streaming on.  Ours (Q15): R4 prod TB >= 32; R5 T_d = TB_d*BM_d*CM_d <= E_d (E_d
 E_SD = SB when streaming); R6 UF_d <= trip_d, the trip count of the loop the kernel path
 unrolls along d (uf_trip; 1 where there is none); R7 prod(BM*CM) <= 16; R8 streaming =>
 SD != 1; R9 prefetch > 1 => streaming with staging (nothing to prefetch into otherwise);
-R10 modelled smem <= SMEM_LIMIT; R11 modelled registers <= 255; R12 TMA box: T_x even and
+R10 modelled smem <= SMEM_LIMIT; R11 modelled registers <= 255; R12 smem staging (TMA or ld/st):
+T_x even (16-B aligned rows; round 2 extended it to ld/st staging); TMA box: T_x even and
 every box extent <= 256; R14 bt > 1 only for the temporally blocked path: star / box,
 streaming along z with T_SD = 1, TMA staging, retimed accumulators, no cyclic merging,
 BM_x, BM_y <= 2, every UF = 1 (reading Q23); R15 qstore = 2 only for the
@@ -311,6 +312,8 @@ def check(kind: int, r: int, M, s: dict):
     if est_regs(kind, r, s) > REG_LIMIT:
         return "R11"
     if s["staging"] == 3 and not tma_ok(r, s):
+        return "R12"
+    if s["staging"] == 2 and T[0] % 2:       # ld/st rows are read as 16-B pairs as well
         return "R12"
     return None
 

@@ -2807,6 +2807,9 @@ __device__ __forceinline__ void kernel_hyp_tmem(const cst_kparams& P, double* sm
 #else
 #define CST_LB __launch_bounds__(CST_TBX * CST_TBY * CST_TBZ)
 #endif
+// R12: every smem-staged row is read as 16-B pairs somewhere (x windows, walks), so its
+// length T_x + 2 XR must be even (a 1 x 32 ld/st tile faulted with a misaligned address)
+static_assert(STAGING == 1 || TX % 2 == 0, "R12: smem staging needs an even tile extent T_x");
 extern "C" __global__ void CST_LB cst_kernel(const __grid_constant__ cst_kparams P) {
   extern __shared__ __align__(128) double cst_smem[];
   if constexpr (BT > 1) {

@@ -383,6 +383,8 @@ const char* check_rules(const StencilInfo& st, const Tuple& t) {
   if (model_smem_bytes(st.kind, st.r, t) > SMEM_LIMIT) return "R10";
   if (model_regs(st.kind, st.r, t) > REG_LIMIT) return "R11";
   if (t[F_STAGING] == 3 && !tma_ok(st.r, t)) return "R12";
+  // ld/st staging reads its rows as 16-B pairs too: the smem row (T_x + 2 XR) must be even
+  if (t[F_STAGING] == 2 && T[0] % 2) return "R12";
   return nullptr;
 }
 

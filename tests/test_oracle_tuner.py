@@ -188,6 +188,11 @@ def test_space_rules_spot_checks():
     assert S.check(1, 4, M, dict(base, tb_x=128, tb_y=1)) is None
     assert S.check(1, 4, M, dict(base, tb_x=256, tb_y=1)) == "R12"
     assert S.check(1, 4, M, dict(base, tb_x=32, tb_y=1, bm_x=8)) == "R12"
+    # ld/st staging: rows read as 16-B pairs need an even T_x (a 1 x 32 ld/st hypterm tile
+    # faulted with a misaligned shared load on B200)
+    assert S.check(3, 4, M, dict(base, tb_x=1, tb_y=32, staging=2, prefetch=1, sb=16)) == "R12"
+    assert S.check(1, 4, M, dict(base, tb_x=1, tb_y=32, staging=2)) == "R12"
+    assert S.check(1, 4, M, dict(base, tb_x=1, tb_y=32, staging=1, prefetch=1)) is None
     # temporal blocking (field 20): R14 structure, models by hand
     tb = dict(base, bm_x=2, bm_y=2, bt=2)
     assert S.check(2, 1, M, tb) is None
